@@ -1,0 +1,288 @@
+"""Pins for the CPU oracle (``-m "not gpu"``).
+
+Each test checks ``oracle/`` against something other than itself: central
+finite differences, torch CPU autograd, the closed form of a linear stack,
+the paper's invariants (reordering dW changes nothing; §5.1: the DP
+average is the full-batch gradient / N), torch's bf16 cast, and the worked
+examples / pseudocode printed in the paper (tests/golden/*.json).
+"""
+import itertools
+import json
+import os
+import random
+
+import numpy as np
+import pytest
+import torch
+
+from oracle import layers as O
+from oracle import schedule as S
+from oracle import unit_sim as U
+from paper_conf_eurosys_ohlks22_b200 import synth
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _tiny(dims=(8, 16, 12, 8), acts=("gelu", "relu", "id"), M=5, seed=7, dtype="fp64"):
+    rng = np.random.default_rng(seed)
+    W = [rng.standard_normal((dims[i], dims[i + 1])) / np.sqrt(dims[i]) for i in range(len(acts))]
+    b = [0.1 * rng.standard_normal(dims[i + 1]) for i in range(len(acts))]
+    X = rng.standard_normal((M, dims[0]))
+    dY = rng.standard_normal((M, dims[-1]))
+    return list(dims), list(acts), W, b, X, dY
+
+
+# ------------------------------------------------------- finite differences
+def test_activation_derivatives_match_central_fd():
+    z = np.linspace(-4, 4, 801)
+    z = z[np.abs(z) > 1e-3]                       # relu kink excluded
+    h = 1e-6
+    for a in O.ACTS:
+        fd = (O.act_fwd(a, z + h) - O.act_fwd(a, z - h)) / (2 * h)
+        assert np.max(np.abs(fd - O.act_grad(a, z))) < 1e-8, a
+    # relu'(0) = 0 following PyTorch (reading in DESIGN.md)
+    assert O.act_grad("relu", np.array([0.0]))[0] == 0.0
+    # gelu(z) = z * Phi(z): spot values from the normal CDF
+    assert abs(O.act_fwd("gelu", np.array([1.0]))[0] - 0.8413447460685429) < 1e-12
+    assert abs(O.act_fwd("gelu", np.array([-1.0]))[0] + 0.15865525393145707) < 1e-12
+
+
+def test_backward_matches_central_finite_differences():
+    dims, acts, W, b, X, dY = _tiny()
+    L = len(acts)
+    st = O.forward(X, W, b, acts)
+    bs = O.run_backward(S.in_order(L, need_input_grad=True), st, dY, W, acts)
+    h = 1e-6
+
+    def loss(W_, b_, X_):
+        return O.loss_surrogate(O.forward(X_, W_, b_, acts).X[L], dY)
+
+    worst = 0.0
+    for i in range(L):
+        fd = np.zeros_like(W[i])
+        for idx in itertools.product(*map(range, W[i].shape)):
+            Wp = [w.copy() for w in W]; Wm = [w.copy() for w in W]
+            Wp[i][idx] += h; Wm[i][idx] -= h
+            fd[idx] = (loss(Wp, b, X) - loss(Wm, b, X)) / (2 * h)
+        worst = max(worst, O.rel_fro(bs.dW[i + 1], fd))
+        fdb = np.zeros_like(b[i])
+        for j in range(b[i].size):
+            bp = [v.copy() for v in b]; bm = [v.copy() for v in b]
+            bp[i][j] += h; bm[i][j] -= h
+            fdb[j] = (loss(W, bp, X) - loss(W, bm, X)) / (2 * h)
+        worst = max(worst, O.rel_fro(bs.db[i + 1], fdb))
+    fdx = np.zeros_like(X)
+    for idx in itertools.product(*map(range, X.shape)):
+        Xp = X.copy(); Xm = X.copy(); Xp[idx] += h; Xm[idx] -= h
+        fdx[idx] = (loss(W, b, Xp) - loss(W, b, Xm)) / (2 * h)
+    worst = max(worst, O.rel_fro(bs.dX, fdx))
+    assert worst < 1e-6, worst
+
+
+# ---------------------------------------------------------- torch autograd
+@pytest.mark.parametrize("acts", [("gelu", "relu", "id"), ("id", "gelu", "gelu"), ("relu", "relu", "relu")])
+def test_backward_matches_torch_autograd_fp64(acts):
+    dims, acts, W, b, X, dY = _tiny(dims=(16, 24, 8, 12), acts=acts, M=9, seed=11)
+    L = len(acts)
+    st = O.forward(X, W, b, acts)
+    bs = O.run_backward(S.reverse_first_k(L, 2, need_input_grad=True), st, dY, W, acts)
+    tW = [torch.tensor(w, requires_grad=True) for w in W]
+    tb = [torch.tensor(v, requires_grad=True) for v in b]
+    tX = torch.tensor(X, requires_grad=True)
+    h = tX
+    fn = {"id": lambda z: z, "relu": torch.relu,
+          "gelu": lambda z: torch.nn.functional.gelu(z, approximate="none")}
+    for i in range(L):
+        h = fn[acts[i]](h @ tW[i] + tb[i])
+    (h * torch.tensor(dY)).sum().backward()
+    for i in range(L):
+        assert np.allclose(bs.dW[i + 1], tW[i].grad.numpy(), rtol=1e-12, atol=1e-12)
+        assert np.allclose(bs.db[i + 1], tb[i].grad.numpy(), rtol=1e-12, atol=1e-12)
+    assert np.allclose(bs.dX, tX.grad.numpy(), rtol=1e-12, atol=1e-12)
+    assert np.allclose(st.X[L], h.detach().numpy(), rtol=1e-12, atol=1e-12)
+
+
+def test_linear_stack_closed_form():
+    """All-identity stack: Y = X P + c with P = W_1 ... W_L, so
+    dX = dY P^T and dW_1 = X^T dY (W_2 ... W_L)^T, db_L = 1^T dY."""
+    dims, acts, W, b, X, dY = _tiny(dims=(6, 10, 7, 5), acts=("id", "id", "id"), M=4, seed=3)
+    st = O.forward(X, W, b, acts)
+    bs = O.run_backward(S.in_order(3, need_input_grad=True), st, dY, W, acts)
+    P = W[0] @ W[1] @ W[2]
+    assert np.allclose(bs.dX, dY @ P.T, rtol=1e-12, atol=1e-12)
+    assert np.allclose(bs.dW[1], X.T @ (dY @ (W[1] @ W[2]).T), rtol=1e-12, atol=1e-12)
+    assert np.allclose(bs.db[3], dY.sum(axis=0), rtol=1e-12, atol=1e-12)
+    assert np.allclose(bs.db[1], (dY @ (W[1] @ W[2]).T).sum(axis=0), rtol=1e-12, atol=1e-12)
+
+
+# -------------------------------------------------- ordering invariance
+def _random_topo_order(L, rng, need_input_grad):
+    have, D, pending = {L}, [], {+i for i in range(2, L + 1)} | {-i for i in range(1, L + 1)}
+    if need_input_grad:
+        pending.add(+1)
+    while pending:
+        ready = sorted(op for op in pending if abs(op) in have)
+        op = rng.choice(ready)
+        D.append(op); pending.remove(op)
+        if op > 1:
+            have.add(op - 1)
+    return D
+
+
+@pytest.mark.parametrize("dtype", ["fp64", "bf16"])
+def test_every_schedule_gives_bit_identical_gradients(dtype):
+    dims = (16, 32, 24, 16, 8, 16)
+    acts = ("gelu", "relu", "id", "gelu", "id")
+    L = len(acts)
+    W, b = synth.weights(dims, acts, "bf16" if dtype == "bf16" else "fp32")
+    X = synth.x_shard(7, dims[0], 0, "bf16")
+    dY = synth.dy_shard(7, dims[-1], 0, "bf16")
+    st = O.forward(X, W, b, acts, dtype)
+    ref = O.run_backward(S.in_order(L, True), st, dY, W, acts, dtype)
+    orders = []
+    for k in range(L + 2):
+        for wl in ("paper", "critical_first"):
+            orders.append(S.reverse_first_k(L, k, True, wl))
+    rng = random.Random(5)
+    orders += [_random_topo_order(L, rng, True) for _ in range(40)]
+    for D in orders:
+        assert S.is_valid_order(D, L, True)
+        bs = O.run_backward(D, st, dY, W, acts, dtype)
+        for i in range(1, L + 1):
+            assert np.array_equal(bs.dW[i], ref.dW[i]) and np.array_equal(bs.db[i], ref.db[i])
+        assert np.array_equal(bs.dX, ref.dX)
+
+
+def test_invalid_schedule_is_rejected():
+    dims, acts, W, b, X, dY = _tiny()
+    st = O.forward(X, W, b, acts)
+    with pytest.raises(RuntimeError):
+        O.run_backward([-1, 3, 2, -2, -3], st, dY, W, acts)      # dW_1 before G_1 exists
+    with pytest.raises(RuntimeError):
+        O.run_backward([3, 2, -2, -3], st, dY, W, acts)          # dW_1 missing
+    assert not S.is_valid_order([2, 3, -3, -2, -1], 3)
+
+
+# ------------------------------------------------------ DP averaging (§5.1)
+def test_dp_average_equals_full_batch_gradient():
+    dims, acts = (12, 20, 16, 12), ("gelu", "relu", "id")
+    L = 3
+    W, b = synth.weights(dims, acts, "fp32")
+    N, M = 4, 6
+    Xs = [synth.x_shard(M, dims[0], r, "fp32") for r in range(N)]
+    dYs = [synth.dy_shard(M, dims[-1], r, "fp32") for r in range(N)]
+    D = S.reverse_first_k(L, 2)
+    res = O.dp_step(Xs, dYs, W, b, acts, D, "fp64")
+    full = O.dp_step([np.concatenate(Xs)], [np.concatenate(dYs)], W, b, acts, D, "fp64")
+    for i in range(L):
+        assert np.allclose(res.gW[i], full.gW[i] / N, rtol=1e-12, atol=1e-13)
+        assert np.allclose(res.gb[i], full.gb[i] / N, rtol=1e-12, atol=1e-13)
+
+
+def test_power_of_two_prescale_is_exact_in_bf16():
+    """Reading Q9: scaling by 1/N (N in 1,2,4,8) before bf16 rounding equals
+    rounding then scaling, bit for bit (no subnormals in range)."""
+    x = np.random.default_rng(0).standard_normal(100_000) * 10.0
+    for N in (1, 2, 4, 8):
+        assert np.array_equal(O.round_bf16(x * (1.0 / N)), O.round_bf16(x) * (1.0 / N))
+
+
+# ------------------------------------------------------------ bf16 rounding
+def test_round_bf16_matches_torch_cast():
+    rng = np.random.default_rng(1)
+    x = np.concatenate([
+        rng.standard_normal(500_000).astype(np.float32),
+        (rng.standard_normal(200_000) * 1e-38).astype(np.float32),       # subnormals
+        (rng.standard_normal(200_000) * 1e30).astype(np.float32),
+        np.array([0.0, -0.0, 1.0, 1.00390625, 1.01171875, 3.3895314e38, -3.3895314e38,
+                  np.inf, -np.inf], dtype=np.float32),
+    ])
+    # exact ties: bf16 midpoints
+    mids = (np.arange(1, 20000, dtype=np.uint32) << np.uint32(15)) | np.uint32(0x3F800000)
+    x = np.concatenate([x, mids.view(np.float32)]).astype(np.float64)
+    ours = O.round_bf16(x)
+    ref = torch.from_numpy(x.astype(np.float32)).to(torch.bfloat16).to(torch.float64).numpy()
+    assert np.array_equal(ours, ref)
+    assert np.isnan(O.round_bf16(np.array([np.nan])))[0]
+    # the shared input generator's rounding agrees too
+    assert np.array_equal(synth.to_storage(x, "bf16"), ref)
+
+
+def test_bf16_mode_stores_only_bf16_values_and_tracks_fp64():
+    dims, acts = (64, 128, 64, 64), ("gelu", "id", "gelu")   # ReLU sign flips are O(1)
+    W, b = synth.weights(dims, acts, "bf16")
+    X = synth.x_shard(32, 64, 0, "bf16")
+    dY = synth.dy_shard(32, 64, 0, "bf16")
+    D = S.reverse_first_k(3, 3)
+    st = O.forward(X, W, b, acts, "bf16")
+    bs = O.run_backward(D, st, dY, W, acts, "bf16")
+    for t in st.X + st.Z + list(bs.G.values()):
+        assert np.array_equal(t, O.round_bf16(t))
+    st64 = O.forward(X, W, b, acts, "fp64")
+    bs64 = O.run_backward(D, st64, dY, W, acts, "fp64")
+    for i in range(1, 4):
+        assert O.rel_fro(bs.dW[i], bs64.dW[i]) < 2e-2
+        assert O.rel_fro(bs.dW[i], bs64.dW[i]) > 0.0     # rounding really happens
+
+
+# ---------------------------------------------- Algorithm 2
+def test_alg2_sequences_match_hand_expanded_pseudocode():
+    gold = json.load(open(os.path.join(GOLD, "alg2_sequences.json")))
+    for c in gold["cases"]:
+        k = S.clamp_k(c["k"], c["L"])
+        if "k_clamped" in c:
+            assert k == c["k_clamped"]
+        D = S.reverse_first_k(c["L"], k, c["need_input_grad"], c["within_layer"])
+        assert D == c["D"], c
+        assert S.is_valid_order(D, c["L"], c["need_input_grad"])
+
+
+def test_alg2_prose_k3_and_k0():
+    # with k = 3, dW_2 and dW_3 follow dW_1, in that order, at the end.
+    D = S.reverse_first_k(5, 3)
+    assert D[-3:] == [-1, -2, -3]
+    # k = 0 is conventional backprop (every dW_i right after layer i's dO).
+    assert [abs(x) for x in S.reverse_first_k(8, 0)] == [8, 8, 7, 7, 6, 6, 5, 5, 4, 4, 3, 3, 2, 2, 1]
+    with pytest.raises(ValueError):
+        S.reverse_first_k(5, -1)
+
+
+def test_max_k_behaviour_unpinned():
+    """PARITY UNPINNED (garbled formula, no example): behavioural checks only."""
+    m_dO = [10.0] * 6
+    m_dW = [5.0] * 6
+    assert S.max_k(100.0, m_dO, m_dW, 0) == 6             # unlimited
+    ks = [S.max_k(100.0, m_dO, m_dW, mx) for mx in (1, 45, 60, 75, 200)]
+    assert ks == sorted(ks)                                # monotone in MXM
+    assert ks[0] == 0 and ks[-1] == 6
+    assert S.clamp_k(4, 6, 100.0, m_dO, m_dW, 45) == min(4, S.max_k(100.0, m_dO, m_dW, 45))
+
+
+def test_k_search_finds_peak_of_concave_curves_unpinned():
+    """PARITY UNPINNED (P:212-214 prose only): on concave curves the search
+    returns the argmax, visiting far fewer than L+1 points for large L."""
+    for L, peak in [(144, 37), (144, 0), (144, 143), (72, 50), (10, 4), (5, 3)]:
+        visited = []
+        k = S.search_k(L, lambda kk: -(kk - peak) ** 2, visited)
+        assert k == peak, (L, peak, k)
+        if L >= 72:
+            assert len(visited) < L // 2
+
+
+# ---------------------------------------------- worked examples (simulator)
+def test_fig5_cross_layer_mp_unit_counts():
+    g = json.load(open(os.path.join(GOLD, "worked_examples.json")))["fig5_cross_layer_mp"]
+    assert U.mp_iteration(g["L"], g["n_gpu"], "contiguous", False) == g["conventional"]
+    assert U.mp_iteration(g["L"], g["n_gpu"], "contiguous", True) == g["fast_forwarding"]
+    assert U.mp_iteration(g["L"], g["n_gpu"], "modulo", True) == g["modulo"]
+
+
+def test_fig4_data_parallel_unit_counts():
+    g = json.load(open(os.path.join(GOLD, "worked_examples.json")))["fig4_data_parallel"]
+    L, c = g["L"], g["sync_cost"]
+    assert U.dp_iteration(L, S.in_order(L), c, "fifo") == g["conventional_fifo"]
+    assert U.dp_iteration(L, S.in_order(L), c, "preemptive") == g["prioritised_comm"]
+    assert U.dp_iteration(L, S.reverse_first_k(L, 3), c, "preemptive") == g["reverse_first_k3"]
+    t = {k: U.dp_iteration(L, S.reverse_first_k(L, k), c, "preemptive") for k in range(L + 1)}
+    best = min(t.values())
+    assert sorted(k for k, v in t.items() if v == best) == g["optimal_k"]
