@@ -1,0 +1,224 @@
+/*
+ * ooo.h -- C ABI of the B200-native out-of-order backprop (ooo backprop)
+ *          data-parallel hot path.
+ *
+ * Paper: H. Oh, J. Lee, H. Kim, J. Seo, "Out-Of-Order BackProp: An Effective
+ * Scheduling Technique for Deep Learning", EuroSys'22.  "P:N" = line N of the
+ * paper text, followed by the section it is in.
+ *
+ * What one iteration is (§2, problem statement P:81-95): starting from the
+ * loss gradient dO_{L+1} at time 0, the backward ops of every layer -- the
+ * output-gradient op dO_i and the weight-gradient op dW_i -- then the
+ * gradient synchronisation S[dW_i] of every layer (data parallelism, §5.1
+ * P:176-180), and finally the next iteration's forward F_1..F_L, where
+ * F_i may start only after S[dW_i] (T(F_i) >= T(S[dW_i]) + S[dW_i]).
+ * dW_i feeds no other gradient (§3), so it may run out of layer order;
+ * ooo_backward(schedule = OOO_SCHED_FIRST_K, k) issues the dW ops in the
+ * order of Algorithm 2 "Reverse First-K Scheduling".
+ *
+ * Model: a stack of L dense (Linear) layers, layer i = 1..L:
+ *     Z_i = X_i W_i + 1 b_i^T,      X_{i+1} = act_i(Z_i)
+ *     W_i: d_{i-1} x d_i, row-major (d_i contiguous);  b_i: d_i
+ *     X_i, Z_i, dZ_i: M x d, row-major (d contiguous), M = tokens per rank.
+ *   Backward (dY = dLoss/dX_{L+1}, given by the caller; reading Q8):
+ *     dZ_L     = dY (.) act_L'(Z_L)                               (seed)
+ *     dO_i:  dZ_{i-1} = (dZ_i W_i^T) (.) act_{i-1}'(Z_{i-1})      (i >= 2)
+ *            dX       =  dZ_1 W_1^T       (i == 1, only if need_input_grad)
+ *     dW_i:  dW_i = X_i^T dZ_i,  db_i = 1^T dZ_i
+ *   Data parallel (§5.1): every rank holds the same W, b and its own M-token
+ *   shard; the library returns the rank average (1/N) sum_r dW_i^(r)
+ *   (reading Q9: pre-scaled by 1/N, then an in-place NCCL sum all-reduce per
+ *   bucket, issued in the order the dW ops complete).
+ *
+ * Precision (reading Q10): OOO_BF16 = bf16 storage of X, Z, dZ, W, b and
+ * gradients, fp32 accumulation (tcgen05 tensor cores), bf16 RNE rounding at
+ * every store; OOO_FP32 = fp32 everywhere (exact fp32 FFMA, no TF32).
+ *
+ * Memory ownership: every device buffer is allocated by the caller (e.g. a
+ * torch tensor); the library never allocates device memory.  The stack owns
+ * host objects only: CUDA streams and events, TMA descriptors, the NCCL
+ * communicator and captured graphs.
+ *
+ * Stream semantics: every call is stream-ordered after prior work on the
+ * caller's stream `st`.  ooo_backward returns with work still in flight on
+ * the library's internal streams (hi priority: dO ops; lo priority: dW ops;
+ * comm: all-reduces).  The next ooo_forward joins it per layer (F_i waits for
+ * layer i's synchronised gradient) and finally joins everything into
+ * `st`; ooo_join joins it explicitly.  Gradients in `grads` are valid only
+ * after one of those.  No call synchronises the host or allocates, so the
+ * sequence ooo_backward; ooo_forward is CUDA-graph capturable on `st`.
+ *
+ * Errors: argument/shape errors are detected before anything is enqueued;
+ * the call returns a non-zero ooo_status and ooo_last_error() describes it.
+ * Asynchronous CUDA / NCCL failures surface as OOO_ERR_CUDA / OOO_ERR_NCCL
+ * from a later call (ooo_join polls ncclCommGetAsyncError).  No C++
+ * exception crosses this ABI.  Threading: one stack is used by one host
+ * thread at a time; ooo_last_error is thread-local.
+ *
+ * Collective rule: with world_size > 1 every rank must call ooo_backward with
+ * the same schedule (D and the NCCL issue order depend only on (L, k));
+ * a mismatch is undefined behaviour (NCCL hang).
+ */
+#ifndef OOO_H_
+#define OOO_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define OOO_ABI_VERSION 1
+#define OOO_UNIQUE_ID_BYTES 128
+
+typedef struct ooo_stack ooo_stack;   /* opaque */
+typedef struct ooo_graph ooo_graph;   /* opaque, a captured [backward; forward] step */
+
+typedef enum {
+  OOO_OK = 0,
+  OOO_ERR_INVALID_ARGUMENT = 1,
+  OOO_ERR_UNSUPPORTED = 2,
+  OOO_ERR_CUDA = 3,
+  OOO_ERR_NCCL = 4,
+  OOO_ERR_STATE = 5
+} ooo_status;
+
+typedef enum { OOO_BF16 = 0, OOO_FP32 = 1 } ooo_dtype;
+
+/* act_i of layer i (applied to Z_i).  ReLU: relu'(0) = 0.  GELU: exact erf
+ * form gelu(z) = z Phi(z), gelu'(z) = Phi(z) + z phi(z). */
+typedef enum { OOO_ACT_IDENTITY = 0, OOO_ACT_RELU = 1, OOO_ACT_GELU_ERF = 2 } ooo_act;
+
+/* OOO_SCHED_IN_ORDER: conventional backprop with per-layer
+ *   overlapped sync (wait-free backprop): one compute stream runs, for
+ *   i = L..1, dO_i then dW_i (+ its bucket pack); each bucket's all-reduce is
+ *   issued as soon as it is packed.
+ * OOO_SCHED_FIRST_K: Algorithm 2 with k <- min(max_k, k)
+ *   (l.1-2): dO ops on the high-priority stream, dW ops on the low-priority
+ *   stream in D's order (critical ops high priority, sub-stream
+ *   kernels serialise), all-reduces on the comm stream in D's dW order.
+ *   k = 0 is dual-stream without reordering (the P:312 ablation). */
+typedef enum { OOO_SCHED_IN_ORDER = 0, OOO_SCHED_FIRST_K = 1 } ooo_sched_kind;
+
+typedef struct {
+  int32_t kind;   /* ooo_sched_kind */
+  int32_t k;      /* >= 0; clamped to [0, min(L, max_k)] (Alg. 2 l.2); k < 0 -> INVALID_ARGUMENT */
+} ooo_schedule;
+
+typedef struct {
+  int32_t num_layers;          /* L >= 1 */
+  const int32_t *dims;         /* L+1 host ints d_0..d_L; each >= 64 and % 64 == 0, else UNSUPPORTED */
+  const int32_t *acts;         /* L host ints (ooo_act) */
+  int32_t tokens;              /* M rows per rank per call; >= 1 and % 8 == 0 (TMA row alignment) */
+  int32_t dtype;               /* ooo_dtype */
+  int32_t need_input_grad;     /* 1: emit dO_1 and write dX (reading Q1); 0: omit dO_1 */
+  int32_t bucket_layers;       /* >= 1 consecutive layers per all-reduce bucket; schedule independent */
+  int64_t max_temp_bytes;      /* MXM of Alg. 2 l.1 (bytes); <= 0 = unlimited */
+  const void *const *W;        /* L device pointers, W_i [d_{i-1}][d_i] row-major, dtype */
+  const void *const *b;        /* L device pointers, b_i [d_i], dtype */
+  void *grads;                 /* device, grads_bytes (ooo_query_sizes), dtype: layer i at
+                                  ooo_grad_offsets: dW_i [d_{i-1}][d_i] row-major then db_i [d_i];
+                                  layers contiguous in increasing i, so a bucket of consecutive
+                                  layers is one contiguous all-reduce buffer.  Output. */
+  void *workspace;             /* device, workspace_bytes (ooo_query_sizes), 256-B aligned:
+                                  X_i / Z_i / dZ_i stores, split-K and bias-grad partials */
+  int32_t world_size;          /* N >= 1 */
+  int32_t rank;                /* 0 <= rank < N */
+  const void *nccl_unique_id;  /* OOO_UNIQUE_ID_BYTES from ooo_get_unique_id on rank 0, shared by
+                                  the caller (e.g. torch.distributed broadcast); NULL iff N == 1 */
+  int32_t comm_enabled;        /* 1: all-reduce each bucket.  0: comm-off control -- same streams,
+                                  events and kernels, the all-reduce is skipped (exposed-comm
+                                  measurement); gradients are then the local shard's. */
+  int32_t nccl_max_ctas;       /* > 0: ncclConfig_t.maxCTAs (bounds SMs taken from the GEMMs); 0 = NCCL default */
+} ooo_stack_desc;
+
+/* ---------------------------------------------------------------- info */
+int32_t ooo_abi_version(void);
+const char *ooo_last_error(void);                  /* thread-local message of the last non-OK status */
+const char *ooo_status_string(int32_t status);
+
+/* ------------------------------------------------------ host-only helpers */
+/* Sizes of the caller-allocated device buffers.  No device access. */
+ooo_status ooo_query_sizes(const ooo_stack_desc *d, size_t *workspace_bytes, size_t *grads_bytes);
+
+/* offsets[2*(i-1)] = element offset of dW_i, offsets[2*(i-1)+1] = of db_i, inside `grads`. */
+ooo_status ooo_grad_offsets(const ooo_stack_desc *d, int64_t *offsets /* 2L */);
+
+/* The backward order D as the library issues it (Alg. 2 lines 3-6, P:195-201;
+ * within a layer the paper's order dW_i before dO_i; IN_ORDER = dO_i first).
+ * ops[j] = +i for dO_i, -i for dW_i.  `ops` has room for 2L entries; *n
+ * receives the count.  `k` is clamped to [0, L] only (memory clamp: ooo_max_k). */
+ooo_status ooo_schedule_order(int32_t L, ooo_schedule sch, int32_t need_input_grad,
+                              int32_t *ops, int32_t *n);
+
+/* Alg. 2 line 1 (garbled in the text; reading Q3, parity unpinned):
+ * max_k = largest j in [0, L] with f(j) = m_fwd - sum_{i>j} m_dO[i-1] + sum_{i<=j} m_dW[i-1] < mxm;
+ * mxm <= 0 -> L.  Byte counts are host arrays of length L. */
+int32_t ooo_max_k(int32_t L, int64_t m_fwd, const int64_t *m_dO, const int64_t *m_dW, int64_t mxm);
+
+/* Extra bytes kept alive by deferring dW_1..dW_k (the memory cost of
+ * deferral, §3; E8 at P:352-354): sum_{i=2..k} |dZ_i|. */
+int64_t ooo_deferral_bytes(const ooo_stack_desc *d, int32_t k);
+
+/* NCCL bootstrap id (rank 0 calls, caller broadcasts).  Needs libnccl.so.2. */
+ooo_status ooo_get_unique_id(void *out /* OOO_UNIQUE_ID_BYTES */);
+
+/* ------------------------------------------------------------- the path */
+/* Validates, plans the workspace, encodes TMA descriptors, creates the
+ * priority streams / events and (N > 1) the NCCL communicator -- collective
+ * over ranks.  Uses the current CUDA device. */
+ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out);
+
+/* F_1..F_L: X [M][d_0] (device, dtype) -> Y [M][d_L] (device, dtype).
+ * X is copied into the stack's X_1 store; Y is written by F_L.  If a backward
+ * is pending, F_i first waits for layer i's synchronised gradient (and for
+ * dW_{i+1}, which still reads X_{i+1}). */
+ooo_status ooo_forward(ooo_stack *s, const void *X, void *Y, void *stream /* cudaStream_t */);
+
+/* Backward of the last forward: dY [M][d_L] (device, dtype).  dX [M][d_0]
+ * (device) is written iff need_input_grad, else must be NULL.
+ * OOO_ERR_STATE if no forward preceded it. */
+ooo_status ooo_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void *dX, void *stream);
+
+/* `stream` waits for all outstanding backward work, all-reduces included. */
+ooo_status ooo_join(ooo_stack *s, void *stream);
+
+/* Pre-compiled issue (§4.2): capture one training step
+ * [ooo_backward(dY, sch, dX); ooo_forward(X, Y)] into an executable CUDA graph
+ * instantiated with per-node priorities.  A plain ooo_forward(X, Y) must have
+ * run before.  Pointers are baked into the graph. */
+ooo_status ooo_graph_create(ooo_stack *s, const void *X, void *Y, const void *dY, ooo_schedule sch,
+                            void *dX, ooo_graph **out);
+ooo_status ooo_graph_launch(ooo_graph *g, void *stream);
+ooo_status ooo_graph_destroy(ooo_graph *g);
+
+ooo_status ooo_destroy(ooo_stack *s);             /* joins, then frees host/NCCL resources */
+
+/* ------------------------------------------------- introspection / timing */
+/* Device pointer of an internal store (teacher-forced parity tests):
+ * kind 0 = X_i (i = 1..L), 1 = Z_i (NULL for identity layers: Z_i aliases
+ * X_{i+1}), 2 = dZ_i, 3 = bias-grad partials of layer i ([rows][d_i] fp32). */
+ooo_status ooo_tensor(ooo_stack *s, int32_t kind, int32_t layer, void **ptr, int64_t *rows);
+
+/* Per-launch timing.  ooo_set_timing(s, 1) makes subsequently enqueued or
+ * captured calls bracket every kernel launch with CUDA events on the stream
+ * it is launched on.  After the work completed (e.g. after the last graph
+ * replay of a timed region), ooo_timing_read fills up to `cap` records
+ * describing the most recent execution of each bracketed launch. */
+typedef struct {
+  int32_t kind;       /* 0 fwd GEMM, 1 dX GEMM, 2 dW GEMM, 3 seed act-grad, 4 pack, 5 all-reduce, 6 copy */
+  int32_t layer;
+  int32_t stream;     /* 0 hi, 1 lo, 2 comm */
+  int32_t grid;       /* CTAs launched */
+  double flops;       /* algorithmic FLOPs of the launch (GEMMs) */
+  double bytes;       /* algorithmic HBM bytes of the launch (pack / seed / copy / all-reduce payload) */
+  float ms;           /* event-measured duration */
+} ooo_launch_record;
+ooo_status ooo_set_timing(ooo_stack *s, int32_t enable);
+ooo_status ooo_timing_read(ooo_stack *s, ooo_launch_record *out, int32_t cap, int32_t *n);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* OOO_H_ */

@@ -1,0 +1,142 @@
+"""ctypes declarations of the C ABI in include/ooo.h (argument marshalling only).
+
+Loading fails loudly if libooo.so has not been built: there is no fallback
+path of any kind.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from ctypes import POINTER, c_char_p, c_double, c_float, c_int32, c_int64, c_size_t, c_void_p
+
+LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "lib", "libooo.so")
+
+OOO_OK = 0
+STATUS = {0: "OOO_OK", 1: "OOO_ERR_INVALID_ARGUMENT", 2: "OOO_ERR_UNSUPPORTED", 3: "OOO_ERR_CUDA",
+          4: "OOO_ERR_NCCL", 5: "OOO_ERR_STATE"}
+DTYPES = {"bf16": 0, "fp32": 1}
+ACTS = {"id": 0, "relu": 1, "gelu": 2}
+SCHED_IN_ORDER = 0
+SCHED_FIRST_K = 1
+UNIQUE_ID_BYTES = 128
+
+
+class StackDesc(ctypes.Structure):
+    _fields_ = [
+        ("num_layers", c_int32),
+        ("dims", POINTER(c_int32)),
+        ("acts", POINTER(c_int32)),
+        ("tokens", c_int32),
+        ("dtype", c_int32),
+        ("need_input_grad", c_int32),
+        ("bucket_layers", c_int32),
+        ("max_temp_bytes", c_int64),
+        ("W", POINTER(c_void_p)),
+        ("b", POINTER(c_void_p)),
+        ("grads", c_void_p),
+        ("workspace", c_void_p),
+        ("world_size", c_int32),
+        ("rank", c_int32),
+        ("nccl_unique_id", c_void_p),
+        ("comm_enabled", c_int32),
+        ("nccl_max_ctas", c_int32),
+    ]
+
+
+class Schedule(ctypes.Structure):
+    _fields_ = [("kind", c_int32), ("k", c_int32)]
+
+
+class LaunchRecord(ctypes.Structure):
+    _fields_ = [
+        ("kind", c_int32),
+        ("layer", c_int32),
+        ("stream", c_int32),
+        ("grid", c_int32),
+        ("flops", c_double),
+        ("bytes", c_double),
+        ("ms", c_float),
+    ]
+
+
+KIND_NAMES = {0: "fwd_gemm", 1: "dx_gemm", 2: "dw_gemm", 3: "seed", 4: "pack", 5: "allreduce", 6: "copy"}
+
+EXPORTS = [
+    "ooo_abi_version", "ooo_last_error", "ooo_status_string", "ooo_query_sizes", "ooo_grad_offsets",
+    "ooo_schedule_order", "ooo_max_k", "ooo_deferral_bytes", "ooo_get_unique_id", "ooo_create_stack",
+    "ooo_forward", "ooo_backward", "ooo_join", "ooo_graph_create", "ooo_graph_launch",
+    "ooo_graph_destroy", "ooo_destroy", "ooo_tensor", "ooo_set_timing", "ooo_timing_read",
+]
+
+_lib = None
+
+
+class OooError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+def load() -> ctypes.CDLL:
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise RuntimeError(
+            f"{LIB_PATH} is missing: build it with `python -m paper_conf_eurosys_ohlks22_b200.build` "
+            "(or __graft_entry__.build()); there is no fallback path")
+    lib = ctypes.CDLL(LIB_PATH)
+    S = c_int32
+    lib.ooo_abi_version.restype = c_int32
+    lib.ooo_last_error.restype = c_char_p
+    lib.ooo_status_string.restype = c_char_p
+    lib.ooo_status_string.argtypes = [c_int32]
+    lib.ooo_query_sizes.restype = S
+    lib.ooo_query_sizes.argtypes = [POINTER(StackDesc), POINTER(c_size_t), POINTER(c_size_t)]
+    lib.ooo_grad_offsets.restype = S
+    lib.ooo_grad_offsets.argtypes = [POINTER(StackDesc), POINTER(c_int64)]
+    lib.ooo_schedule_order.restype = S
+    lib.ooo_schedule_order.argtypes = [c_int32, Schedule, c_int32, POINTER(c_int32), POINTER(c_int32)]
+    lib.ooo_max_k.restype = c_int32
+    lib.ooo_max_k.argtypes = [c_int32, c_int64, POINTER(c_int64), POINTER(c_int64), c_int64]
+    lib.ooo_deferral_bytes.restype = c_int64
+    lib.ooo_deferral_bytes.argtypes = [POINTER(StackDesc), c_int32]
+    lib.ooo_get_unique_id.restype = S
+    lib.ooo_get_unique_id.argtypes = [c_void_p]
+    lib.ooo_create_stack.restype = S
+    lib.ooo_create_stack.argtypes = [POINTER(StackDesc), POINTER(c_void_p)]
+    lib.ooo_forward.restype = S
+    lib.ooo_forward.argtypes = [c_void_p, c_void_p, c_void_p, c_void_p]
+    lib.ooo_backward.restype = S
+    lib.ooo_backward.argtypes = [c_void_p, c_void_p, Schedule, c_void_p, c_void_p]
+    lib.ooo_join.restype = S
+    lib.ooo_join.argtypes = [c_void_p, c_void_p]
+    lib.ooo_graph_create.restype = S
+    lib.ooo_graph_create.argtypes = [c_void_p, c_void_p, c_void_p, c_void_p, Schedule, c_void_p,
+                                     POINTER(c_void_p)]
+    lib.ooo_graph_launch.restype = S
+    lib.ooo_graph_launch.argtypes = [c_void_p, c_void_p]
+    lib.ooo_graph_destroy.restype = S
+    lib.ooo_graph_destroy.argtypes = [c_void_p]
+    lib.ooo_destroy.restype = S
+    lib.ooo_destroy.argtypes = [c_void_p]
+    lib.ooo_tensor.restype = S
+    lib.ooo_tensor.argtypes = [c_void_p, c_int32, c_int32, POINTER(c_void_p), POINTER(c_int64)]
+    lib.ooo_set_timing.restype = S
+    lib.ooo_set_timing.argtypes = [c_void_p, c_int32]
+    lib.ooo_timing_read.restype = S
+    lib.ooo_timing_read.argtypes = [c_void_p, POINTER(LaunchRecord), c_int32, POINTER(c_int32)]
+    _lib = lib
+    return lib
+
+
+def check(status: int) -> None:
+    if status != OOO_OK:
+        msg = load().ooo_last_error()
+        raise OooError(status, msg.decode() if msg else "")
+
+
+def schedule(kind: str | int, k: int = 0) -> Schedule:
+    if isinstance(kind, str):
+        kind = {"in_order": SCHED_IN_ORDER, "first_k": SCHED_FIRST_K, "ooo_first_k": SCHED_FIRST_K}[kind]
+    return Schedule(int(kind), int(k))

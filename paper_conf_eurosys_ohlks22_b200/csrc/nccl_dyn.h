@@ -1,0 +1,26 @@
+// Runtime-loaded NCCL (libnccl.so.2).  The library does not link NCCL so
+// that it loads on hosts without it (the CPU build/test box) and so that, in
+// a process that already loaded torch's bundled NCCL, the same copy is used.
+#pragma once
+#include <nccl.h>
+
+namespace ooo {
+
+struct NcclApi {
+  bool ok = false;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId *) = nullptr;
+  ncclResult_t (*CommInitRankConfig)(ncclComm_t *, int, ncclUniqueId, int, ncclConfig_t *) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*AllReduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t,
+                            cudaStream_t) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*CommAbort)(ncclComm_t) = nullptr;
+  ncclResult_t (*CommGetAsyncError)(ncclComm_t, ncclResult_t *) = nullptr;
+  const char *(*GetErrorString)(ncclResult_t) = nullptr;
+  ncclResult_t (*GetVersion)(int *) = nullptr;
+};
+
+// Loads once; returns nullptr (and a reason) if libnccl.so.2 is unavailable.
+const NcclApi *nccl_api(const char **why);
+
+}  // namespace ooo

@@ -1,0 +1,923 @@
+// C ABI (include/ooo.h) and the dependency-driven scheduler of the
+// out-of-order backprop data-parallel hot path.
+//
+// Paper mapping ("P:N" = line of /root/reference/PAPER.md):
+//   * iteration = backward(t) + S[dW_i] + forward(t+1), F_i gated on S[dW_i]
+//     (§2 problem statement, eq. at)
+//   * dW_i is consumed only by the update (§3) -> it may run out of
+//     order on a low-priority stream while the critical dO chain runs on a
+//     high-priority stream (§4.1; the sub-stream serialises its
+//     kernels); events enforce the cross-stream dependencies (§7)
+//   * the dW order is Algorithm 2 "Reverse First-K" (§5.1); S[dW_i]
+//     is one NCCL all-reduce per bucket issued in that order on a comm stream
+//   * a step can be captured as one executable CUDA graph (§4.2)
+//   * static per-stream workspaces planned at create time replace the paper's
+//     separate sub-stream allocator / XLA heap simulator (§7)
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdarg.h>
+#include <stdio.h>
+#include <string.h>
+
+#include <algorithm>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/ooo.h"
+#include "kernels.h"
+#include "nccl_dyn.h"
+
+using namespace ooo;
+
+// ------------------------------------------------------------------ errors
+namespace {
+thread_local std::string t_err;
+
+ooo_status fail(ooo_status st, const char *fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  t_err = buf;
+  return st;
+}
+
+#define CU_TRY(expr)                                                                   \
+  do {                                                                                 \
+    cudaError_t _e = (expr);                                                           \
+    if (_e != cudaSuccess)                                                             \
+      return fail(OOO_ERR_CUDA, "%s failed: %s (%s:%d)", #expr, cudaGetErrorString(_e), \
+                  __FILE__, __LINE__);                                                 \
+  } while (0)
+
+#define OOO_TRY(expr)                  \
+  do {                                 \
+    ooo_status _s = (expr);            \
+    if (_s != OOO_OK) return _s;       \
+  } while (0)
+
+size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+// ------------------------------------------------------------------ plan
+struct GemmPlan {
+  int bn = 128;
+  int splits = 1;
+  int kb_per_split = 1;
+  dim3 grid;
+};
+
+struct LayerPlan {
+  int din = 0, dout = 0, act = 0;
+  size_t off_X = 0;            // X_i (input of layer i)
+  size_t off_Z = SIZE_MAX;     // Z_i (only for non-identity act)
+  size_t off_Xn = SIZE_MAX;    // X_{i+1} (i < L)
+  size_t off_dZ = 0;
+  size_t off_db = 0;           // bias-grad partials [R][dout] fp32
+  int64_t goff_w = 0, goff_b = 0;
+  int bucket = 0;
+  GemmPlan fwd, dx, dw;
+};
+
+struct Plan {
+  int L = 0, M = 0, dtype = 0, elt = 2, R = 0, nbuckets = 0;
+  std::vector<LayerPlan> layer;  // index i-1
+  std::vector<int> bucket_first, bucket_last;
+  size_t off_wpart = 0, wpart_bytes = 0;
+  size_t workspace_bytes = 0;
+  int64_t grad_elems = 0;
+};
+
+constexpr int kSMs = 148;
+
+GemmPlan plan_tc_mn(int M, int N, int K, bool weight_grad) {
+  GemmPlan p;
+  const int mt = (M + 127) / 128;
+  const int nkb = (K + 63) / 64;
+  int best_bn = 64;
+  // largest tile that still fills the machine; else the one with most CTAs
+  const int cands[3] = {256, 128, 64};
+  bool chosen = false;
+  for (int bn : cands) {
+    if (N % bn != 0) continue;
+    const int tiles = mt * (N / bn);
+    if (tiles >= kSMs) { best_bn = bn; chosen = true; break; }
+  }
+  if (!chosen) {
+    // not a full wave: prefer 128 unless 64 gives markedly more CTAs
+    best_bn = (N % 128 == 0) ? 128 : 64;
+    if (!weight_grad && mt * ((N + 127) / 128) < kSMs / 2) best_bn = 64;
+  }
+  if (weight_grad) best_bn = (N % 128 == 0) ? 128 : 64;
+  p.bn = best_bn;
+  const int tiles = mt * ((N + p.bn - 1) / p.bn);
+  int S = 1;
+  if (weight_grad && tiles < kSMs) {
+    S = kSMs / tiles;
+    S = std::min(S, std::max(1, nkb / 4));
+    S = std::max(S, 1);
+  }
+  p.kb_per_split = (nkb + S - 1) / S;
+  p.splits = (nkb + p.kb_per_split - 1) / p.kb_per_split;   // every split >= 1 k-block
+  p.grid = dim3(mt, (N + p.bn - 1) / p.bn, p.splits);
+  return p;
+}
+
+GemmPlan plan_simt(int M, int N, int K, bool weight_grad) {
+  GemmPlan p;
+  p.bn = 64;
+  const int nkb = (K + 15) / 16;
+  const int tiles = ((M + 63) / 64) * ((N + 63) / 64);
+  int S = 1;
+  if (weight_grad && tiles < kSMs) S = std::max(1, std::min(kSMs / tiles, nkb / 8));
+  p.kb_per_split = (nkb + S - 1) / S;
+  p.splits = (nkb + p.kb_per_split - 1) / p.kb_per_split;
+  p.grid = dim3((M + 63) / 64, (N + 63) / 64, p.splits);
+  return p;
+}
+
+ooo_status validate_desc(const ooo_stack_desc *d, bool need_pointers) {
+  if (!d) return fail(OOO_ERR_INVALID_ARGUMENT, "desc is NULL");
+  if (d->num_layers < 1) return fail(OOO_ERR_INVALID_ARGUMENT, "num_layers must be >= 1");
+  if (!d->dims || !d->acts) return fail(OOO_ERR_INVALID_ARGUMENT, "dims/acts NULL");
+  for (int i = 0; i <= d->num_layers; ++i) {
+    if (d->dims[i] < 64 || d->dims[i] % 64 != 0)
+      return fail(OOO_ERR_UNSUPPORTED, "dims[%d] = %d: widths must be >= 64 and multiples of 64", i,
+                  d->dims[i]);
+  }
+  for (int i = 0; i < d->num_layers; ++i)
+    if (d->acts[i] < 0 || d->acts[i] > 2)
+      return fail(OOO_ERR_INVALID_ARGUMENT, "acts[%d] = %d invalid", i, d->acts[i]);
+  if (d->tokens < 1 || d->tokens % 8 != 0)
+    return fail(OOO_ERR_UNSUPPORTED, "tokens = %d: must be >= 1 and a multiple of 8", d->tokens);
+  if (d->dtype != OOO_BF16 && d->dtype != OOO_FP32)
+    return fail(OOO_ERR_INVALID_ARGUMENT, "dtype %d invalid", d->dtype);
+  if (d->bucket_layers < 1) return fail(OOO_ERR_INVALID_ARGUMENT, "bucket_layers must be >= 1");
+  if (d->world_size < 1 || d->rank < 0 || d->rank >= d->world_size)
+    return fail(OOO_ERR_INVALID_ARGUMENT, "world_size %d / rank %d invalid", d->world_size, d->rank);
+  if (need_pointers) {
+    if (!d->W || !d->b) return fail(OOO_ERR_INVALID_ARGUMENT, "W/b arrays NULL");
+    for (int i = 0; i < d->num_layers; ++i)
+      if (!d->W[i] || !d->b[i]) return fail(OOO_ERR_INVALID_ARGUMENT, "W[%d]/b[%d] NULL", i, i);
+    if (!d->grads || !d->workspace) return fail(OOO_ERR_INVALID_ARGUMENT, "grads/workspace NULL");
+    if (reinterpret_cast<uintptr_t>(d->workspace) % 256 != 0 ||
+        reinterpret_cast<uintptr_t>(d->grads) % 256 != 0)
+      return fail(OOO_ERR_INVALID_ARGUMENT, "grads/workspace must be 256-byte aligned");
+    if (d->world_size > 1 && !d->nccl_unique_id)
+      return fail(OOO_ERR_INVALID_ARGUMENT, "world_size > 1 needs nccl_unique_id");
+  }
+  return OOO_OK;
+}
+
+Plan make_plan(const ooo_stack_desc *d) {
+  Plan p;
+  p.L = d->num_layers;
+  p.M = d->tokens;
+  p.dtype = d->dtype;
+  p.elt = d->dtype == OOO_BF16 ? 2 : 4;
+  const int bm = d->dtype == OOO_BF16 ? kTcBM : kSimtBM;
+  p.R = (p.M + bm - 1) / bm;
+  p.layer.resize(p.L);
+  size_t off = 0;
+  auto take = [&](size_t bytes) {
+    size_t o = off;
+    off = align_up(off + bytes, 256);
+    return o;
+  };
+  const size_t M = p.M;
+  // X_1, then per layer Z_i (non-identity) and X_{i+1}
+  size_t xoff = take(M * d->dims[0] * p.elt);
+  int64_t goff = 0;
+  size_t wpart = 0;
+  for (int i = 1; i <= p.L; ++i) {
+    LayerPlan &lp = p.layer[i - 1];
+    lp.din = d->dims[i - 1];
+    lp.dout = d->dims[i];
+    lp.act = d->acts[i - 1];
+    lp.off_X = xoff;
+    if (lp.act != OOO_ACT_IDENTITY) lp.off_Z = take(M * lp.dout * p.elt);
+    if (i < p.L) {
+      lp.off_Xn = take(M * lp.dout * p.elt);
+      xoff = lp.off_Xn;
+    }
+    lp.goff_w = goff;
+    lp.goff_b = goff + (int64_t)lp.din * lp.dout;
+    goff = lp.goff_b + lp.dout;
+    lp.bucket = (i - 1) / d->bucket_layers;
+    if (p.dtype == OOO_BF16) {
+      lp.fwd = plan_tc_mn(p.M, lp.dout, lp.din, false);
+      lp.dx = plan_tc_mn(p.M, lp.din, lp.dout, false);
+      lp.dw = plan_tc_mn(lp.din, lp.dout, p.M, true);
+    } else {
+      lp.fwd = plan_simt(p.M, lp.dout, lp.din, false);
+      lp.dx = plan_simt(p.M, lp.din, lp.dout, false);
+      lp.dw = plan_simt(lp.din, lp.dout, p.M, true);
+    }
+    if (lp.dw.splits > 1) wpart = std::max(wpart, (size_t)lp.dw.splits * lp.din * lp.dout * 4);
+  }
+  for (int i = 1; i <= p.L; ++i) p.layer[i - 1].off_dZ = take(M * p.layer[i - 1].dout * p.elt);
+  for (int i = 1; i <= p.L; ++i) p.layer[i - 1].off_db = take((size_t)p.R * p.layer[i - 1].dout * 4);
+  p.wpart_bytes = wpart;
+  p.off_wpart = wpart ? take(wpart) : 0;
+  p.workspace_bytes = std::max<size_t>(off, 256);
+  p.grad_elems = goff;
+  p.nbuckets = (p.L + d->bucket_layers - 1) / d->bucket_layers;
+  p.bucket_first.resize(p.nbuckets);
+  p.bucket_last.resize(p.nbuckets);
+  for (int b = 0; b < p.nbuckets; ++b) {
+    p.bucket_first[b] = b * d->bucket_layers + 1;
+    p.bucket_last[b] = std::min(p.L, (b + 1) * d->bucket_layers);
+  }
+  return p;
+}
+
+// Alg. 2 lines 3-6.  Reading Q1: dO_1 only if need_input_grad.
+// in_order (k = 0, dO_i first within a layer, reading Q2).
+void schedule_ops(int L, int kind, int k, bool need_dx, std::vector<int> &D) {
+  D.clear();
+  if (kind == OOO_SCHED_IN_ORDER) {
+    for (int i = L; i >= 1; --i) {
+      if (i > 1 || need_dx) D.push_back(+i);
+      D.push_back(-i);
+    }
+    return;
+  }
+  k = std::min(std::max(k, 0), L);
+  for (int i = L; i >= 1; --i) {           // l.3
+    if (i > k) D.push_back(-i);            // l.4
+    if (i > 1 || need_dx) D.push_back(+i); // l.5
+  }
+  for (int i = 1; i <= k; ++i) D.push_back(-i);   // l.6
+}
+
+// ------------------------------------------------------------ tensor maps
+typedef CUresult (*EncodeTiledFn)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *,
+                                  const cuuint64_t *, const cuuint64_t *, const cuuint32_t *,
+                                  const cuuint32_t *, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn get_encode() {
+  static EncodeTiledFn fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(p);
+  });
+  return fn;
+}
+
+// 2-D bf16 row-major tensor [outer][inner], 128-B swizzled box {box_inner, box_outer}.
+ooo_status make_map(CUtensorMap *m, const void *ptr, uint64_t inner, uint64_t outer,
+                    uint32_t box_inner, uint32_t box_outer) {
+  EncodeTiledFn enc = get_encode();
+  if (!enc) return fail(OOO_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {inner * 2};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(ptr), dims, strides, box,
+                   es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
+  return OOO_OK;
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ stack
+struct LayerRt {
+  void *W = nullptr, *b = nullptr;
+  void *X = nullptr, *Z = nullptr, *Xn = nullptr, *dZ = nullptr;
+  float *db = nullptr;
+  void *gw = nullptr, *gb = nullptr;
+  CUtensorMap fwdA, fwdB, dxA, dxB, dwA, dwB;
+};
+
+struct TimedRec {
+  ooo_launch_record info;
+  cudaEvent_t a = nullptr, b = nullptr;
+};
+
+struct ooo_stack {
+  ooo_stack_desc d;
+  std::vector<int> dims, acts;
+  Plan p;
+  std::vector<LayerRt> lr;
+  uint8_t *ws = nullptr;
+  uint8_t *grads = nullptr;
+  cudaStream_t hi = nullptr, lo = nullptr, comm = nullptr;
+  int prio_hi = 0, prio_lo = 0;
+  std::vector<cudaEvent_t> ev_dz, ev_pack, ev_ar;   // ev_dz[i], ev_pack[i] (1-based), ev_ar[b]
+  cudaEvent_t ev_fork = nullptr, ev_j_hi = nullptr, ev_j_lo = nullptr, ev_j_comm = nullptr;
+  bool have_fwd = false;
+  bool bwd_pending = false;
+  ncclComm_t nccl = nullptr;
+  const NcclApi *api = nullptr;
+  bool timing = false;
+  std::vector<TimedRec> recs;
+  size_t rec_cursor = 0;
+  std::vector<int> D;
+};
+
+struct ooo_graph {
+  ooo_stack *s = nullptr;
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t exec = nullptr;
+};
+
+namespace {
+
+ooo_status begin_rec(ooo_stack *s, cudaStream_t st, int kind, int layer, int sid, TimedRec **out) {
+  *out = nullptr;
+  if (!s->timing) return OOO_OK;
+  if (s->rec_cursor >= s->recs.size()) {
+    TimedRec r;
+    CU_TRY(cudaEventCreate(&r.a));
+    CU_TRY(cudaEventCreate(&r.b));
+    s->recs.push_back(r);
+  }
+  TimedRec *r = &s->recs[s->rec_cursor++];
+  memset(&r->info, 0, sizeof(r->info));
+  r->info.kind = kind;
+  r->info.layer = layer;
+  r->info.stream = sid;
+  CU_TRY(cudaEventRecordWithFlags(r->a, st, cudaEventRecordExternal));
+  *out = r;
+  return OOO_OK;
+}
+ooo_status end_rec(TimedRec *r, cudaStream_t st, int grid, double flops, double bytes) {
+  if (!r) return OOO_OK;
+  r->info.grid = grid;
+  r->info.flops = flops;
+  r->info.bytes = bytes;
+  CU_TRY(cudaEventRecordWithFlags(r->b, st, cudaEventRecordExternal));
+  return OOO_OK;
+}
+
+// ---- op launchers ------------------------------------------------------
+ooo_status launch_fwd(ooo_stack *s, int i, void *Y, cudaStream_t st, int prio) {
+  const LayerPlan &lp = s->p.layer[i - 1];
+  LayerRt &r = s->lr[i - 1];
+  EpiArgs a = {};
+  a.M = s->p.M; a.N = lp.dout; a.K = lp.din;
+  a.kb_per_split = lp.fwd.kb_per_split; a.splits = 1;
+  a.act = lp.act; a.ldc = lp.dout; a.alpha = 1.f;
+  a.bias = r.b; a.z_out = r.Z; a.x_out = (i == s->p.L) ? Y : r.Xn;
+  TimedRec *tr;
+  OOO_TRY(begin_rec(s, st, 0, i, 0, &tr));
+  LaunchCtx ctx{st, prio};
+  int grid = lp.fwd.grid.x * lp.fwd.grid.y * lp.fwd.grid.z;
+  if (s->p.dtype == OOO_BF16) {
+    CU_TRY(launch_gemm_tc(EPI_FWD, lp.fwd.bn, &r.fwdA, &r.fwdB, a, lp.fwd.grid, ctx));
+  } else {
+    SimtOperands o{static_cast<const float *>(r.X), lp.din, 1, static_cast<const float *>(r.W), lp.dout, 1};
+    CU_TRY(launch_gemm_simt(EPI_FWD, o, a, ctx, &grid));
+  }
+  return end_rec(tr, st, grid, 2.0 * s->p.M * lp.din * lp.dout, 0);
+}
+
+// dO_i: i >= 2 -> dZ_{i-1} (+ db_{i-1} partials); i == 1 -> dX (no epilogue)
+ooo_status launch_dx(ooo_stack *s, int i, void *dX, cudaStream_t st, int prio) {
+  const LayerPlan &lp = s->p.layer[i - 1];
+  LayerRt &r = s->lr[i - 1];
+  EpiArgs a = {};
+  a.M = s->p.M; a.N = lp.din; a.K = lp.dout;
+  a.kb_per_split = lp.dx.kb_per_split; a.splits = 1;
+  a.ldc = lp.din; a.alpha = 1.f;
+  if (i >= 2) {
+    const LayerPlan &pp = s->p.layer[i - 2];
+    LayerRt &pr = s->lr[i - 2];
+    a.act = pp.act;
+    a.zin = pr.Z;            // null for identity (act' = 1, not read)
+    a.x_out = pr.dZ;
+    a.dbpart = pr.db;
+  } else {
+    a.act = OOO_ACT_IDENTITY;
+    a.x_out = dX;
+    a.dbpart = nullptr;
+  }
+  TimedRec *tr;
+  OOO_TRY(begin_rec(s, st, 1, i, st == s->hi ? 0 : 1, &tr));
+  LaunchCtx ctx{st, prio};
+  int grid = lp.dx.grid.x * lp.dx.grid.y * lp.dx.grid.z;
+  if (s->p.dtype == OOO_BF16) {
+    CU_TRY(launch_gemm_tc(EPI_DGRAD, lp.dx.bn, &r.dxA, &r.dxB, a, lp.dx.grid, ctx));
+  } else {
+    SimtOperands o{static_cast<const float *>(r.dZ), lp.dout, 1, static_cast<const float *>(r.W), 1, lp.dout};
+    CU_TRY(launch_gemm_simt(EPI_DGRAD, o, a, ctx, &grid));
+  }
+  return end_rec(tr, st, grid, 2.0 * s->p.M * lp.din * lp.dout, 0);
+}
+
+// dW_i (+ pack: split-K reduction, db reduction, 1/N scale -> bucket)
+ooo_status launch_dw_pack(ooo_stack *s, int i, cudaStream_t st, int prio, int sid) {
+  const LayerPlan &lp = s->p.layer[i - 1];
+  LayerRt &r = s->lr[i - 1];
+  const float alpha = 1.0f / (float)s->d.world_size;
+  EpiArgs a = {};
+  a.M = lp.din; a.N = lp.dout; a.K = s->p.M;
+  a.kb_per_split = lp.dw.kb_per_split; a.splits = lp.dw.splits;
+  a.ldc = lp.dout; a.alpha = alpha;
+  a.x_out = r.gw;
+  a.fpart = reinterpret_cast<float *>(s->ws + s->p.off_wpart);
+  TimedRec *tr;
+  OOO_TRY(begin_rec(s, st, 2, i, sid, &tr));
+  LaunchCtx ctx{st, prio};
+  int grid = lp.dw.grid.x * lp.dw.grid.y * lp.dw.grid.z;
+  if (s->p.dtype == OOO_BF16) {
+    CU_TRY(launch_gemm_tc(EPI_WGRAD, lp.dw.bn, &r.dwA, &r.dwB, a, lp.dw.grid, ctx));
+  } else {
+    SimtOperands o{static_cast<const float *>(r.X), 1, lp.din, static_cast<const float *>(r.dZ), lp.dout, 1};
+    CU_TRY(launch_gemm_simt(EPI_WGRAD, o, a, ctx, &grid));
+  }
+  OOO_TRY(end_rec(tr, st, grid, 2.0 * s->p.M * lp.din * lp.dout, 0));
+  // pack
+  OOO_TRY(begin_rec(s, st, 4, i, sid, &tr));
+  const bool split = lp.dw.splits > 1;
+  const long long wcount = (long long)lp.din * lp.dout;
+  int pgrid = 0;
+  CU_TRY(launch_pack(s->p.dtype == OOO_BF16, split ? a.fpart : nullptr, lp.dw.splits, wcount, r.gw, r.db,
+                     s->p.R, lp.dout, r.gb, alpha, ctx, &pgrid));
+  const double pbytes = (split ? (double)wcount * (4.0 * lp.dw.splits + s->p.elt) : 0.0) +
+                        (double)lp.dout * (4.0 * s->p.R + s->p.elt);
+  return end_rec(tr, st, pgrid, 0, pbytes);
+}
+
+ooo_status launch_seed_op(ooo_stack *s, const void *dY, cudaStream_t st, int prio) {
+  const int L = s->p.L;
+  const LayerPlan &lp = s->p.layer[L - 1];
+  LayerRt &r = s->lr[L - 1];
+  TimedRec *tr;
+  OOO_TRY(begin_rec(s, st, 3, L, 0, &tr));
+  int grid = 0;
+  LaunchCtx ctx{st, prio};
+  const int bm = s->p.dtype == OOO_BF16 ? kTcBM : kSimtBM;
+  CU_TRY(launch_seed(s->p.dtype == OOO_BF16, dY, r.Z, lp.act, r.dZ, r.db, s->p.M, lp.dout, bm, ctx, &grid));
+  const double bytes = (double)s->p.M * lp.dout * s->p.elt * (lp.act != OOO_ACT_IDENTITY ? 3.0 : 2.0) +
+                       (double)s->p.R * lp.dout * 4.0;
+  return end_rec(tr, st, grid, 0, bytes);
+}
+
+ooo_status launch_allreduce(ooo_stack *s, int b) {
+  const int first = s->p.bucket_first[b], last = s->p.bucket_last[b];
+  const LayerPlan &f = s->p.layer[first - 1];
+  const LayerPlan &l = s->p.layer[last - 1];
+  const int64_t e0 = f.goff_w, e1 = l.goff_b + l.dout;
+  if (s->nccl && s->d.comm_enabled) {
+    TimedRec *tr;
+    OOO_TRY(begin_rec(s, s->comm, 5, b, 2, &tr));
+    void *buf = s->grads + e0 * s->p.elt;
+    ncclResult_t rr = s->api->AllReduce(buf, buf, (size_t)(e1 - e0),
+                                        s->p.dtype == OOO_BF16 ? ncclBfloat16 : ncclFloat32, ncclSum,
+                                        s->nccl, s->comm);
+    if (rr != ncclSuccess)
+      return fail(OOO_ERR_NCCL, "ncclAllReduce: %s", s->api->GetErrorString(rr));
+    const double n = s->d.world_size;
+    OOO_TRY(end_rec(tr, s->comm, 0, 0, 2.0 * (n - 1) / n * (double)(e1 - e0) * s->p.elt));
+  }
+  return OOO_OK;
+}
+
+ooo_status fork_from(ooo_stack *s, cudaStream_t st) {
+  CU_TRY(cudaEventRecord(s->ev_fork, st));
+  CU_TRY(cudaStreamWaitEvent(s->hi, s->ev_fork, 0));
+  CU_TRY(cudaStreamWaitEvent(s->lo, s->ev_fork, 0));
+  CU_TRY(cudaStreamWaitEvent(s->comm, s->ev_fork, 0));
+  return OOO_OK;
+}
+
+ooo_status join_into(ooo_stack *s, cudaStream_t st) {
+  CU_TRY(cudaEventRecord(s->ev_j_hi, s->hi));
+  CU_TRY(cudaEventRecord(s->ev_j_lo, s->lo));
+  CU_TRY(cudaEventRecord(s->ev_j_comm, s->comm));
+  CU_TRY(cudaStreamWaitEvent(st, s->ev_j_hi, 0));
+  CU_TRY(cudaStreamWaitEvent(st, s->ev_j_lo, 0));
+  CU_TRY(cudaStreamWaitEvent(st, s->ev_j_comm, 0));
+  return OOO_OK;
+}
+
+ooo_status check_async(ooo_stack *s) {
+  if (s->nccl) {
+    ncclResult_t ar = ncclSuccess;
+    ncclResult_t rr = s->api->CommGetAsyncError(s->nccl, &ar);
+    if (rr != ncclSuccess || ar != ncclSuccess)
+      return fail(OOO_ERR_NCCL, "NCCL async error: %s",
+                  s->api->GetErrorString(rr != ncclSuccess ? rr : ar));
+  }
+  cudaError_t e = cudaPeekAtLastError();
+  if (e != cudaSuccess) return fail(OOO_ERR_CUDA, "pending CUDA error: %s", cudaGetErrorString(e));
+  return OOO_OK;
+}
+
+ooo_status enqueue_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st) {
+  const int L = s->p.L;
+  OOO_TRY(fork_from(s, st));
+  const bool pend = s->bwd_pending;
+  if (pend) CU_TRY(cudaStreamWaitEvent(s->hi, s->ev_pack[1], 0));   // dW_1(t) still reads X_1
+  {
+    TimedRec *tr;
+    OOO_TRY(begin_rec(s, s->hi, 6, 1, 0, &tr));
+    const size_t bytes = (size_t)s->p.M * s->dims[0] * s->p.elt;
+    CU_TRY(cudaMemcpyAsync(s->lr[0].X, X, bytes, cudaMemcpyDeviceToDevice, s->hi));
+    OOO_TRY(end_rec(tr, s->hi, 0, 0, 2.0 * bytes));
+  }
+  for (int i = 1; i <= L; ++i) {
+    if (pend) {
+      // T(F_i) >= T(S[dW_i]) + S[dW_i]
+      CU_TRY(cudaStreamWaitEvent(s->hi, s->ev_ar[s->p.layer[i - 1].bucket], 0));
+      // WAR guard of the static buffers: dW_{i+1}(t) reads X_{i+1}, which F_i overwrites
+      if (i < L) CU_TRY(cudaStreamWaitEvent(s->hi, s->ev_pack[i + 1], 0));
+    }
+    OOO_TRY(launch_fwd(s, i, Y, s->hi, s->prio_hi));
+  }
+  s->bwd_pending = false;
+  s->have_fwd = true;
+  return join_into(s, st);
+}
+
+ooo_status enqueue_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void *dX, cudaStream_t st) {
+  const int L = s->p.L;
+  int k = sch.k;
+  if (sch.kind == OOO_SCHED_FIRST_K) {
+    int mk = ooo_max_k(L, 0, nullptr, nullptr, 0);
+    if (s->d.max_temp_bytes > 0) {
+      std::vector<int64_t> mdo(L), mdw(L);
+      int64_t mf = (int64_t)s->p.M * s->dims[0] * s->p.elt;
+      for (int i = 1; i <= L; ++i) {
+        const LayerPlan &lp = s->p.layer[i - 1];
+        const int64_t act_bytes = (int64_t)s->p.M * lp.din * s->p.elt +
+                                  (lp.act != OOO_ACT_IDENTITY ? (int64_t)s->p.M * lp.dout * s->p.elt : 0);
+        mdo[i - 1] = act_bytes;
+        mdw[i - 1] = (int64_t)s->p.M * lp.dout * s->p.elt;
+        mf += (lp.act != OOO_ACT_IDENTITY ? (int64_t)s->p.M * lp.dout * s->p.elt : 0) +
+              (i < L ? (int64_t)s->p.M * lp.dout * s->p.elt : 0);
+      }
+      mk = ooo_max_k(L, mf, mdo.data(), mdw.data(), s->d.max_temp_bytes);
+    }
+    k = std::min(k, mk);
+  }
+  schedule_ops(L, sch.kind, k, s->d.need_input_grad != 0, s->D);
+  if (s->timing) s->rec_cursor = 0;
+  OOO_TRY(fork_from(s, st));
+  const bool single = sch.kind == OOO_SCHED_IN_ORDER;
+  cudaStream_t wst = single ? s->hi : s->lo;
+  const int wprio = single ? s->prio_hi : s->prio_lo;
+  const int wsid = single ? 0 : 1;
+  // seed dO_{L+1} at time 0
+  OOO_TRY(launch_seed_op(s, dY, s->hi, s->prio_hi));
+  CU_TRY(cudaEventRecord(s->ev_dz[L], s->hi));
+  std::vector<int> left(s->p.nbuckets);
+  for (int b = 0; b < s->p.nbuckets; ++b) left[b] = s->p.bucket_last[b] - s->p.bucket_first[b] + 1;
+  for (int op : s->D) {
+    if (op > 0) {
+      const int i = op;
+      OOO_TRY(launch_dx(s, i, dX, s->hi, s->prio_hi));
+      if (i >= 2) CU_TRY(cudaEventRecord(s->ev_dz[i - 1], s->hi));
+    } else {
+      const int i = -op;
+      if (!single) CU_TRY(cudaStreamWaitEvent(s->lo, s->ev_dz[i], 0));
+      OOO_TRY(launch_dw_pack(s, i, wst, wprio, wsid));
+      CU_TRY(cudaEventRecord(s->ev_pack[i], wst));
+      const int b = s->p.layer[i - 1].bucket;
+      if (--left[b] == 0) {
+        // S[dW] for the bucket, issued in D's dW order on every rank (FIFO comm stream)
+        CU_TRY(cudaStreamWaitEvent(s->comm, s->ev_pack[i], 0));
+        OOO_TRY(launch_allreduce(s, b));
+        CU_TRY(cudaEventRecord(s->ev_ar[b], s->comm));
+      }
+    }
+  }
+  s->have_fwd = false;
+  s->bwd_pending = true;
+  return OOO_OK;
+}
+
+}  // namespace
+
+// ======================================================================
+extern "C" {
+
+int32_t ooo_abi_version(void) { return OOO_ABI_VERSION; }
+
+const char *ooo_last_error(void) { return t_err.c_str(); }
+
+const char *ooo_status_string(int32_t st) {
+  switch (st) {
+    case OOO_OK: return "OOO_OK";
+    case OOO_ERR_INVALID_ARGUMENT: return "OOO_ERR_INVALID_ARGUMENT";
+    case OOO_ERR_UNSUPPORTED: return "OOO_ERR_UNSUPPORTED";
+    case OOO_ERR_CUDA: return "OOO_ERR_CUDA";
+    case OOO_ERR_NCCL: return "OOO_ERR_NCCL";
+    case OOO_ERR_STATE: return "OOO_ERR_STATE";
+  }
+  return "unknown";
+}
+
+ooo_status ooo_query_sizes(const ooo_stack_desc *d, size_t *workspace_bytes, size_t *grads_bytes) {
+  OOO_TRY(validate_desc(d, false));
+  if (!workspace_bytes || !grads_bytes) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL output");
+  Plan p = make_plan(d);
+  *workspace_bytes = p.workspace_bytes;
+  *grads_bytes = align_up((size_t)p.grad_elems * p.elt, 256);
+  return OOO_OK;
+}
+
+ooo_status ooo_grad_offsets(const ooo_stack_desc *d, int64_t *offsets) {
+  OOO_TRY(validate_desc(d, false));
+  if (!offsets) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL output");
+  Plan p = make_plan(d);
+  for (int i = 0; i < p.L; ++i) {
+    offsets[2 * i] = p.layer[i].goff_w;
+    offsets[2 * i + 1] = p.layer[i].goff_b;
+  }
+  return OOO_OK;
+}
+
+ooo_status ooo_schedule_order(int32_t L, ooo_schedule sch, int32_t need_input_grad, int32_t *ops,
+                              int32_t *n) {
+  if (L < 1) return fail(OOO_ERR_INVALID_ARGUMENT, "L must be >= 1");
+  if (sch.kind != OOO_SCHED_IN_ORDER && sch.kind != OOO_SCHED_FIRST_K)
+    return fail(OOO_ERR_INVALID_ARGUMENT, "schedule kind %d invalid", sch.kind);
+  if (sch.k < 0) return fail(OOO_ERR_INVALID_ARGUMENT, "k must be >= 0");
+  if (!ops || !n) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL output");
+  std::vector<int> D;
+  schedule_ops(L, sch.kind, sch.k, need_input_grad != 0, D);
+  for (size_t j = 0; j < D.size(); ++j) ops[j] = D[j];
+  *n = (int32_t)D.size();
+  return OOO_OK;
+}
+
+int32_t ooo_max_k(int32_t L, int64_t m_fwd, const int64_t *m_dO, const int64_t *m_dW, int64_t mxm) {
+  if (mxm <= 0 || !m_dO || !m_dW) return L;
+  // f(j) = m_fwd - sum_{i=j+1..L} m_dO[i] + sum_{i=1..j} m_dW[i]   (Alg. 2 l.1, reading Q3)
+  int best = 0;
+  for (int j = 0; j <= L; ++j) {
+    int64_t f = m_fwd;
+    for (int i = j + 1; i <= L; ++i) f -= m_dO[i - 1];
+    for (int i = 1; i <= j; ++i) f += m_dW[i - 1];
+    if (f < mxm) best = j;
+  }
+  return best;
+}
+
+int64_t ooo_deferral_bytes(const ooo_stack_desc *d, int32_t k) {
+  if (validate_desc(d, false) != OOO_OK) return -1;
+  int64_t s = 0;
+  const int elt = d->dtype == OOO_BF16 ? 2 : 4;
+  for (int i = 2; i <= std::min<int>(k, d->num_layers); ++i) s += (int64_t)d->tokens * d->dims[i] * elt;
+  return s;
+}
+
+ooo_status ooo_get_unique_id(void *out) {
+  if (!out) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL output");
+  const char *why = nullptr;
+  const NcclApi *api = nccl_api(&why);
+  if (!api) return fail(OOO_ERR_NCCL, "NCCL unavailable: %s", why);
+  ncclUniqueId id;
+  ncclResult_t r = api->GetUniqueId(&id);
+  if (r != ncclSuccess) return fail(OOO_ERR_NCCL, "ncclGetUniqueId: %s", api->GetErrorString(r));
+  memcpy(out, &id, sizeof(id) < OOO_UNIQUE_ID_BYTES ? sizeof(id) : OOO_UNIQUE_ID_BYTES);
+  return OOO_OK;
+}
+
+ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
+  if (!out) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL output");
+  *out = nullptr;
+  OOO_TRY(validate_desc(d, true));
+  ooo_stack *s = new ooo_stack();
+  s->d = *d;
+  s->dims.assign(d->dims, d->dims + d->num_layers + 1);
+  s->acts.assign(d->acts, d->acts + d->num_layers);
+  s->d.dims = s->dims.data();
+  s->d.acts = s->acts.data();
+  s->p = make_plan(d);
+  s->ws = static_cast<uint8_t *>(d->workspace);
+  s->grads = static_cast<uint8_t *>(d->grads);
+  const Plan &p = s->p;
+  auto cleanup_fail = [&](ooo_status st) {
+    std::string msg = t_err;
+    ooo_destroy(s);
+    t_err = msg;
+    return st;
+  };
+  static std::once_flag init_once;
+  static cudaError_t init_err = cudaSuccess;
+  std::call_once(init_once, [] { init_err = gemm_tc_init(); });
+  if (init_err != cudaSuccess)
+    return cleanup_fail(fail(OOO_ERR_CUDA, "kernel attribute init: %s", cudaGetErrorString(init_err)));
+  s->lr.resize(p.L);
+  for (int i = 1; i <= p.L; ++i) {
+    const LayerPlan &lp = p.layer[i - 1];
+    LayerRt &r = s->lr[i - 1];
+    r.W = const_cast<void *>(d->W[i - 1]);
+    r.b = const_cast<void *>(d->b[i - 1]);
+    r.X = s->ws + lp.off_X;
+    r.Z = lp.off_Z != SIZE_MAX ? s->ws + lp.off_Z : nullptr;
+    r.Xn = lp.off_Xn != SIZE_MAX ? s->ws + lp.off_Xn : nullptr;
+    r.dZ = s->ws + lp.off_dZ;
+    r.db = reinterpret_cast<float *>(s->ws + lp.off_db);
+    r.gw = s->grads + lp.goff_w * p.elt;
+    r.gb = s->grads + lp.goff_b * p.elt;
+    if (p.dtype == OOO_BF16) {
+      ooo_status st;
+      if ((st = make_map(&r.fwdA, r.X, lp.din, p.M, 64, 128)) != OOO_OK ||
+          (st = make_map(&r.fwdB, r.W, lp.dout, lp.din, 64, 64)) != OOO_OK ||
+          (st = make_map(&r.dxA, r.dZ, lp.dout, p.M, 64, 128)) != OOO_OK ||
+          (st = make_map(&r.dxB, r.W, lp.dout, lp.din, 64, lp.dx.bn)) != OOO_OK ||
+          (st = make_map(&r.dwA, r.X, lp.din, p.M, 64, 64)) != OOO_OK ||
+          (st = make_map(&r.dwB, r.dZ, lp.dout, p.M, 64, 64)) != OOO_OK)
+        return cleanup_fail(st);
+    }
+  }
+  int least = 0, greatest = 0;
+  cudaError_t e = cudaDeviceGetStreamPriorityRange(&least, &greatest);
+  if (e != cudaSuccess) return cleanup_fail(fail(OOO_ERR_CUDA, "priority range: %s", cudaGetErrorString(e)));
+  s->prio_hi = greatest;
+  s->prio_lo = least;
+  if ((e = cudaStreamCreateWithPriority(&s->hi, cudaStreamNonBlocking, greatest)) != cudaSuccess ||
+      (e = cudaStreamCreateWithPriority(&s->lo, cudaStreamNonBlocking, least)) != cudaSuccess ||
+      (e = cudaStreamCreateWithPriority(&s->comm, cudaStreamNonBlocking, greatest)) != cudaSuccess)
+    return cleanup_fail(fail(OOO_ERR_CUDA, "stream create: %s", cudaGetErrorString(e)));
+  auto mk = [&](cudaEvent_t *ev) { return cudaEventCreateWithFlags(ev, cudaEventDisableTiming); };
+  s->ev_dz.assign(p.L + 1, nullptr);
+  s->ev_pack.assign(p.L + 2, nullptr);
+  s->ev_ar.assign(p.nbuckets, nullptr);
+  for (int i = 1; i <= p.L; ++i) {
+    if ((e = mk(&s->ev_dz[i])) != cudaSuccess || (e = mk(&s->ev_pack[i])) != cudaSuccess)
+      return cleanup_fail(fail(OOO_ERR_CUDA, "event create: %s", cudaGetErrorString(e)));
+  }
+  for (int b = 0; b < p.nbuckets; ++b)
+    if ((e = mk(&s->ev_ar[b])) != cudaSuccess)
+      return cleanup_fail(fail(OOO_ERR_CUDA, "event create: %s", cudaGetErrorString(e)));
+  if ((e = mk(&s->ev_fork)) != cudaSuccess || (e = mk(&s->ev_j_hi)) != cudaSuccess ||
+      (e = mk(&s->ev_j_lo)) != cudaSuccess || (e = mk(&s->ev_j_comm)) != cudaSuccess)
+    return cleanup_fail(fail(OOO_ERR_CUDA, "event create: %s", cudaGetErrorString(e)));
+  if (d->world_size > 1) {
+    const char *why = nullptr;
+    s->api = nccl_api(&why);
+    if (!s->api) return cleanup_fail(fail(OOO_ERR_NCCL, "NCCL unavailable: %s", why));
+    ncclUniqueId id;
+    memcpy(&id, d->nccl_unique_id, sizeof(id));
+    ncclResult_t r;
+    if (s->api->CommInitRankConfig && d->nccl_max_ctas > 0) {
+      ncclConfig_t cfg = NCCL_CONFIG_INITIALIZER;
+      cfg.maxCTAs = d->nccl_max_ctas;
+      r = s->api->CommInitRankConfig(&s->nccl, d->world_size, id, d->rank, &cfg);
+    } else {
+      r = s->api->CommInitRank(&s->nccl, d->world_size, id, d->rank);
+    }
+    if (r != ncclSuccess) {
+      s->nccl = nullptr;
+      return cleanup_fail(fail(OOO_ERR_NCCL, "ncclCommInitRank: %s", s->api->GetErrorString(r)));
+    }
+  }
+  *out = s;
+  return OOO_OK;
+}
+
+ooo_status ooo_forward(ooo_stack *s, const void *X, void *Y, void *stream) {
+  if (!s || !X || !Y) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
+  OOO_TRY(check_async(s));
+  return enqueue_forward(s, X, Y, static_cast<cudaStream_t>(stream));
+}
+
+ooo_status ooo_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void *dX, void *stream) {
+  if (!s || !dY) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (sch.kind != OOO_SCHED_IN_ORDER && sch.kind != OOO_SCHED_FIRST_K)
+    return fail(OOO_ERR_INVALID_ARGUMENT, "schedule kind %d invalid", sch.kind);
+  if (sch.k < 0) return fail(OOO_ERR_INVALID_ARGUMENT, "k must be >= 0");
+  if (s->d.need_input_grad && !dX) return fail(OOO_ERR_INVALID_ARGUMENT, "need_input_grad set but dX NULL");
+  if (!s->d.need_input_grad && dX) return fail(OOO_ERR_INVALID_ARGUMENT, "dX given but need_input_grad = 0");
+  if (!s->have_fwd) return fail(OOO_ERR_STATE, "ooo_backward without a preceding ooo_forward");
+  OOO_TRY(check_async(s));
+  return enqueue_backward(s, dY, sch, dX, static_cast<cudaStream_t>(stream));
+}
+
+ooo_status ooo_join(ooo_stack *s, void *stream) {
+  if (!s) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL stack");
+  OOO_TRY(join_into(s, static_cast<cudaStream_t>(stream)));
+  return check_async(s);
+}
+
+ooo_status ooo_graph_create(ooo_stack *s, const void *X, void *Y, const void *dY, ooo_schedule sch,
+                            void *dX, ooo_graph **out) {
+  if (!s || !X || !Y || !dY || !out) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
+  *out = nullptr;
+  if (!s->have_fwd) return fail(OOO_ERR_STATE, "ooo_graph_create needs a preceding ooo_forward");
+  if (sch.kind != OOO_SCHED_IN_ORDER && sch.kind != OOO_SCHED_FIRST_K)
+    return fail(OOO_ERR_INVALID_ARGUMENT, "schedule kind %d invalid", sch.kind);
+  if (sch.k < 0) return fail(OOO_ERR_INVALID_ARGUMENT, "k must be >= 0");
+  if (s->d.need_input_grad && !dX) return fail(OOO_ERR_INVALID_ARGUMENT, "need_input_grad set but dX NULL");
+  if (!s->d.need_input_grad && dX) return fail(OOO_ERR_INVALID_ARGUMENT, "dX given but need_input_grad = 0");
+  cudaStream_t cap;
+  CU_TRY(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
+  cudaError_t e = cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal);
+  if (e != cudaSuccess) {
+    cudaStreamDestroy(cap);
+    return fail(OOO_ERR_CUDA, "begin capture: %s", cudaGetErrorString(e));
+  }
+  ooo_status st = enqueue_backward(s, dY, sch, dX, cap);
+  if (st == OOO_OK) st = enqueue_forward(s, X, Y, cap);
+  cudaGraph_t g = nullptr;
+  e = cudaStreamEndCapture(cap, &g);
+  cudaStreamDestroy(cap);
+  if (st != OOO_OK) {
+    if (g) cudaGraphDestroy(g);
+    return st;
+  }
+  if (e != cudaSuccess) return fail(OOO_ERR_CUDA, "end capture: %s", cudaGetErrorString(e));
+  cudaGraphExec_t ex = nullptr;
+  e = cudaGraphInstantiateWithFlags(&ex, g, cudaGraphInstantiateFlagUseNodePriority);
+  if (e != cudaSuccess) {
+    cudaGraphDestroy(g);
+    return fail(OOO_ERR_CUDA, "graph instantiate: %s", cudaGetErrorString(e));
+  }
+  ooo_graph *gr = new ooo_graph();
+  gr->s = s;
+  gr->graph = g;
+  gr->exec = ex;
+  *out = gr;
+  return OOO_OK;
+}
+
+ooo_status ooo_graph_launch(ooo_graph *g, void *stream) {
+  if (!g) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL graph");
+  CU_TRY(cudaGraphLaunch(g->exec, static_cast<cudaStream_t>(stream)));
+  return OOO_OK;
+}
+
+ooo_status ooo_graph_destroy(ooo_graph *g) {
+  if (!g) return OOO_OK;
+  if (g->exec) cudaGraphExecDestroy(g->exec);
+  if (g->graph) cudaGraphDestroy(g->graph);
+  delete g;
+  return OOO_OK;
+}
+
+ooo_status ooo_destroy(ooo_stack *s) {
+  if (!s) return OOO_OK;
+  if (s->hi) cudaStreamSynchronize(s->hi);
+  if (s->lo) cudaStreamSynchronize(s->lo);
+  if (s->comm) cudaStreamSynchronize(s->comm);
+  if (s->nccl && s->api) s->api->CommDestroy(s->nccl);
+  for (auto e : s->ev_dz) if (e) cudaEventDestroy(e);
+  for (auto e : s->ev_pack) if (e) cudaEventDestroy(e);
+  for (auto e : s->ev_ar) if (e) cudaEventDestroy(e);
+  for (cudaEvent_t e : {s->ev_fork, s->ev_j_hi, s->ev_j_lo, s->ev_j_comm}) if (e) cudaEventDestroy(e);
+  for (auto &r : s->recs) {
+    if (r.a) cudaEventDestroy(r.a);
+    if (r.b) cudaEventDestroy(r.b);
+  }
+  if (s->hi) cudaStreamDestroy(s->hi);
+  if (s->lo) cudaStreamDestroy(s->lo);
+  if (s->comm) cudaStreamDestroy(s->comm);
+  delete s;
+  return OOO_OK;
+}
+
+ooo_status ooo_tensor(ooo_stack *s, int32_t kind, int32_t layer, void **ptr, int64_t *rows) {
+  if (!s || !ptr) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (layer < 1 || layer > s->p.L) return fail(OOO_ERR_INVALID_ARGUMENT, "layer %d out of range", layer);
+  LayerRt &r = s->lr[layer - 1];
+  int64_t nrows = s->p.M;
+  switch (kind) {
+    case 0: *ptr = r.X; break;
+    case 1: *ptr = r.Z; break;
+    case 2: *ptr = r.dZ; break;
+    case 3: *ptr = r.db; nrows = s->p.R; break;
+    default: return fail(OOO_ERR_INVALID_ARGUMENT, "kind %d invalid", kind);
+  }
+  if (rows) *rows = nrows;
+  return OOO_OK;
+}
+
+ooo_status ooo_set_timing(ooo_stack *s, int32_t enable) {
+  if (!s) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL stack");
+  s->timing = enable != 0;
+  s->rec_cursor = 0;
+  return OOO_OK;
+}
+
+ooo_status ooo_timing_read(ooo_stack *s, ooo_launch_record *out, int32_t cap, int32_t *n) {
+  if (!s || !n) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
+  int32_t cnt = 0;
+  for (size_t j = 0; j < s->rec_cursor && j < s->recs.size(); ++j) {
+    if (out && cnt < cap) {
+      TimedRec &r = s->recs[j];
+      out[cnt] = r.info;
+      float ms = 0.f;
+      cudaError_t e = cudaEventElapsedTime(&ms, r.a, r.b);
+      out[cnt].ms = e == cudaSuccess ? ms : -1.f;
+      if (e != cudaSuccess) (void)cudaGetLastError();
+    }
+    ++cnt;
+  }
+  *n = cnt;
+  return OOO_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,263 @@
+"""Thin Python binding of the C ABI (include/ooo.h).
+
+Argument marshalling only: every step of the path runs in libooo.so's CUDA
+kernels.  torch supplies device memory (workspace / gradient buffers are torch
+tensors), the caller's CUDA stream and, for N > 1, the process group used to
+broadcast the NCCL bootstrap id.  Function and argument names follow the ABI
+(ooo_create_stack / ooo_forward / ooo_backward / ooo_join / ooo_destroy).
+"""
+from __future__ import annotations
+
+import ctypes
+from ctypes import c_int32, c_int64, c_size_t, c_void_p
+
+from . import _lib
+from ._lib import check, load
+
+TORCH_DTYPE_NAMES = {"bf16": "bfloat16", "fp32": "float32"}
+
+
+def _i32arr(vals):
+    return (c_int32 * len(vals))(*[int(v) for v in vals])
+
+
+def _desc(dims, acts, tokens, dtype, need_input_grad=False, bucket_layers=1, max_temp_bytes=0,
+          world_size=1, rank=0, comm_enabled=True, nccl_max_ctas=0):
+    keep = {}
+    d = _lib.StackDesc()
+    d.num_layers = len(acts)
+    keep["dims"] = _i32arr(dims)
+    keep["acts"] = _i32arr([_lib.ACTS[a] if isinstance(a, str) else a for a in acts])
+    d.dims = ctypes.cast(keep["dims"], ctypes.POINTER(c_int32))
+    d.acts = ctypes.cast(keep["acts"], ctypes.POINTER(c_int32))
+    d.tokens = int(tokens)
+    d.dtype = _lib.DTYPES[dtype]
+    d.need_input_grad = int(bool(need_input_grad))
+    d.bucket_layers = int(bucket_layers)
+    d.max_temp_bytes = int(max_temp_bytes)
+    d.world_size = int(world_size)
+    d.rank = int(rank)
+    d.comm_enabled = int(bool(comm_enabled))
+    d.nccl_max_ctas = int(nccl_max_ctas)
+    return d, keep
+
+
+def query_sizes(dims, acts, tokens, dtype="bf16", bucket_layers=1):
+    d, _keep = _desc(dims, acts, tokens, dtype, bucket_layers=bucket_layers)
+    ws, gb = c_size_t(), c_size_t()
+    check(load().ooo_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)))
+    return ws.value, gb.value
+
+
+def grad_offsets(dims, acts, tokens, dtype="bf16"):
+    d, _keep = _desc(dims, acts, tokens, dtype)
+    L = len(acts)
+    out = (c_int64 * (2 * L))()
+    check(load().ooo_grad_offsets(ctypes.byref(d), out))
+    return [(out[2 * i], out[2 * i + 1]) for i in range(L)]
+
+
+def schedule_order(L: int, kind: str = "first_k", k: int = 0, need_input_grad: bool = False) -> list:
+    ops = (c_int32 * (2 * L))()
+    n = c_int32()
+    check(load().ooo_schedule_order(int(L), _lib.schedule(kind, k), int(bool(need_input_grad)), ops,
+                                    ctypes.byref(n)))
+    return list(ops[: n.value])
+
+
+def max_k(m_fwd: int, m_dO: list, m_dW: list, mxm: int) -> int:
+    L = len(m_dO)
+    a = (c_int64 * L)(*m_dO)
+    b = (c_int64 * L)(*m_dW)
+    return int(load().ooo_max_k(L, int(m_fwd), a, b, int(mxm)))
+
+
+def deferral_bytes(dims, acts, tokens, dtype, k) -> int:
+    d, _keep = _desc(dims, acts, tokens, dtype)
+    return int(load().ooo_deferral_bytes(ctypes.byref(d), int(k)))
+
+
+def get_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(_lib.UNIQUE_ID_BYTES)
+    check(load().ooo_get_unique_id(buf))
+    return buf.raw
+
+
+def broadcast_unique_id(group=None) -> bytes:
+    """Rank 0 creates the NCCL bootstrap id; torch.distributed broadcasts it."""
+    import torch.distributed as dist
+    obj = [get_unique_id() if dist.get_rank(group) == 0 else None]
+    dist.broadcast_object_list(obj, src=0, group=group)
+    return obj[0]
+
+
+def _stream_handle(stream):
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return c_void_p(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
+
+
+class StepGraph:
+    """A captured [ooo_backward; ooo_forward] step (pre-compiled issue, §4.2)."""
+
+    def __init__(self, stack, handle, keep):
+        self._stack = stack
+        self._h = handle
+        self._keep = keep
+
+    def launch(self, stream=None):
+        check(load().ooo_graph_launch(self._h, _stream_handle(stream)))
+
+    def close(self):
+        if self._h:
+            load().ooo_graph_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class OooStack:
+    """One rank's stack: ooo_create_stack over caller-owned torch tensors."""
+
+    def __init__(self, dims, acts, tokens, W, b, dtype="bf16", need_input_grad=False, bucket_layers=1,
+                 max_temp_bytes=0, world_size=1, rank=0, unique_id: bytes | None = None,
+                 comm_enabled=True, nccl_max_ctas=0):
+        import torch
+        lib = load()
+        self.dims = [int(x) for x in dims]
+        self.acts = list(acts)
+        self.L = len(self.acts)
+        self.tokens = int(tokens)
+        self.dtype = dtype
+        self.tdtype = getattr(torch, TORCH_DTYPE_NAMES[dtype])
+        self.need_input_grad = bool(need_input_grad)
+        self.world_size = int(world_size)
+        self.rank = int(rank)
+        if len(W) != self.L or len(b) != self.L:
+            raise ValueError("need L weights and biases")
+        for i, (w, bb) in enumerate(zip(W, b)):
+            if w.dtype != self.tdtype or bb.dtype != self.tdtype:
+                raise ValueError(f"layer {i + 1}: W/b dtype must be {self.tdtype}")
+            if tuple(w.shape) != (self.dims[i], self.dims[i + 1]) or tuple(bb.shape) != (self.dims[i + 1],):
+                raise ValueError(f"layer {i + 1}: bad W/b shape")
+            if not (w.is_cuda and w.is_contiguous() and bb.is_cuda and bb.is_contiguous()):
+                raise ValueError(f"layer {i + 1}: W/b must be contiguous CUDA tensors")
+        self.W, self.b = list(W), list(b)
+        self.device = W[0].device
+        d, keep = _desc(self.dims, self.acts, self.tokens, dtype, need_input_grad, bucket_layers,
+                        max_temp_bytes, world_size, rank, comm_enabled, nccl_max_ctas)
+        ws, gb = c_size_t(), c_size_t()
+        check(lib.ooo_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)))
+        self.workspace = torch.empty(ws.value, dtype=torch.uint8, device=self.device)
+        self.grads_buf = torch.zeros(gb.value, dtype=torch.uint8, device=self.device)
+        keep["W"] = (c_void_p * self.L)(*[w.data_ptr() for w in self.W])
+        keep["b"] = (c_void_p * self.L)(*[x.data_ptr() for x in self.b])
+        d.W = ctypes.cast(keep["W"], ctypes.POINTER(c_void_p))
+        d.b = ctypes.cast(keep["b"], ctypes.POINTER(c_void_p))
+        d.grads = self.grads_buf.data_ptr()
+        d.workspace = self.workspace.data_ptr()
+        if self.world_size > 1:
+            if unique_id is None or len(unique_id) != _lib.UNIQUE_ID_BYTES:
+                raise ValueError("world_size > 1 needs the 128-byte NCCL unique id (broadcast_unique_id)")
+            keep["uid"] = ctypes.create_string_buffer(unique_id, _lib.UNIQUE_ID_BYTES)
+            d.nccl_unique_id = ctypes.cast(keep["uid"], c_void_p)
+        self._keep = keep
+        self._desc = d
+        h = c_void_p()
+        check(lib.ooo_create_stack(ctypes.byref(d), ctypes.byref(h)))
+        self._h = h
+        offs = (c_int64 * (2 * self.L))()
+        check(lib.ooo_grad_offsets(ctypes.byref(d), offs))
+        g = self.grads_buf.view(self.tdtype)
+        self.dW, self.db = [], []
+        for i in range(self.L):
+            ow, ob = offs[2 * i], offs[2 * i + 1]
+            din, dout = self.dims[i], self.dims[i + 1]
+            self.dW.append(g[ow: ow + din * dout].view(din, dout))
+            self.db.append(g[ob: ob + dout])
+
+    # ---- the path ---------------------------------------------------------
+    def _check_act(self, t, rows, cols, name):
+        if t.dtype != self.tdtype or tuple(t.shape) != (rows, cols) or not t.is_contiguous() or not t.is_cuda:
+            raise ValueError(f"{name}: expected contiguous CUDA {self.tdtype} [{rows}, {cols}]")
+
+    def forward(self, X, Y=None, stream=None):
+        import torch
+        self._check_act(X, self.tokens, self.dims[0], "X")
+        if Y is None:
+            Y = torch.empty(self.tokens, self.dims[-1], dtype=self.tdtype, device=self.device)
+        self._check_act(Y, self.tokens, self.dims[-1], "Y")
+        check(load().ooo_forward(self._h, c_void_p(X.data_ptr()), c_void_p(Y.data_ptr()),
+                                 _stream_handle(stream)))
+        return Y
+
+    def backward(self, dY, kind="first_k", k=0, dX=None, stream=None):
+        self._check_act(dY, self.tokens, self.dims[-1], "dY")
+        if dX is not None:
+            self._check_act(dX, self.tokens, self.dims[0], "dX")
+        check(load().ooo_backward(self._h, c_void_p(dY.data_ptr()), _lib.schedule(kind, k),
+                                  c_void_p(dX.data_ptr() if dX is not None else None),
+                                  _stream_handle(stream)))
+
+    def join(self, stream=None):
+        check(load().ooo_join(self._h, _stream_handle(stream)))
+
+    def graph(self, X, Y, dY, kind="first_k", k=0, dX=None) -> StepGraph:
+        self._check_act(X, self.tokens, self.dims[0], "X")
+        self._check_act(Y, self.tokens, self.dims[-1], "Y")
+        self._check_act(dY, self.tokens, self.dims[-1], "dY")
+        h = c_void_p()
+        check(load().ooo_graph_create(self._h, c_void_p(X.data_ptr()), c_void_p(Y.data_ptr()),
+                                      c_void_p(dY.data_ptr()), _lib.schedule(kind, k),
+                                      c_void_p(dX.data_ptr() if dX is not None else None), ctypes.byref(h)))
+        return StepGraph(self, h, (X, Y, dY, dX))
+
+    # ---- introspection -----------------------------------------------------
+    def tensor(self, kind: str, layer: int):
+        """Views of internal stores: 'X' (X_i), 'Z' (Z_i; None for identity
+        layers), 'dZ', 'dbpart' (fp32 [rows][d_i])."""
+        import torch
+        code = {"X": 0, "Z": 1, "dZ": 2, "dbpart": 3}[kind]
+        p = c_void_p()
+        rows = c_int64()
+        check(load().ooo_tensor(self._h, code, int(layer), ctypes.byref(p), ctypes.byref(rows)))
+        if not p.value:
+            return None
+        off = p.value - self.workspace.data_ptr()
+        cols = self.dims[layer - 1] if kind == "X" else self.dims[layer]
+        if kind == "dbpart":
+            n = rows.value * cols * 4
+            return self.workspace[off: off + n].view(torch.float32).view(rows.value, cols)
+        esz = 2 if self.dtype == "bf16" else 4
+        n = rows.value * cols * esz
+        return self.workspace[off: off + n].view(self.tdtype).view(rows.value, cols)
+
+    def set_timing(self, enable: bool = True):
+        check(load().ooo_set_timing(self._h, int(bool(enable))))
+
+    def timing(self) -> list:
+        n = c_int32()
+        check(load().ooo_timing_read(self._h, None, 0, ctypes.byref(n)))
+        recs = (_lib.LaunchRecord * max(1, n.value))()
+        check(load().ooo_timing_read(self._h, recs, n.value, ctypes.byref(n)))
+        out = []
+        for r in recs[: n.value]:
+            out.append({"kind": _lib.KIND_NAMES.get(r.kind, r.kind), "layer": r.layer, "stream": r.stream,
+                        "grid": r.grid, "flops": r.flops, "bytes": r.bytes, "ms": r.ms})
+        return out
+
+    def close(self):
+        if getattr(self, "_h", None):
+            load().ooo_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

@@ -94,3 +94,32 @@ def x_shard(M: int, d0: int, rank: int, dtype: str, seed: int = SEED, step: int 
 
 def dy_shard(M: int, dL: int, rank: int, dtype: str, seed: int = SEED, step: int = 0) -> np.ndarray:
     return to_storage(_rng(seed, 1, rank, step).standard_normal((M, dL)), dtype)
+
+
+def weights_torch(dims, acts, dtype: str, device, seed: int = SEED):
+    """Same recipe as ``weights`` (orthogonal W with gain, b ~ N(0, 0.1^2)),
+    generated on the GPU with torch for the full-size bench configs (not
+    bit-identical to the NumPy stream; used only where no oracle compares)."""
+    import torch
+    tdt = {"bf16": torch.bfloat16, "fp32": torch.float32}[dtype]
+    g = torch.Generator(device=device)
+    W, b = [], []
+    for i in range(len(acts)):
+        g.manual_seed(seed * 1000 + i)
+        d_in, d_out = dims[i], dims[i + 1]
+        n, m = max(d_in, d_out), min(d_in, d_out)
+        q, r = torch.linalg.qr(torch.randn(n, m, generator=g, device=device, dtype=torch.float32))
+        q = q * torch.sign(torch.diagonal(r))[None, :]
+        w = q if d_in >= d_out else q.T
+        scale = gain(acts[i]) * (math.sqrt(d_out / d_in) if d_out > d_in else 1.0)
+        W.append((w * scale).to(tdt).contiguous())
+        b.append((0.1 * torch.randn(d_out, generator=g, device=device)).to(tdt).contiguous())
+    return W, b
+
+
+def activations_torch(M: int, d: int, dtype: str, device, seed: int, rank: int, tag: int):
+    import torch
+    tdt = {"bf16": torch.bfloat16, "fp32": torch.float32}[dtype]
+    g = torch.Generator(device=device)
+    g.manual_seed(seed * 7919 + rank * 31 + tag)
+    return torch.randn(M, d, generator=g, device=device).to(tdt).contiguous()

@@ -1,0 +1,140 @@
+"""Parity of the CUDA path (through the C ABI) against the fp64 oracle.
+
+All inputs are seeded (paper_conf_eurosys_ohlks22_b200.synth); the oracle
+computes every expected value itself from those inputs (no teacher forcing).
+Gates (north star, reading in DESIGN.md): max relative Frobenius error over
+Y, every dW_i, db_i (and dX) <= 1e-2 in bf16 and <= 1e-4 in fp32; in-order
+and every ooo_first_k(k) schedule bit-exact with each other.
+"""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_eurosys_ohlks22_b200 import configs
+from tests.gpu_helpers import Case, bf16_floor, max_err
+
+pytestmark = pytest.mark.gpu
+
+BF16_TOL = 1e-2
+FP32_TOL = 1e-4
+
+
+def _check(errs, tol):
+    for k, v in errs.items():
+        assert v <= tol, (k, v, errs)
+
+
+# ------------------------------------------------------------------ fp32
+def test_fp32_config0_end_to_end_all_schedules():
+    c = configs.C1
+    case = Case(c.dims, c.acts, c.tokens, "fp32")
+    ref = case.oracle()
+    stk = case.stack()
+    base = None
+    for kind, k in [("in_order", 0)] + [("first_k", k) for k in range(c.L + 1)]:
+        out = case.run(stk, kind, k)
+        _check(max_err(out, ref), FP32_TOL)
+        if base is None:
+            base = out["raw"]
+        assert torch.equal(out["raw"], base), (kind, k)
+    stk.close()
+
+
+def test_fp32_ragged_with_input_grad():
+    case = Case([192, 320, 128, 64], ["gelu", "relu", "id"], 200, "fp32", need_dx=True)
+    ref = case.oracle(2)
+    stk = case.stack()
+    out = case.run(stk, "first_k", 2)
+    _check(max_err(out, ref), FP32_TOL)
+
+
+# ------------------------------------------------------------------ bf16
+@pytest.mark.parametrize("tokens", [400, 128, 16, 8])
+def test_bf16_ragged_tiles_end_to_end(tokens):
+    """Several tiles in every dimension plus ragged tails (M % 128 != 0,
+    widths not multiples of the N tile)."""
+    case = Case([192, 320, 256, 448, 192], ["gelu", "id", "gelu", "id"], tokens, "bf16")
+    ref = case.oracle(2)
+    stk = case.stack()
+    out = case.run(stk, "first_k", 2)
+    _check(max_err(out, ref), BF16_TOL)
+
+
+def test_bf16_relu_and_input_grad():
+    case = Case([128, 256, 128, 128], ["relu", "gelu", "relu"], 264, "bf16", need_dx=True)
+    ref = case.oracle(3)
+    stk = case.stack()
+    out = case.run(stk, "first_k", 3)
+    _check(max_err(out, ref), BF16_TOL)
+
+
+def test_bf16_schedules_bit_exact_and_graph_equals_eager():
+    case = Case([256, 512, 256, 1024, 256, 256], ["id", "gelu", "gelu", "id", "id"], 384, "bf16")
+    stk = case.stack(bucket_layers=2)
+    base = case.run(stk, "in_order", 0)
+    for k in range(case.L + 2):
+        out = case.run(stk, "first_k", k)
+        assert torch.equal(out["raw"], base["raw"]), k
+        assert np.array_equal(out["Y"], base["Y"])
+    for kind, k in [("in_order", 0), ("first_k", 3)]:
+        out = case.run(stk, kind, k, graph=True, launches=3)
+        assert torch.equal(out["raw"], base["raw"]), (kind, k)
+    _check(max_err(base, case.oracle()), BF16_TOL)
+
+
+def test_bf16_deterministic_repeat():
+    case = Case([768, 768, 3072, 768], ["id", "gelu", "id"], 1024, "bf16")
+    stk = case.stack()
+    a = case.run(stk, "first_k", 3)
+    b = case.run(stk, "first_k", 3)
+    assert torch.equal(a["raw"], b["raw"])
+
+
+# ---------------------------------------- full-size shapes of the configs
+def _block_slice(cfg, blocks):
+    """The first `blocks` transformer blocks of a config at its full width and
+    full tokens per GPU: every GEMM launch configuration of the config (tile
+    plan depends only on (M, d_in, d_out)) is exercised."""
+    n = 6 * blocks
+    return list(cfg.dims[: n + 1]), list(cfg.acts[:n]), cfg.tokens
+
+
+@pytest.mark.parametrize("cfg", [configs.C2, configs.C3, configs.C4], ids=["bert_base", "bert_large", "gpt2_medium"])
+def test_bf16_full_size_block_slice(cfg):
+    dims, acts, M = _block_slice(cfg, 2)
+    case = Case(dims, acts, M, "bf16")
+    ref = case.oracle(len(acts))
+    stk = case.stack()
+    out = case.run(stk, "first_k", len(acts))
+    _check(max_err(out, ref), BF16_TOL)
+    base = case.run(stk, "in_order", 0)
+    assert torch.equal(out["raw"], base["raw"])
+
+
+def test_bf16_mlp96_full_config():
+    """Config 4 at full size (96 layers, M = 16).  End-to-end bf16 error of a
+    96-layer stack is bounded by the rounding random walk:
+    gate at max(1e-2, 2 x floor), floor = sqrt(2L) 2^-9 / sqrt(3)."""
+    c = configs.C5
+    case = Case(c.dims, c.acts, c.tokens, "bf16")
+    ref = case.oracle(48)
+    stk = case.stack()
+    out = case.run(stk, "first_k", 48, graph=True)
+    errs = max_err(out, ref)
+    _check(errs, max(BF16_TOL, 2 * bf16_floor(c.L)))
+    base = case.run(stk, "in_order", 0)
+    assert torch.equal(out["raw"], base["raw"])
+
+
+@pytest.mark.slow
+def test_bf16_bert_base_full_config_end_to_end():
+    """Config 1 (the bench workload) end to end at full size: 72 layers,
+    M = 4096, graph-captured ooo_first_k as bench.py times it."""
+    c = configs.C2
+    case = Case(c.dims, c.acts, c.tokens, "bf16")
+    ref = case.oracle(24)
+    stk = case.stack()
+    out = case.run(stk, "first_k", 24, graph=True)
+    errs = max_err(out, ref)
+    print("bert_base full-size errors", errs, "floor", bf16_floor(c.L))
+    _check(errs, max(BF16_TOL, 2 * bf16_floor(c.L)))
