@@ -1,0 +1,451 @@
+#!/usr/bin/env python
+"""Benchmark of the ooo-backprop data-parallel hot path (one JSON line).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--k auto|INT]
+    torchrun --nproc-per-node N bench.py --gpus N ...     (N > 1, NCCL)
+    python bench.py --impl reference ...                   (the CPU oracle arm)
+
+A step = one training iteration of the paper's problem statement (§2,
+P:81-95): backward(t) of the whole dense stack (dO chain on the high-priority
+stream, dW ops in Algorithm 2 "reverse first-k" order on the low-priority
+stream, one NCCL all-reduce per gradient bucket) followed by forward(t+1),
+each F_i gated on its layer's synchronised gradient -- captured once as a
+CUDA graph (pre-compiled issue, §4.2) and replayed.  Inputs are synthetic
+(seeded, shaped like BASELINE.json's configs; reading Q13) and resident in
+HBM for `value`; `e2e` adds the per-step host->device copy of X, dY and the
+device->host read of Y through the same public API.
+
+The oracle (oracle/) is imported only by the cpu_baseline leg and by
+--impl reference.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "train iters/sec at 1/2/4/8 B200; exposed allreduce ms/iter; ooo vs in-order"
+UNIT = "iters/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="C2", help="C1..C5 or a config name (default: configs[1] = BERT-base stack)")
+    ap.add_argument("--k", default="auto", help="reverse first-k parameter, or 'auto' (paper's search, P:212-214)")
+    ap.add_argument("--bucket-layers", type=int, default=1)
+    ap.add_argument("--nccl-max-ctas", type=int, default=0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-sample-tokens", type=int, default=0)
+    return ap.parse_args()
+
+
+# --------------------------------------------------------------- helpers
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return {"hbm_gbs": d["hbm_gbs"], "bf16_tflops": d["bf16_tflops"],
+                "bf16_tflops_sustained": d.get("bf16_tflops_sustained", d["bf16_tflops"]), "source": "measured"}
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0, "source": "fallback"}
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.p = None
+
+    def __enter__(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                                       "-lms", "100", "-i", str(self.gpu)],
+                                      stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.p = None
+        return self
+
+    def __exit__(self, *a):
+        self.lines = []
+        if self.p is not None:
+            time.sleep(0.15)
+            self.p.terminate()
+            try:
+                out, _ = self.p.communicate(timeout=5)
+            except Exception:
+                self.p.kill()
+                out = ""
+            self.lines = [l for l in out.splitlines() if l.strip()]
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in self.lines:
+            f = [x.strip() for x in l.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx = float(f[2])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[5:9]):
+                if v.lower() == "active":
+                    reasons.add(n)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        loaded = [x for x in sm if x > 0.5 * max(sm)] or sm
+        return {"sm_mhz": statistics.median(loaded), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def dist_setup(args):
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        if world == 1 and args.gpus > 1:
+            raise SystemExit("--gpus N > 1 must be launched with torchrun --nproc-per-node N")
+    return world, rank, local
+
+
+def time_cpu_oracle(cfg, sample_tokens: int):
+    """The fp64 oracle (bf16 storage mode) as it stands, one forward+backward
+    of `sample_tokens` rows of this config; returns (seconds, threads)."""
+    import numpy as np
+    from oracle import layers as O
+    from oracle import schedule as S
+    from paper_conf_eurosys_ohlks22_b200 import synth
+    try:
+        from threadpoolctl import threadpool_info
+        threads = max((i.get("num_threads", 1) for i in threadpool_info()), default=1)
+    except Exception:
+        threads = len(os.sched_getaffinity(0))
+    rng = np.random.default_rng(1)
+    dt = "bf16" if cfg.dtype == "bf16" else "fp32"
+    W = [synth.to_storage(rng.standard_normal((cfg.dims[i], cfg.dims[i + 1])) / math.sqrt(cfg.dims[i]), dt)
+         for i in range(cfg.L)]
+    b = [synth.to_storage(0.1 * rng.standard_normal(cfg.dims[i + 1]), dt) for i in range(cfg.L)]
+    X = synth.x_shard(sample_tokens, cfg.dims[0], 0, dt)
+    dY = synth.dy_shard(sample_tokens, cfg.dims[-1], 0, dt)
+    D = S.reverse_first_k(cfg.L, cfg.L)
+    t0 = time.perf_counter()
+    O.dp_step([X], [dY], W, b, list(cfg.acts), D, "bf16" if cfg.dtype == "bf16" else "fp64")
+    return time.perf_counter() - t0, threads
+
+
+def cpu_sample_tokens(cfg, requested):
+    if requested:
+        return requested
+    # aim at ~10-30 s of fp64 work on a few host cores: ~2.5e11 FLOP
+    per_token = cfg.gemm_flops() / cfg.tokens
+    t = int(2.5e11 / per_token) // 8 * 8
+    return max(8, min(cfg.tokens, t))
+
+
+# ---------------------------------------------------------- reference arm
+def run_reference(args):
+    world, rank, _ = dist_setup(args)
+    if rank != 0:
+        return
+    from paper_conf_eurosys_ohlks22_b200 import configs
+    cfg = configs.get(args.config)
+    tok = cpu_sample_tokens(cfg, args.cpu_sample_tokens)
+    steps = max(1, min(args.steps, 3))
+    for _ in range(min(args.warmup, 1)):
+        time_cpu_oracle(cfg, min(tok, 64))
+    times = []
+    threads = 1
+    for _ in range(steps):
+        t, threads = time_cpu_oracle(cfg, tok)
+        times.append(t)
+    sec = statistics.mean(times)
+    value = (tok / cfg.tokens) / sec        # full-config iterations per second (scaled)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": steps, "warmup": min(args.warmup, 1), "ms_per_step": 1e3 / value, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"{cfg.name} ({cfg.note})", "tokens_per_gpu": cfg.tokens, "layers": cfg.L,
+                   "parallelism": f"dp{args.gpus}"},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
+                         "sample": f"one fp64 forward+backward of {tok} of {cfg.tokens} tokens/GPU, "
+                                   f"scaled by {tok}/{cfg.tokens}; {steps} step(s), mean"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ------------------------------------------------------------------ ours
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    import torch
+    import torch.distributed as dist
+    from paper_conf_eurosys_ohlks22_b200 import configs, synth
+    from paper_conf_eurosys_ohlks22_b200.stack import OooStack, broadcast_unique_id
+
+    world, rank, local = dist_setup(args)
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    cfg = configs.get(args.config)
+    dt = cfg.dtype
+    M = cfg.tokens
+    peaks = load_peaks()
+
+    W, b = synth.weights_torch(cfg.dims, cfg.acts, dt, dev)
+    uid = broadcast_unique_id() if world > 1 else None
+    stk = OooStack(cfg.dims, cfg.acts, M, W, b, dtype=dt, bucket_layers=args.bucket_layers,
+                   world_size=world, rank=rank, unique_id=uid, nccl_max_ctas=args.nccl_max_ctas)
+    X = synth.activations_torch(M, cfg.dims[0], dt, dev, synth.SEED, rank, 0)
+    dY = synth.activations_torch(M, cfg.dims[-1], dt, dev, synth.SEED, rank, 1)
+    Y = torch.empty(M, cfg.dims[-1], dtype=X.dtype, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def timed(graph, steps, sampler=None):
+        barrier()
+        torch.cuda.synchronize()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        if sampler:
+            sampler.__enter__()
+            time.sleep(0.2)
+        e0.record(stream)
+        for _ in range(steps):
+            graph.launch(stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        if sampler:
+            sampler.__exit__(None, None, None)
+        barrier()
+        return max_over_ranks(e0.elapsed_time(e1) / steps)
+
+    stk.forward(X, Y)
+    torch.cuda.synchronize()
+    graphs = {}
+
+    def graph_for(kind, k, s=stk):
+        key = (id(s), kind, k)
+        if key not in graphs:
+            graphs[key] = s.graph(X, Y, dY, kind, k)
+        return graphs[key]
+
+    # ---- choose k: the paper's heuristic search (§5.1) on measured throughput
+    L = cfg.L
+    if args.k == "auto":
+        from paper_conf_eurosys_ohlks22_b200.ksearch import search_k
+        probe = max(5, min(20, args.steps // 2))
+
+        def tput(k):
+            g = graph_for("first_k", k)
+            for _ in range(2):
+                g.launch(stream)
+            return 1e3 / timed(g, probe)
+        k_best, visited = search_k(L, tput)
+    else:
+        k_best, visited = int(args.k), []
+    g_ooo = graph_for("first_k", k_best)
+    g_in = graph_for("in_order", 0)
+    for _ in range(max(3, args.warmup)):
+        g_ooo.launch(stream)
+        g_in.launch(stream)
+    torch.cuda.synchronize()
+
+    sampler = ClockSampler(local)
+    ms_ooo = timed(g_ooo, args.steps, sampler)
+    clocks = sampler.summary()
+    ms_in = timed(g_in, args.steps)
+
+    # ---- exposed communication: same graph with the all-reduce skipped (comm-off control)
+    exposed = None
+    ar_ms = None
+    if world > 1:
+        stk_off = OooStack(cfg.dims, cfg.acts, M, W, b, dtype=dt, bucket_layers=args.bucket_layers,
+                           world_size=world, rank=rank, unique_id=broadcast_unique_id(), comm_enabled=False)
+        stk_off.forward(X, Y)
+        g_off = stk_off.graph(X, Y, dY, "first_k", k_best)
+        for _ in range(3):
+            g_off.launch(stream)
+        ms_off = timed(g_off, args.steps)
+        exposed = {"ooo_first_k": ms_ooo - ms_off}
+        g_off_in = stk_off.graph(X, Y, dY, "in_order", 0)
+        for _ in range(3):
+            g_off_in.launch(stream)
+        exposed["in_order"] = ms_in - timed(g_off_in, args.steps)
+        # standalone all-reduce time: every bucket back to back, no compute
+        views = []
+        for i in range(L):
+            views.append(stk.dW[i].view(-1))
+            views.append(stk.db[i])
+        torch.cuda.synchronize()
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        reps = 5
+        e0.record(stream)
+        for _ in range(reps):
+            for v in views:
+                dist.all_reduce(v)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        ar_ms = max_over_ranks(e0.elapsed_time(e1) / reps)
+        g_off.close()
+        g_off_in.close()
+        stk_off.close()
+
+    # ---- per-kernel durations: instrumented replay of the same step (CUDA events per launch)
+    stk.set_timing(True)
+    g_t = stk.graph(X, Y, dY, "first_k", k_best)
+    for _ in range(3):
+        g_t.launch(stream)
+    ms_timed = timed(g_t, max(3, args.steps // 2))
+    recs = stk.timing()
+    g_t.close()
+    stk.set_timing(False)
+    by_kind = {}
+    for r in recs:
+        d = by_kind.setdefault(r["kind"], {"ms": 0.0, "flops": 0.0, "bytes": 0.0, "n": 0})
+        d["ms"] += max(r["ms"], 0.0)
+        d["flops"] += r["flops"]
+        d["bytes"] += r["bytes"]
+        d["n"] += 1
+    ours = {k: v for k, v in by_kind.items() if k not in ("allreduce", "copy")}
+    dom = max(ours, key=lambda k: ours[k]["ms"])
+    dd = ours[dom]
+    launches_per_step = sum(v["n"] for v in ours.values())
+    if dd["flops"] > 0:
+        achieved = dd["flops"] / (dd["ms"] * 1e-3) / 1e12
+        peak = peaks["bf16_tflops_sustained"] if dt == "bf16" else 75.0
+        roof = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak}
+    else:
+        achieved = dd["bytes"] / (dd["ms"] * 1e-3) / 1e9
+        peak = peaks["hbm_gbs"]
+        roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak}
+    roof["kernel"] = dom
+    roof["launches_per_step"] = dd["n"]
+    roof["avg_launch_us"] = dd["ms"] * 1e3 / max(1, dd["n"])
+    roof["share_of_step"] = dd["ms"] / ms_timed
+    roof["peak_source"] = f"{peaks['source']} ({'bf16_tflops_sustained' if dd['flops'] > 0 else 'hbm_gbs'})"
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        try:
+            tr = json.load(open(tp))
+            traffic = tr.get(cfg.name, {}).get(dom)
+        except Exception:
+            traffic = None
+    roof["traffic"] = traffic
+
+    # ---- north-star roofline of the whole step: max(GEMM FLOP at peak, ring AR bytes at link bw)
+    flops = cfg.gemm_flops()
+    t_tensor = flops / (peaks["bf16_tflops_sustained"] * 1e12) * 1e3 if dt == "bf16" else None
+    grad_bytes = cfg.params() * (2 if dt == "bf16" else 4)
+    t_ar = 2 * (world - 1) / world * grad_bytes / 770e9 * 1e3 if world > 1 else 0.0
+    step_roof_ms = max(t_tensor or 0.0, t_ar)
+
+    # ---- e2e through the public API with host buffers
+    e2e = None
+    if not args.no_e2e:
+        hX = torch.empty(X.shape, dtype=X.dtype, pin_memory=True)
+        hdY = torch.empty(dY.shape, dtype=dY.dtype, pin_memory=True)
+        hY = torch.empty(Y.shape, dtype=Y.dtype, pin_memory=True)
+        hX.copy_(X.cpu())
+        hdY.copy_(dY.cpu())
+
+        def e2e_step():
+            X.copy_(hX, non_blocking=True)
+            dY.copy_(hdY, non_blocking=True)
+            g_ooo.launch(stream)
+            hY.copy_(Y, non_blocking=True)
+
+        for _ in range(3):
+            e2e_step()
+        barrier()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(args.steps):
+            e2e_step()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ms_e2e = max_over_ranks(e0.elapsed_time(e1) / args.steps)
+        ebytes = X.element_size()
+        e2e = {"value": 1e3 / ms_e2e, "unit": UNIT,
+               "h2d_bytes_per_step": (X.numel() + dY.numel()) * ebytes, "d2h_bytes_per_step": Y.numel() * ebytes}
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        tok = cpu_sample_tokens(cfg, args.cpu_sample_tokens)
+        sec, threads = time_cpu_oracle(cfg, tok)
+        cpu = {"value": (tok / M) / sec, "unit": UNIT, "cores": threads, "kind": "oracle",
+               "sample": f"one fp64 (bf16-storage) forward+backward of {tok} of {M} tokens of {cfg.name}, "
+                         f"{sec:.1f} s, scaled by {tok}/{M}"}
+
+    value = 1e3 / ms_ooo
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_ooo, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": dt, "data": "synthetic",
+        "config": {"workload": f"{cfg.name} ({cfg.note})", "layers": L, "tokens_per_gpu": M,
+                   "global_batch_tokens": M * world, "dims": f"{cfg.dims[0]}/{max(cfg.dims)}",
+                   "schedule": "ooo_first_k", "k": k_best, "k_search_visited": visited,
+                   "bucket_layers": args.bucket_layers, "parallelism": f"dp{world}",
+                   "l2": "working set (weights+activations+grads) >> 126 MB L2; no flush"},
+        "tokens_per_s": value * M * world,
+        "in_order": {"value": 1e3 / ms_in, "ms_per_step": ms_in},
+        "ooo_speedup_vs_in_order": ms_in / ms_ooo,
+        "exposed_allreduce_ms": exposed,
+        "allreduce_standalone_ms": ar_ms,
+        "hidden_fraction": (None if not exposed or not ar_ms else 1.0 - exposed["ooo_first_k"] / ar_ms),
+        "step_roofline": {"ms": step_roof_ms, "frac": step_roof_ms / ms_ooo if step_roof_ms else None,
+                          "tensor_ms": t_tensor, "allreduce_ms_at_770GBps": t_ar, "gemm_flops": flops},
+        "roofline": roof,
+        "kernels": {k: {"ms_per_step": v["ms"], "launches": v["n"]} for k, v in by_kind.items()},
+        "instrumented_ms_per_step": ms_timed,
+        "gpu_launches": launches_per_step * args.steps,
+        "clocks": clocks,
+        "e2e": e2e,
+        "cpu_baseline": cpu,
+    }
+    for g in graphs.values():
+        g.close()
+    stk.close()
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

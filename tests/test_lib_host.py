@@ -100,3 +100,20 @@ def test_sizes_offsets_and_deferral_bytes(lib):
     for k in (0, 1, 2, 10, 72):
         want = sum(c.tokens * c.dims[i] * 2 for i in range(2, min(k, c.L) + 1))
         assert stack.deferral_bytes(c.dims, c.acts, c.tokens, "bf16", k) == want
+
+
+def test_product_k_search_matches_oracle_reading():
+    """bench.py's k search (product side, P:212-214) and the oracle's
+    transcription are independent implementations of the same reading."""
+    import random
+    from paper_conf_eurosys_ohlks22_b200.ksearch import search_k
+    rng = random.Random(9)
+    for L in (5, 10, 24, 72, 144):
+        for _ in range(20):
+            vals = {k: rng.random() for k in range(L + 1)}
+            kp, visited = search_k(L, lambda k: vals[k])
+            ko = S.search_k(L, lambda k: vals[k])
+            assert kp == ko
+            assert len(set(visited)) == len(visited)
+        peak = rng.randint(0, L - 1)
+        assert search_k(L, lambda k: -abs(k - peak))[0] == peak
