@@ -214,6 +214,7 @@ typedef struct {
   double flops;       /* algorithmic FLOPs of the launch (GEMMs) */
   double bytes;       /* algorithmic HBM bytes of the launch (pack / seed / copy / all-reduce payload) */
   float ms;           /* event-measured duration */
+  float start_ms;     /* start relative to the first record's start (timeline) */
 } ooo_launch_record;
 ooo_status ooo_set_timing(ooo_stack *s, int32_t enable);
 ooo_status ooo_timing_read(ooo_stack *s, ooo_launch_record *out, int32_t cap, int32_t *n);

@@ -56,6 +56,7 @@ class LaunchRecord(ctypes.Structure):
         ("flops", c_double),
         ("bytes", c_double),
         ("ms", c_float),
+        ("start_ms", c_float),
     ]
 
 

@@ -8,12 +8,20 @@
 // (§7, tf.group removal; §4.1: the two GEMMs share only their
 // smaller inputs, so splitting them costs little locality).
 //
-// Structure (one 128 x BN output tile per CTA, non-persistent so that stream
-// priorities act at CTA-dispatch granularity):
+// Persistent, warp-specialised kernel: each CTA walks output tiles
+// t = blockIdx.x, blockIdx.x + gridDim.x, ... (128 x BN tiles, optional
+// split-K units), so the prologue (barrier init, TMEM alloc, descriptor
+// prefetch) is paid once per CTA and the epilogue of tile j overlaps the
+// mainloop of tile j+1 through a double-buffered TMEM accumulator:
 //   warp 0 lane 0 : TMA producer, STAGES-deep smem ring (128B swizzle)
-//   warp 1        : TMEM allocator; lane 0 issues tcgen05.mma (M=128, N=BN, K=16)
+//   warp 1        : TMEM allocator (2 x BN columns); lane 0 issues
+//                   tcgen05.mma (M=128, N=BN, K=16) into accumulator j&1
 //   warps 2..5    : epilogue -- tcgen05.ld 32x32b.x32 -> registers -> fused
 //                   bias / activation / act-grad / bias-grad / scale -> global
+// Programmatic dependent launch: every thread waits (griddepcontrol.wait)
+// for the previous kernel in the stream only after its prologue, and the
+// next kernel is released (launch_dependents) right away, so back-to-back
+// layer kernels overlap their launch + prologue with the predecessor's tail.
 // Operand majors: A K-major (X_i, dZ_i as A of F_i / dO_i) or MN-major
 // (X_i^T as A of dW_i); B MN-major (W_i in F_i, dZ_i in dW_i) or K-major
 // (W_i^T in dO_i).  16-bit types allow MN-major operands directly, so no
@@ -32,18 +40,22 @@ constexpr int BM = 128;
 constexpr int BK = 64;                 // 64 bf16 = 128 B = one swizzle row
 constexpr int A_BYTES = BM * BK * 2;   // 16 KiB
 constexpr int kThreads = 192;
+constexpr int kSmemBudget = 227 * 1024;
 
 template <int BN> struct Cfg {
   static constexpr int B_BYTES = BN * BK * 2;
   static constexpr int STAGE = A_BYTES + B_BYTES;
-  static constexpr int STAGES = (BN == 64) ? 8 : (BN == 128 ? 6 : 4);
+  static constexpr int STAGES_RAW = (kSmemBudget - 8 * 1024) / STAGE;
+  static constexpr int STAGES = STAGES_RAW > 8 ? 8 : STAGES_RAW;
   static constexpr int RING = STAGE * STAGES;
-  static constexpr int TMEM_COLS = BN < 32 ? 32 : BN;
-  // ring | full[STAGES] | empty[STAGES] | accum | tmem slot | db scratch [4][BN]
+  static constexpr int TMEM_COLS = (2 * BN <= 64) ? 64 : (2 * BN <= 128 ? 128 : (2 * BN <= 256 ? 256 : 512));
+  // ring | full[S] | empty[S] | tfull[2] | tempty[2] | tmem slot | bias[BN] f32 | red[4][BN] f32
   static constexpr int BAR_OFF = RING;
-  static constexpr int SLOT_OFF = BAR_OFF + (2 * STAGES + 1) * 8;
-  static constexpr int RED_OFF = (SLOT_OFF + 16 + 15) / 16 * 16;
+  static constexpr int SLOT_OFF = BAR_OFF + (2 * STAGES + 4) * 8;
+  static constexpr int BIAS_OFF = (SLOT_OFF + 16 + 15) / 16 * 16;
+  static constexpr int RED_OFF = BIAS_OFF + BN * 4;
   static constexpr int SMEM = RED_OFF + 4 * BN * 4 + 1024;   // + alignment slack
+  static_assert(SMEM <= kSmemBudget, "smem budget");
 };
 
 // ----------------------------------------------------------------- PTX
@@ -56,6 +68,9 @@ __device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
 __device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes)
                : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
 }
 __device__ __forceinline__ bool mbar_try_wait(uint32_t bar, uint32_t parity) {
   uint32_t ok;
@@ -115,6 +130,11 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
       : "r"(taddr));
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+__device__ __forceinline__ void epi_bar() { asm volatile("bar.sync 1, 128;" ::: "memory"); }
 
 // UMMA shared-memory descriptor, SWIZZLE_128B (layout type 2), version 1.
 //   K-major : rows of 128 B (64 K-elements), 8-row groups 1024 B apart (SBO).
@@ -150,20 +170,22 @@ __device__ __forceinline__ uint32_t pack_bf2(float a, float b) {
   __nv_bfloat162 h = __floats2bfloat162_rn(a, b);   // RNE
   return *reinterpret_cast<uint32_t *>(&h);
 }
-// load 32 consecutive bf16 (64 B, 16-B aligned) as fp32
-__device__ __forceinline__ void ld_bf16x32(const __nv_bfloat16 *p, float (&f)[32]) {
-  const uint4 *q = reinterpret_cast<const uint4 *>(p);
+__device__ __forceinline__ void unpack_bf16x32(const uint4 (&u)[4], float (&f)[32]) {
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
-    uint4 u = __ldg(q + j);
-    f[8 * j + 0] = bf_lo(u.x); f[8 * j + 1] = bf_hi(u.x);
-    f[8 * j + 2] = bf_lo(u.y); f[8 * j + 3] = bf_hi(u.y);
-    f[8 * j + 4] = bf_lo(u.z); f[8 * j + 5] = bf_hi(u.z);
-    f[8 * j + 6] = bf_lo(u.w); f[8 * j + 7] = bf_hi(u.w);
+    f[8 * j + 0] = bf_lo(u[j].x); f[8 * j + 1] = bf_hi(u[j].x);
+    f[8 * j + 2] = bf_lo(u[j].y); f[8 * j + 3] = bf_hi(u[j].y);
+    f[8 * j + 4] = bf_lo(u[j].z); f[8 * j + 5] = bf_hi(u[j].z);
+    f[8 * j + 6] = bf_lo(u[j].w); f[8 * j + 7] = bf_hi(u[j].w);
   }
 }
-// store 32 fp32 as bf16 (RNE) and return the rounded values in f
-__device__ __forceinline__ void st_bf16x32(__nv_bfloat16 *p, float (&f)[32]) {
+__device__ __forceinline__ void ld_raw32(const __nv_bfloat16 *p, uint4 (&u)[4]) {
+  const uint4 *q = reinterpret_cast<const uint4 *>(p);
+#pragma unroll
+  for (int j = 0; j < 4; ++j) u[j] = __ldg(q + j);
+}
+// store 32 fp32 as bf16 (RNE)
+__device__ __forceinline__ void st_bf16x32(__nv_bfloat16 *p, const float (&f)[32]) {
   uint4 *q = reinterpret_cast<uint4 *>(p);
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
@@ -195,6 +217,24 @@ __device__ __forceinline__ float warp_colsum32(float (&v)[32], int lane) {
   return v[0];
 }
 
+struct TileIdx {
+  int m0, n0, split, kb_begin, nkb;
+};
+__device__ __forceinline__ TileIdx decode(int t, int mt, int nt, int BN, const EpiArgs &a) {
+  TileIdx r;
+  const int per = mt * nt;
+  r.split = t / per;
+  const int rem = t - r.split * per;
+  r.m0 = (rem % mt) * BM;
+  r.n0 = (rem / mt) * BN;
+  const int nkb_total = (a.K + BK - 1) / BK;
+  r.kb_begin = r.split * a.kb_per_split;
+  int kb_end = r.kb_begin + a.kb_per_split;
+  if (kb_end > nkb_total) kb_end = nkb_total;
+  r.nkb = kb_end - r.kb_begin;
+  return r;
+}
+
 // ------------------------------------------------------------------ kernel
 template <int BN, bool A_MN, bool B_MN, int EPI>
 __global__ void __launch_bounds__(kThreads, 1)
@@ -207,19 +247,17 @@ __global__ void __launch_bounds__(kThreads, 1)
   const uint32_t sbase = smem_u32(smem);
   const uint32_t bar_full = sbase + C::BAR_OFF;
   const uint32_t bar_empty = bar_full + 8 * C::STAGES;
-  const uint32_t bar_accum = bar_empty + 8 * C::STAGES;
+  const uint32_t bar_tfull = bar_empty + 8 * C::STAGES;
+  const uint32_t bar_tempty = bar_tfull + 16;
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(smem + C::SLOT_OFF);
+  float *bias_s = reinterpret_cast<float *>(smem + C::BIAS_OFF);
   float *red = reinterpret_cast<float *>(smem + C::RED_OFF);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
-  const int m0 = blockIdx.x * BM;
-  const int n0 = blockIdx.y * BN;
-  const int nkb_total = (args.K + BK - 1) / BK;
-  const int kb_begin = blockIdx.z * args.kb_per_split;
-  int kb_end = kb_begin + args.kb_per_split;
-  if (kb_end > nkb_total) kb_end = nkb_total;
-  const int nkb = kb_end - kb_begin;
+  const int mt = (args.M + BM - 1) / BM;
+  const int nt = (args.N + BN - 1) / BN;
+  const int units = mt * nt * args.splits;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch(&tmA);
@@ -228,7 +266,10 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(bar_full + 8 * s, 1);
       mbar_init(bar_empty + 8 * s, 1);
     }
-    mbar_init(bar_accum, 1);
+    for (int a = 0; a < 2; ++a) {
+      mbar_init(bar_tfull + 8 * a, 1);
+      mbar_init(bar_tempty + 8 * a, 4);    // one arrive per epilogue warp
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   }
@@ -243,29 +284,36 @@ __global__ void __launch_bounds__(kThreads, 1)
   __syncthreads();
   fence_after();
   const uint32_t tmem = *tmem_slot;
+  // everything above overlaps the previous kernel's tail (PDL)
+  pdl_wait();
+  pdl_launch_dependents();
 
   if (warp == 0) {
     // ===================== TMA producer =====================
     if (lane == 0) {
-      for (int kb = 0; kb < nkb; ++kb) {
-        const int s = kb % C::STAGES;
-        if (kb >= C::STAGES) mbar_wait(bar_empty + 8 * s, ((kb / C::STAGES) - 1) & 1);
-        const uint32_t fb = bar_full + 8 * s;
-        mbar_expect_tx(fb, C::STAGE);
-        const uint32_t sa = sbase + s * C::STAGE;
-        const uint32_t sb = sa + A_BYTES;
-        const int k0 = (kb_begin + kb) * BK;
-        if (!A_MN) {
-          tma_load_2d(sa, &tmA, fb, k0, m0);                 // box {64 K, 128 M}
-        } else {
-          tma_load_2d(sa, &tmA, fb, m0, k0);                 // box {64 M, 64 K}
-          tma_load_2d(sa + 8192, &tmA, fb, m0 + 64, k0);
-        }
-        if (!B_MN) {
-          tma_load_2d(sb, &tmB, fb, k0, n0);                 // box {64 K, BN N}
-        } else {
+      int it = 0;
+      for (int t = blockIdx.x; t < units; t += gridDim.x) {
+        const TileIdx ti = decode(t, mt, nt, BN, args);
+        for (int kb = 0; kb < ti.nkb; ++kb, ++it) {
+          const int s = it % C::STAGES;
+          if (it >= C::STAGES) mbar_wait(bar_empty + 8 * s, ((it / C::STAGES) - 1) & 1);
+          const uint32_t fb = bar_full + 8 * s;
+          mbar_expect_tx(fb, C::STAGE);
+          const uint32_t sa = sbase + s * C::STAGE;
+          const uint32_t sb = sa + A_BYTES;
+          const int k0 = (ti.kb_begin + kb) * BK;
+          if (!A_MN) {
+            tma_load_2d(sa, &tmA, fb, k0, ti.m0);                 // box {64 K, 128 M}
+          } else {
+            tma_load_2d(sa, &tmA, fb, ti.m0, k0);                 // box {64 M, 64 K}
+            tma_load_2d(sa + 8192, &tmA, fb, ti.m0 + 64, k0);
+          }
+          if (!B_MN) {
+            tma_load_2d(sb, &tmB, fb, k0, ti.n0);                 // box {64 K, BN N}
+          } else {
 #pragma unroll
-          for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + 8192 * j, &tmB, fb, n0 + 64 * j, k0);
+            for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + 8192 * j, &tmB, fb, ti.n0 + 64 * j, k0);
+          }
         }
       }
     }
@@ -273,104 +321,137 @@ __global__ void __launch_bounds__(kThreads, 1)
     // ===================== MMA issuer =====================
     if (lane == 0) {
       constexpr uint32_t ID = idesc<BN, A_MN, B_MN>();
-      for (int kb = 0; kb < nkb; ++kb) {
-        const int s = kb % C::STAGES;
-        mbar_wait(bar_full + 8 * s, (kb / C::STAGES) & 1);
+      int it = 0, j = 0;
+      for (int t = blockIdx.x; t < units; t += gridDim.x, ++j) {
+        const TileIdx ti = decode(t, mt, nt, BN, args);
+        const int acc = j & 1;
+        if (j >= 2) mbar_wait(bar_tempty + 8 * acc, ((j >> 1) - 1) & 1);   // epilogue drained it
         fence_after();
-        const uint32_t sa = sbase + s * C::STAGE;
-        const uint32_t sb = sa + A_BYTES;
+        const uint32_t dtm = tmem + (uint32_t)(acc * BN);
+        for (int kb = 0; kb < ti.nkb; ++kb, ++it) {
+          const int s = it % C::STAGES;
+          mbar_wait(bar_full + 8 * s, (it / C::STAGES) & 1);
+          fence_after();
+          const uint32_t sa = sbase + s * C::STAGE;
+          const uint32_t sb = sa + A_BYTES;
 #pragma unroll
-        for (int kk = 0; kk < BK / 16; ++kk) {
-          const uint64_t ad = A_MN ? sdesc(sa + kk * 2048, 8192, 1024) : sdesc(sa + kk * 32, 16, 1024);
-          const uint64_t bd = B_MN ? sdesc(sb + kk * 2048, 8192, 1024) : sdesc(sb + kk * 32, 16, 1024);
-          umma_bf16(tmem, ad, bd, ID, (kb | kk) != 0 ? 1u : 0u);
+          for (int kk = 0; kk < BK / 16; ++kk) {
+            const uint64_t ad = A_MN ? sdesc(sa + kk * 2048, 8192, 1024) : sdesc(sa + kk * 32, 16, 1024);
+            const uint64_t bd = B_MN ? sdesc(sb + kk * 2048, 8192, 1024) : sdesc(sb + kk * 32, 16, 1024);
+            umma_bf16(dtm, ad, bd, ID, (kb | kk) != 0 ? 1u : 0u);
+          }
+          umma_commit(bar_empty + 8 * s);     // smem slot free once these MMAs retire
         }
-        umma_commit(bar_empty + 8 * s);     // smem slot free once these MMAs retire
+        umma_commit(bar_tfull + 8 * acc);     // accumulator complete
       }
-      umma_commit(bar_accum);               // accumulator complete
     }
     __syncwarp();
   } else {
     // ===================== epilogue (warps 2..5) =====================
     const int q = warp & 3;                  // TMEM lane quarter this warp may access
-    const int row = m0 + q * 32 + lane;
-    const bool row_ok = row < args.M;
-    if (nkb > 0) {
-      mbar_wait(bar_accum, 0);
-      fence_after();
-    }
-#pragma unroll 1
-    for (int c = 0; c < BN / 32; ++c) {
-      const int col0 = n0 + c * 32;
-      if (col0 >= args.N) break;             // warp-uniform (N % 64 == 0)
-      float v[32];
-      if (nkb > 0) {
-        uint32_t r[32];
-        tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(c * 32), r);
-#pragma unroll
-        for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]);
-      } else {
-#pragma unroll
-        for (int j = 0; j < 32; ++j) v[j] = 0.f;
-      }
-      const size_t off = (size_t)row * args.ldc + col0;
+    const int et = threadIdx.x - 64;         // 0..127
+    int j = 0;
+    for (int t = blockIdx.x; t < units; t += gridDim.x, ++j) {
+      const TileIdx ti = decode(t, mt, nt, BN, args);
+      const int acc = j & 1;
+      const int row = ti.m0 + q * 32 + lane;
+      const bool row_ok = row < args.M;
       if (EPI == EPI_FWD) {
-        float bias[32];
-        ld_bf16x32(reinterpret_cast<const __nv_bfloat16 *>(args.bias) + col0, bias);
-#pragma unroll
-        for (int j = 0; j < 32; ++j) v[j] += bias[j];
-        round_bf16x32(v);                                    // Z_i storage point
-        if (row_ok && args.z_out)
-          st_bf16x32(reinterpret_cast<__nv_bfloat16 *>(args.z_out) + off, v);
-        if (args.act != ACT_ID) {
-#pragma unroll
-          for (int j = 0; j < 32; ++j) v[j] = act_f(args.act, v[j]);
+        // stage the tile's bias in smem while the MMAs run
+        epi_bar();                                           // previous tile done reading bias_s
+        for (int c = et; c < BN; c += 128) {
+          const int n = ti.n0 + c;
+          bias_s[c] = n < args.N ? __bfloat162float(reinterpret_cast<const __nv_bfloat16 *>(args.bias)[n]) : 0.f;
         }
-        if (row_ok) st_bf16x32(reinterpret_cast<__nv_bfloat16 *>(args.x_out) + off, v);
-      } else if (EPI == EPI_DGRAD) {
-        if (args.act != ACT_ID) {
-          float z[32];
+        epi_bar();
+      }
+      const bool have = ti.nkb > 0;
+      if (have) {
+        mbar_wait(bar_tfull + 8 * acc, (j >> 1) & 1);
+        fence_after();
+      }
+      uint4 zraw[4];
+      const __nv_bfloat16 *zrow =
+          reinterpret_cast<const __nv_bfloat16 *>(args.zin) + (size_t)row * args.ldc + ti.n0;
+      const bool need_z = (EPI == EPI_DGRAD) && args.act != ACT_ID && row_ok;
+      if (need_z) ld_raw32(zrow, zraw);
+#pragma unroll 1
+      for (int c = 0; c < BN / 32; ++c) {
+        const int col0 = ti.n0 + c * 32;
+        if (col0 >= args.N) break;             // warp-uniform (N % 32 == 0)
+        float v[32];
+        if (have) {
+          uint32_t r[32];
+          tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * BN + c * 32), r);
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+        } else {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = 0.f;
+        }
+        const size_t off = (size_t)row * args.ldc + col0;
+        if (EPI == EPI_FWD) {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] += bias_s[c * 32 + i];
+          round_bf16x32(v);                                    // Z_i storage point
+          if (row_ok && args.z_out)
+            st_bf16x32(reinterpret_cast<__nv_bfloat16 *>(args.z_out) + off, v);
+          if (args.act != ACT_ID) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = act_f(args.act, v[i]);
+          }
+          if (row_ok) st_bf16x32(reinterpret_cast<__nv_bfloat16 *>(args.x_out) + off, v);
+        } else if (EPI == EPI_DGRAD) {
+          if (args.act != ACT_ID) {
+            float z[32];
+            if (need_z) {
+              unpack_bf16x32(zraw, z);
+              if (c + 1 < BN / 32 && col0 + 32 < args.N) ld_raw32(zrow + (c + 1) * 32, zraw);  // prefetch
+            } else {
+#pragma unroll
+              for (int i = 0; i < 32; ++i) z[i] = 0.f;
+            }
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] *= act_grad_f(args.act, z[i]);
+          }
+          round_bf16x32(v);                                    // dZ_{i-1} storage point
           if (row_ok) {
-            ld_bf16x32(reinterpret_cast<const __nv_bfloat16 *>(args.zin) + off, z);
+            st_bf16x32(reinterpret_cast<__nv_bfloat16 *>(args.x_out) + off, v);
           } else {
 #pragma unroll
-            for (int j = 0; j < 32; ++j) z[j] = 0.f;
+            for (int i = 0; i < 32; ++i) v[i] = 0.f;
           }
+          if (args.dbpart) {
+            const float s = warp_colsum32(v, lane);           // lane l: column col0 + l
+            red[q * BN + c * 32 + lane] = s;
+          }
+        } else {  // EPI_WGRAD
+          if (args.splits == 1) {
 #pragma unroll
-          for (int j = 0; j < 32; ++j) v[j] *= act_grad_f(args.act, z[j]);
-        }
-        round_bf16x32(v);                                    // dZ_{i-1} storage point
-        if (!row_ok) {
+            for (int i = 0; i < 32; ++i) v[i] *= args.alpha;
+            if (row_ok) st_bf16x32(reinterpret_cast<__nv_bfloat16 *>(args.x_out) + off, v);
+          } else if (row_ok) {
+            float4 *dst = reinterpret_cast<float4 *>(args.fpart + (size_t)ti.split * args.M * args.ldc + off);
 #pragma unroll
-          for (int j = 0; j < 32; ++j) v[j] = 0.f;
-        }
-        if (row_ok) st_bf16x32(reinterpret_cast<__nv_bfloat16 *>(args.x_out) + off, v);
-        if (args.dbpart) {
-          const float s = warp_colsum32(v, lane);           // lane l: column col0 + l
-          red[q * BN + c * 32 + lane] = s;
-        }
-      } else {  // EPI_WGRAD
-        if (args.splits == 1) {
-#pragma unroll
-          for (int j = 0; j < 32; ++j) v[j] *= args.alpha;
-          if (row_ok) st_bf16x32(reinterpret_cast<__nv_bfloat16 *>(args.x_out) + off, v);
-        } else if (row_ok) {
-          float4 *dst = reinterpret_cast<float4 *>(args.fpart + (size_t)blockIdx.z * args.M * args.ldc + off);
-#pragma unroll
-          for (int j = 0; j < 8; ++j) dst[j] = make_float4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]);
+            for (int i = 0; i < 8; ++i) dst[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+          }
         }
       }
-    }
-    if (EPI == EPI_DGRAD && args.dbpart) {
-      // sum the four row quarters in fixed order q = 0..3 (deterministic)
-      asm volatile("bar.sync 1, 128;" ::: "memory");
-      const int t = threadIdx.x - 64;                        // 0..127
-      for (int cc = t; cc < BN; cc += 128) {
-        const int col = n0 + cc;
-        if (col < args.N) {
-          const float s = ((red[cc] + red[BN + cc]) + red[2 * BN + cc]) + red[3 * BN + cc];
-          args.dbpart[(size_t)blockIdx.x * args.N + col] = s;
+      // accumulator buffer may be reused by the MMA warp
+      fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(bar_tempty + 8 * acc);
+      if (EPI == EPI_DGRAD && args.dbpart) {
+        // sum the four row quarters in fixed order q = 0..3 (deterministic)
+        epi_bar();
+        for (int cc = et; cc < BN; cc += 128) {
+          const int col = ti.n0 + cc;
+          if (col < args.N) {
+            const float s = ((red[cc] + red[BN + cc]) + red[2 * BN + cc]) + red[3 * BN + cc];
+            args.dbpart[(size_t)(ti.m0 / BM) * args.N + col] = s;
+          }
         }
+        epi_bar();
       }
     }
   }
@@ -386,17 +467,19 @@ __global__ void __launch_bounds__(kThreads, 1)
 
 template <int BN, bool A_MN, bool B_MN, int EPI>
 cudaError_t launch_one(const CUtensorMap *tmA, const CUtensorMap *tmB, const EpiArgs &args,
-                       dim3 grid, const LaunchCtx &ctx) {
+                       int ctas, const LaunchCtx &ctx) {
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = grid;
+  cfg.gridDim = dim3(ctas, 1, 1);
   cfg.blockDim = dim3(kThreads, 1, 1);
   cfg.dynamicSmemBytes = Cfg<BN>::SMEM;
   cfg.stream = ctx.stream;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributePriority;
   attr[0].val.priority = ctx.priority;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = ctx.pdl ? 1 : 0;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = 2;
   return cudaLaunchKernelEx(&cfg, gemm_tc_kernel<BN, A_MN, B_MN, EPI>, *tmA, *tmB, args);
 }
 
@@ -412,15 +495,15 @@ int gemm_tc_smem_bytes(int bn) {
   switch (bn) {
     case 64: return tc::Cfg<64>::SMEM;
     case 128: return tc::Cfg<128>::SMEM;
+    case 192: return tc::Cfg<192>::SMEM;
     case 256: return tc::Cfg<256>::SMEM;
   }
   return -1;
 }
 
-#define OOO_TC_ALL(X)                                                   \
-  X(64, false, true, EPI_FWD) X(128, false, true, EPI_FWD) X(256, false, true, EPI_FWD) \
-  X(64, false, false, EPI_DGRAD) X(128, false, false, EPI_DGRAD) X(256, false, false, EPI_DGRAD) \
-  X(64, true, true, EPI_WGRAD) X(128, true, true, EPI_WGRAD) X(256, true, true, EPI_WGRAD)
+#define OOO_TC_BN(X, AM, BMJ, EP) X(64, AM, BMJ, EP) X(128, AM, BMJ, EP) X(192, AM, BMJ, EP) X(256, AM, BMJ, EP)
+#define OOO_TC_ALL(X) \
+  OOO_TC_BN(X, false, true, EPI_FWD) OOO_TC_BN(X, false, false, EPI_DGRAD) OOO_TC_BN(X, true, true, EPI_WGRAD)
 
 cudaError_t gemm_tc_init() {
   cudaError_t e = cudaSuccess;
@@ -432,9 +515,9 @@ cudaError_t gemm_tc_init() {
 }
 
 cudaError_t launch_gemm_tc(int epi, int bn, const CUtensorMap *tmA, const CUtensorMap *tmB,
-                           const EpiArgs &args, dim3 grid, const LaunchCtx &ctx) {
+                           const EpiArgs &args, int ctas, const LaunchCtx &ctx) {
 #define OOO_DISPATCH(BN, AM, BMJ, EP) \
-  if (epi == EP && bn == BN) return tc::launch_one<BN, AM, BMJ, EP>(tmA, tmB, args, grid, ctx);
+  if (epi == EP && bn == BN) return tc::launch_one<BN, AM, BMJ, EP>(tmA, tmB, args, ctas, ctx);
   OOO_TC_ALL(OOO_DISPATCH)
 #undef OOO_DISPATCH
   return cudaErrorInvalidValue;

@@ -42,13 +42,15 @@ struct EpiArgs {
 struct LaunchCtx {
   cudaStream_t stream;
   int priority;
+  bool pdl = false;   // programmatic dependent launch (the kernel must griddepcontrol.wait)
 };
 
 // ---- tcgen05 bf16 GEMM (gemm_tc.cu).  A is M x K, B is K x N (logical).
 // a_mn / b_mn: operand stored MN-major (true) or K-major (false) -- see the
 // tensor-map builders below.  Returns a CUDA error code.
+// Persistent: `ctas` CTAs walk the ceil(M/128) x ceil(N/bn) x splits work units.
 cudaError_t launch_gemm_tc(int epi, int bn, const CUtensorMap *tmA, const CUtensorMap *tmB,
-                           const EpiArgs &args, dim3 grid, const LaunchCtx &ctx);
+                           const EpiArgs &args, int ctas, const LaunchCtx &ctx);
 int gemm_tc_smem_bytes(int bn);
 cudaError_t gemm_tc_init();   // sets max dynamic smem on every instantiation
 

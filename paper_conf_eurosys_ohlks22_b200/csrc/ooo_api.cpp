@@ -17,6 +17,7 @@
 #include <cuda_runtime.h>
 #include <stdarg.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 
 #include <algorithm>
@@ -91,36 +92,55 @@ struct Plan {
 
 constexpr int kSMs = 148;
 
+// Tile plan of one tcgen05 GEMM (persistent kernel, 128 x BN tiles).  Cost
+// model: waves x (BN + c0), c0 ~ fixed per-tile overhead in column units,
+// so narrow outputs pick a BN that fills the 148 SMs evenly (e.g. N = 768 ->
+// BN = 192: 32 x 4 = 128 tiles in one wave).  Weight-gradient GEMMs with few
+// output tiles split K (tokens) into S fixed ranges summed by the pack kernel
+// in a fixed order (deterministic).
+int env_int(const char *name, int dflt) {
+  const char *v = getenv(name);
+  return v && *v ? atoi(v) : dflt;
+}
+
 GemmPlan plan_tc_mn(int M, int N, int K, bool weight_grad) {
   GemmPlan p;
   const int mt = (M + 127) / 128;
   const int nkb = (K + 63) / 64;
-  int best_bn = 64;
-  // largest tile that still fills the machine; else the one with most CTAs
-  const int cands[3] = {256, 128, 64};
-  bool chosen = false;
+  const int forced = env_int(weight_grad ? "OOO_BN_DW" : "OOO_BN", 0);
+  const int cands[4] = {256, 192, 128, 64};
+  double best = 1e30;
+  int best_bn = 128, best_S = 1;
   for (int bn : cands) {
-    if (N % bn != 0) continue;
-    const int tiles = mt * (N / bn);
-    if (tiles >= kSMs) { best_bn = bn; chosen = true; break; }
+    if (N % 64 != 0) continue;
+    if (forced && bn != forced) continue;
+    const int nt = (N + bn - 1) / bn;
+    const double waste = (double)(nt * bn - N) / (nt * bn);
+    if (waste > 0.25) continue;
+    const int tiles = mt * nt;
+    int S = 1;
+    if (weight_grad && tiles < kSMs) {
+      S = std::max(1, std::min(kSMs / tiles, nkb / 4));
+    }
+    const int kps = (nkb + S - 1) / S;
+    const int units = tiles * ((nkb + kps - 1) / kps);
+    const int waves = (units + kSMs - 1) / kSMs;
+    // per-unit cost ~ k-blocks x MMA time (N < 96 is shared-memory bound) +
+    // epilogue, + fp32 partial write / pack re-read when split
+    const int Sx = (nkb + kps - 1) / kps;
+    double cost = (double)waves * ((double)kps * (std::max(bn, 96) + 16) + 2.0 * bn + (Sx > 1 ? 6.0 * bn : 0.0));
+    if (cost < best * 0.999) {
+      best = cost;
+      best_bn = bn;
+      best_S = S;
+    }
   }
-  if (!chosen) {
-    // not a full wave: prefer 128 unless 64 gives markedly more CTAs
-    best_bn = (N % 128 == 0) ? 128 : 64;
-    if (!weight_grad && mt * ((N + 127) / 128) < kSMs / 2) best_bn = 64;
-  }
-  if (weight_grad) best_bn = (N % 128 == 0) ? 128 : 64;
   p.bn = best_bn;
-  const int tiles = mt * ((N + p.bn - 1) / p.bn);
-  int S = 1;
-  if (weight_grad && tiles < kSMs) {
-    S = kSMs / tiles;
-    S = std::min(S, std::max(1, nkb / 4));
-    S = std::max(S, 1);
-  }
+  const int S = best_S;
   p.kb_per_split = (nkb + S - 1) / S;
   p.splits = (nkb + p.kb_per_split - 1) / p.kb_per_split;   // every split >= 1 k-block
-  p.grid = dim3(mt, (N + p.bn - 1) / p.bn, p.splits);
+  const int units = mt * ((N + p.bn - 1) / p.bn) * p.splits;
+  p.grid = dim3(std::min(units, kSMs), 1, 1);
   return p;
 }
 
@@ -318,6 +338,7 @@ struct ooo_stack {
   ncclComm_t nccl = nullptr;
   const NcclApi *api = nullptr;
   bool timing = false;
+  bool pdl = true;
   std::vector<TimedRec> recs;
   size_t rec_cursor = 0;
   std::vector<int> D;
@@ -330,6 +351,16 @@ struct ooo_graph {
 };
 
 namespace {
+
+// Timing events become event-record nodes when the stream is being captured
+// (cudaEventRecordExternal); outside capture they are plain records.
+cudaError_t record_timing_event(cudaEvent_t ev, cudaStream_t st) {
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  cudaError_t e = cudaStreamIsCapturing(st, &cs);
+  if (e != cudaSuccess) return e;
+  if (cs == cudaStreamCaptureStatusActive) return cudaEventRecordWithFlags(ev, st, cudaEventRecordExternal);
+  return cudaEventRecord(ev, st);
+}
 
 ooo_status begin_rec(ooo_stack *s, cudaStream_t st, int kind, int layer, int sid, TimedRec **out) {
   *out = nullptr;
@@ -345,7 +376,7 @@ ooo_status begin_rec(ooo_stack *s, cudaStream_t st, int kind, int layer, int sid
   r->info.kind = kind;
   r->info.layer = layer;
   r->info.stream = sid;
-  CU_TRY(cudaEventRecordWithFlags(r->a, st, cudaEventRecordExternal));
+  CU_TRY(record_timing_event(r->a, st));
   *out = r;
   return OOO_OK;
 }
@@ -354,7 +385,7 @@ ooo_status end_rec(TimedRec *r, cudaStream_t st, int grid, double flops, double 
   r->info.grid = grid;
   r->info.flops = flops;
   r->info.bytes = bytes;
-  CU_TRY(cudaEventRecordWithFlags(r->b, st, cudaEventRecordExternal));
+  CU_TRY(record_timing_event(r->b, st));
   return OOO_OK;
 }
 
@@ -369,10 +400,10 @@ ooo_status launch_fwd(ooo_stack *s, int i, void *Y, cudaStream_t st, int prio) {
   a.bias = r.b; a.z_out = r.Z; a.x_out = (i == s->p.L) ? Y : r.Xn;
   TimedRec *tr;
   OOO_TRY(begin_rec(s, st, 0, i, 0, &tr));
-  LaunchCtx ctx{st, prio};
+  LaunchCtx ctx{st, prio, s->pdl};
   int grid = lp.fwd.grid.x * lp.fwd.grid.y * lp.fwd.grid.z;
   if (s->p.dtype == OOO_BF16) {
-    CU_TRY(launch_gemm_tc(EPI_FWD, lp.fwd.bn, &r.fwdA, &r.fwdB, a, lp.fwd.grid, ctx));
+    CU_TRY(launch_gemm_tc(EPI_FWD, lp.fwd.bn, &r.fwdA, &r.fwdB, a, grid, ctx));
   } else {
     SimtOperands o{static_cast<const float *>(r.X), lp.din, 1, static_cast<const float *>(r.W), lp.dout, 1};
     CU_TRY(launch_gemm_simt(EPI_FWD, o, a, ctx, &grid));
@@ -402,10 +433,10 @@ ooo_status launch_dx(ooo_stack *s, int i, void *dX, cudaStream_t st, int prio) {
   }
   TimedRec *tr;
   OOO_TRY(begin_rec(s, st, 1, i, st == s->hi ? 0 : 1, &tr));
-  LaunchCtx ctx{st, prio};
+  LaunchCtx ctx{st, prio, s->pdl};
   int grid = lp.dx.grid.x * lp.dx.grid.y * lp.dx.grid.z;
   if (s->p.dtype == OOO_BF16) {
-    CU_TRY(launch_gemm_tc(EPI_DGRAD, lp.dx.bn, &r.dxA, &r.dxB, a, lp.dx.grid, ctx));
+    CU_TRY(launch_gemm_tc(EPI_DGRAD, lp.dx.bn, &r.dxA, &r.dxB, a, grid, ctx));
   } else {
     SimtOperands o{static_cast<const float *>(r.dZ), lp.dout, 1, static_cast<const float *>(r.W), 1, lp.dout};
     CU_TRY(launch_gemm_simt(EPI_DGRAD, o, a, ctx, &grid));
@@ -426,16 +457,17 @@ ooo_status launch_dw_pack(ooo_stack *s, int i, cudaStream_t st, int prio, int si
   a.fpart = reinterpret_cast<float *>(s->ws + s->p.off_wpart);
   TimedRec *tr;
   OOO_TRY(begin_rec(s, st, 2, i, sid, &tr));
-  LaunchCtx ctx{st, prio};
+  LaunchCtx ctx{st, prio, s->pdl};
   int grid = lp.dw.grid.x * lp.dw.grid.y * lp.dw.grid.z;
   if (s->p.dtype == OOO_BF16) {
-    CU_TRY(launch_gemm_tc(EPI_WGRAD, lp.dw.bn, &r.dwA, &r.dwB, a, lp.dw.grid, ctx));
+    CU_TRY(launch_gemm_tc(EPI_WGRAD, lp.dw.bn, &r.dwA, &r.dwB, a, grid, ctx));
   } else {
     SimtOperands o{static_cast<const float *>(r.X), 1, lp.din, static_cast<const float *>(r.dZ), lp.dout, 1};
     CU_TRY(launch_gemm_simt(EPI_WGRAD, o, a, ctx, &grid));
   }
   OOO_TRY(end_rec(tr, st, grid, 2.0 * s->p.M * lp.din * lp.dout, 0));
-  // pack
+  // pack (plain launch: it does not use griddepcontrol)
+  ctx.pdl = false;
   OOO_TRY(begin_rec(s, st, 4, i, sid, &tr));
   const bool split = lp.dw.splits > 1;
   const long long wcount = (long long)lp.din * lp.dout;
@@ -695,6 +727,7 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
   s->d.dims = s->dims.data();
   s->d.acts = s->acts.data();
   s->p = make_plan(d);
+  s->pdl = env_int("OOO_PDL", 1) != 0;
   s->ws = static_cast<uint8_t *>(d->workspace);
   s->grads = static_cast<uint8_t *>(d->grads);
   const Plan &p = s->p;
@@ -909,9 +942,12 @@ ooo_status ooo_timing_read(ooo_stack *s, ooo_launch_record *out, int32_t cap, in
     if (out && cnt < cap) {
       TimedRec &r = s->recs[j];
       out[cnt] = r.info;
-      float ms = 0.f;
+      float ms = 0.f, st = 0.f;
       cudaError_t e = cudaEventElapsedTime(&ms, r.a, r.b);
       out[cnt].ms = e == cudaSuccess ? ms : -1.f;
+      if (e != cudaSuccess) (void)cudaGetLastError();
+      e = cudaEventElapsedTime(&st, s->recs[0].a, r.a);
+      out[cnt].start_ms = e == cudaSuccess ? st : -1.f;
       if (e != cudaSuccess) (void)cudaGetLastError();
     }
     ++cnt;

@@ -248,7 +248,8 @@ class OooStack:
         out = []
         for r in recs[: n.value]:
             out.append({"kind": _lib.KIND_NAMES.get(r.kind, r.kind), "layer": r.layer, "stream": r.stream,
-                        "grid": r.grid, "flops": r.flops, "bytes": r.bytes, "ms": r.ms})
+                        "grid": r.grid, "flops": r.flops, "bytes": r.bytes, "ms": r.ms,
+                        "start_ms": r.start_ms})
         return out
 
     def close(self):
