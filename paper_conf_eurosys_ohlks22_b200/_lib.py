@@ -9,7 +9,8 @@ import ctypes
 import os
 from ctypes import POINTER, c_char_p, c_double, c_float, c_int32, c_int64, c_size_t, c_void_p
 
-LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "lib", "libooo.so")
+LIB_PATH = os.environ.get("OOO_LIB") or os.path.join(os.path.dirname(os.path.abspath(__file__)), "lib",
+                                                      "libooo.so")
 
 OOO_OK = 0
 STATUS = {0: "OOO_OK", 1: "OOO_ERR_INVALID_ARGUMENT", 2: "OOO_ERR_UNSUPPORTED", 3: "OOO_ERR_CUDA",
@@ -60,7 +61,8 @@ class LaunchRecord(ctypes.Structure):
     ]
 
 
-KIND_NAMES = {0: "fwd_gemm", 1: "dx_gemm", 2: "dw_gemm", 3: "seed", 4: "pack", 5: "allreduce", 6: "copy"}
+KIND_NAMES = {0: "fwd_gemm", 1: "dx_gemm", 2: "dw_gemm", 3: "seed", 4: "pack", 5: "allreduce", 6: "copy",
+              7: "engine_fwd", 8: "engine_bwd"}
 
 EXPORTS = [
     "ooo_abi_version", "ooo_last_error", "ooo_status_string", "ooo_query_sizes", "ooo_grad_offsets",

@@ -24,7 +24,7 @@ LIB = os.path.join(LIBDIR, "libooo.so")
 OBJDIR = os.path.join(PKG, "build_obj")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-SOURCES = ["gemm_tc.cu", "gemm_simt.cu", "ew.cu", "ooo_api.cpp", "nccl_dyn.cpp"]
+SOURCES = ["gemm_tc.cu", "engine.cu", "gemm_simt.cu", "ew.cu", "ooo_api.cpp", "nccl_dyn.cpp"]
 
 
 def _nvcc() -> str:
@@ -64,18 +64,22 @@ def _digest() -> str:
     return h.hexdigest()
 
 
-def build(force: bool = False, verbose: bool = True) -> str:
+def build(force: bool = False, verbose: bool = True, trace: bool = False) -> str:
+    """trace=True builds the debug variant lib/libooo_trace.so (-DOOO_TRACE:
+    per-task timestamps in the engine, tools/engine_trace.py)."""
+    lib = LIB if not trace else os.path.join(LIBDIR, "libooo_trace.so")
+    objdir = OBJDIR if not trace else OBJDIR + "_trace"
     os.makedirs(LIBDIR, exist_ok=True)
-    os.makedirs(OBJDIR, exist_ok=True)
-    stamp = os.path.join(LIBDIR, "libooo.sha256")
-    dig = _digest()
-    if not force and os.path.exists(LIB) and os.path.exists(stamp) and open(stamp).read() == dig:
-        return LIB
+    os.makedirs(objdir, exist_ok=True)
+    stamp = os.path.splitext(lib)[0] + ".sha256"
+    dig = _digest() + ("-trace" if trace else "")
+    if not force and os.path.exists(lib) and os.path.exists(stamp) and open(stamp).read() == dig:
+        return lib
     nvcc = _nvcc()
-    flags = _flags()
+    flags = _flags() + (["-DOOO_TRACE"] if trace else [])
 
     def compile_one(src):
-        obj = os.path.join(OBJDIR, src + ".o")
+        obj = os.path.join(objdir, src + ".o")
         cmd = [nvcc] + flags + ["-Xptxas", "-v"] * (src == "gemm_tc.cu" and verbose is None) + \
               ["-c", os.path.join(CSRC, src), "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
@@ -85,18 +89,18 @@ def build(force: bool = False, verbose: bool = True) -> str:
 
     with cf.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
         objs = list(ex.map(compile_one, SOURCES))
-    tmp = LIB + ".tmp"
+    tmp = lib + ".tmp"
     cmd = [nvcc] + ARCH + ["-shared", "-cudart", "static", "-o", tmp] + objs + ["-ldl", "-lpthread"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         raise RuntimeError(f"link failed:\n{r.stdout}\n{r.stderr}")
-    os.replace(tmp, LIB)
+    os.replace(tmp, lib)
     with open(stamp, "w") as f:
         f.write(dig)
     if verbose:
-        print(f"built {LIB}", file=sys.stderr)
-    return LIB
+        print(f"built {lib}", file=sys.stderr)
+    return lib
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv)
+    build(force="--force" in sys.argv, trace="--trace" in sys.argv)

@@ -49,8 +49,11 @@ struct LaunchCtx {
 // a_mn / b_mn: operand stored MN-major (true) or K-major (false) -- see the
 // tensor-map builders below.  Returns a CUDA error code.
 // Persistent: `ctas` CTAs walk the ceil(M/128) x ceil(N/bn) x splits work units.
+// tmZ / tmX: bf16 output maps (box {64 cols, 32 rows}, 128B swizzle) for the
+// Z / X outputs of F_i, the dZ (or dX) output of dO_i and the bucket of dW_i.
 cudaError_t launch_gemm_tc(int epi, int bn, const CUtensorMap *tmA, const CUtensorMap *tmB,
-                           const EpiArgs &args, int ctas, const LaunchCtx &ctx);
+                           const CUtensorMap *tmZ, const CUtensorMap *tmX, const EpiArgs &args, int ctas,
+                           const LaunchCtx &ctx);
 int gemm_tc_smem_bytes(int bn);
 cudaError_t gemm_tc_init();   // sets max dynamic smem on every instantiation
 

@@ -26,6 +26,7 @@
 #include <vector>
 
 #include "../../include/ooo.h"
+#include "engine.h"
 #include "kernels.h"
 #include "nccl_dyn.h"
 
@@ -79,7 +80,12 @@ struct LayerPlan {
   int64_t goff_w = 0, goff_b = 0;
   int bucket = 0;
   GemmPlan fwd, dx, dw;
+  int ebn_fwd = 0, ebn_dx = 0, ebn_dw = 0;   // engine tile widths
 };
+
+// Map-table slots per layer (engine): operand loads and output stores.
+enum MapSlot { MS_FWD_A = 0, MS_FWD_B, MS_FWD_X, MS_FWD_Z, MS_DX_A, MS_DX_B, MS_DZ_X, MS_DW_A, MS_DW_B,
+               MS_GW_X, MS_COUNT };
 
 struct Plan {
   int L = 0, M = 0, dtype = 0, elt = 2, R = 0, nbuckets = 0;
@@ -88,6 +94,10 @@ struct Plan {
   size_t off_wpart = 0, wpart_bytes = 0;
   size_t workspace_bytes = 0;
   int64_t grad_elems = 0;
+  // engine (bf16): map table, layer table, completion counters
+  bool engine = false;
+  size_t off_maps = 0, off_layers = 0, off_ctr = 0;
+  ooo::eng::CounterLayout cl{};
 };
 
 constexpr int kSMs = 148;
@@ -142,6 +152,16 @@ GemmPlan plan_tc_mn(int M, int N, int K, bool weight_grad) {
   const int units = mt * ((N + p.bn - 1) / p.bn) * p.splits;
   p.grid = dim3(std::min(units, kSMs), 1, 1);
   return p;
+}
+
+// Engine tile width for an output of width N: the widest of 256/192/128/64
+// that divides N (the dataflow pipeline hides wave quantisation, so wider
+// tiles -- better MMA efficiency, less L2 traffic per FLOP -- win).
+int engine_bn(int N) {
+  const int forced = env_int("OOO_EBN", 0);
+  if (forced && N % forced == 0) return forced;
+  for (int bn : {256, 192, 128}) if (N % bn == 0) return bn;
+  return 64;
 }
 
 GemmPlan plan_simt(int M, int N, int K, bool weight_grad) {
@@ -240,9 +260,35 @@ Plan make_plan(const ooo_stack_desc *d) {
   for (int i = 1; i <= p.L; ++i) p.layer[i - 1].off_db = take((size_t)p.R * p.layer[i - 1].dout * 4);
   p.wpart_bytes = wpart;
   p.off_wpart = wpart ? take(wpart) : 0;
+  p.nbuckets = (p.L + d->bucket_layers - 1) / d->bucket_layers;
+  // persistent dataflow engine (bf16): map table, layer table, counters
+  p.engine = p.dtype == OOO_BF16 && 2 * p.L <= ooo::eng::kMaxOps && env_int("OOO_ENGINE", 1) != 0;
+  if (p.engine) {
+    for (int i = 1; i <= p.L; ++i) {
+      LayerPlan &lp = p.layer[i - 1];
+      lp.ebn_fwd = engine_bn(lp.dout);
+      lp.ebn_dx = engine_bn(lp.din);
+      lp.ebn_dw = engine_bn(lp.dout);
+    }
+    p.off_maps = take((size_t)p.L * MS_COUNT * sizeof(CUtensorMap));
+    p.off_layers = take((size_t)p.L * sizeof(ooo::eng::LayerDev));
+    ooo::eng::CounterLayout &cl = p.cl;
+    cl.L = p.L;
+    cl.MT = (p.M + 127) / 128;
+    cl.nb = p.nbuckets;
+    cl.fwd_base = 0;
+    cl.fwd_size = 1 + p.L * cl.MT;
+    cl.bwd_base = align_up(cl.fwd_size, 64);
+    cl.dz_rows = cl.bwd_base + 1;
+    cl.dz_total = cl.dz_rows + p.L * cl.MT;
+    cl.dw_done = cl.dz_total + p.L;
+    cl.bucket_done = cl.dw_done + p.L;
+    cl.ar_done = cl.bucket_done + p.nbuckets;
+    cl.bwd_size = cl.ar_done + p.nbuckets - cl.bwd_base;
+    p.off_ctr = take((size_t)(cl.bwd_base + cl.bwd_size) * 4);
+  }
   p.workspace_bytes = std::max<size_t>(off, 256);
   p.grad_elems = goff;
-  p.nbuckets = (p.L + d->bucket_layers - 1) / d->bucket_layers;
   p.bucket_first.resize(p.nbuckets);
   p.bucket_last.resize(p.nbuckets);
   for (int b = 0; b < p.nbuckets; ++b) {
@@ -314,7 +360,8 @@ struct LayerRt {
   void *X = nullptr, *Z = nullptr, *Xn = nullptr, *dZ = nullptr;
   float *db = nullptr;
   void *gw = nullptr, *gb = nullptr;
-  CUtensorMap fwdA, fwdB, dxA, dxB, dwA, dwB;
+  CUtensorMap fwdA, fwdB, dxA, dxB, dwA, dwB;   // operand loads
+  CUtensorMap fwdZ, fwdX, dzX, gwX;              // output stores: Z_i, X_{i+1}, dZ_i, dW_i bucket
 };
 
 struct TimedRec {
@@ -342,6 +389,11 @@ struct ooo_stack {
   std::vector<TimedRec> recs;
   size_t rec_cursor = 0;
   std::vector<int> D;
+  // persistent dataflow engine (bf16)
+  int32_t *ctr = nullptr;                     // completion counters (workspace)
+  const CUtensorMap *dmaps = nullptr;         // map table (workspace)
+  const ooo::eng::LayerDev *dlayers = nullptr;
+  int engine_ctas = 148;
 };
 
 struct ooo_graph {
@@ -403,7 +455,14 @@ ooo_status launch_fwd(ooo_stack *s, int i, void *Y, cudaStream_t st, int prio) {
   LaunchCtx ctx{st, prio, s->pdl};
   int grid = lp.fwd.grid.x * lp.fwd.grid.y * lp.fwd.grid.z;
   if (s->p.dtype == OOO_BF16) {
-    CU_TRY(launch_gemm_tc(EPI_FWD, lp.fwd.bn, &r.fwdA, &r.fwdB, a, grid, ctx));
+    CUtensorMap ymap;
+    const CUtensorMap *xm = &r.fwdX;
+    if (i == s->p.L) {   // the caller's Y: encoded per call (baked into a captured graph)
+      OOO_TRY(make_map(&ymap, Y, lp.dout, s->p.M, 64, 32));
+      xm = &ymap;
+    }
+    const CUtensorMap *zm = r.Z ? &r.fwdZ : xm;
+    CU_TRY(launch_gemm_tc(EPI_FWD, lp.fwd.bn, &r.fwdA, &r.fwdB, zm, xm, a, grid, ctx));
   } else {
     SimtOperands o{static_cast<const float *>(r.X), lp.din, 1, static_cast<const float *>(r.W), lp.dout, 1};
     CU_TRY(launch_gemm_simt(EPI_FWD, o, a, ctx, &grid));
@@ -436,7 +495,15 @@ ooo_status launch_dx(ooo_stack *s, int i, void *dX, cudaStream_t st, int prio) {
   LaunchCtx ctx{st, prio, s->pdl};
   int grid = lp.dx.grid.x * lp.dx.grid.y * lp.dx.grid.z;
   if (s->p.dtype == OOO_BF16) {
-    CU_TRY(launch_gemm_tc(EPI_DGRAD, lp.dx.bn, &r.dxA, &r.dxB, a, grid, ctx));
+    CUtensorMap dxmap;
+    const CUtensorMap *xm = nullptr;
+    if (i >= 2) {
+      xm = &s->lr[i - 2].dzX;
+    } else {             // the caller's dX: encoded per call
+      OOO_TRY(make_map(&dxmap, dX, lp.din, s->p.M, 64, 32));
+      xm = &dxmap;
+    }
+    CU_TRY(launch_gemm_tc(EPI_DGRAD, lp.dx.bn, &r.dxA, &r.dxB, xm, xm, a, grid, ctx));
   } else {
     SimtOperands o{static_cast<const float *>(r.dZ), lp.dout, 1, static_cast<const float *>(r.W), 1, lp.dout};
     CU_TRY(launch_gemm_simt(EPI_DGRAD, o, a, ctx, &grid));
@@ -460,7 +527,7 @@ ooo_status launch_dw_pack(ooo_stack *s, int i, cudaStream_t st, int prio, int si
   LaunchCtx ctx{st, prio, s->pdl};
   int grid = lp.dw.grid.x * lp.dw.grid.y * lp.dw.grid.z;
   if (s->p.dtype == OOO_BF16) {
-    CU_TRY(launch_gemm_tc(EPI_WGRAD, lp.dw.bn, &r.dwA, &r.dwB, a, grid, ctx));
+    CU_TRY(launch_gemm_tc(EPI_WGRAD, lp.dw.bn, &r.dwA, &r.dwB, &r.gwX, &r.gwX, a, grid, ctx));
   } else {
     SimtOperands o{static_cast<const float *>(r.X), 1, lp.din, static_cast<const float *>(r.dZ), lp.dout, 1};
     CU_TRY(launch_gemm_simt(EPI_WGRAD, o, a, ctx, &grid));
@@ -545,7 +612,186 @@ ooo_status check_async(ooo_stack *s) {
   return OOO_OK;
 }
 
+// ---- persistent dataflow engine (bf16) ---------------------------------
+typedef CUresult (*StreamValueFn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+
+StreamValueFn stream_value_fn(const char *name) {
+  void *p = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &p, cudaEnableDefault, &q) != cudaSuccess || q != cudaDriverEntryPointSuccess)
+    return nullptr;
+  return reinterpret_cast<StreamValueFn>(p);
+}
+
+int map_index(int layer, int slot) { return (layer - 1) * MS_COUNT + slot; }
+
+bool comm_active(const ooo_stack *s) { return s->nccl != nullptr && s->d.comm_enabled; }
+
+ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st) {
+  const Plan &p = s->p;
+  const int L = p.L;
+  OOO_TRY(fork_from(s, st));
+  const bool gate = s->bwd_pending && comm_active(s);
+  CU_TRY(cudaMemsetAsync(s->ctr + p.cl.fwd_base, 0, (size_t)p.cl.fwd_size * 4, s->hi));
+  {
+    TimedRec *tr;
+    OOO_TRY(begin_rec(s, s->hi, 6, 1, 0, &tr));
+    const size_t bytes = (size_t)p.M * s->dims[0] * p.elt;
+    CU_TRY(cudaMemcpyAsync(s->lr[0].X, X, bytes, cudaMemcpyDeviceToDevice, s->hi));
+    OOO_TRY(end_rec(tr, s->hi, 0, 0, 2.0 * bytes));
+  }
+  ooo::eng::Params P = {};
+  P.M = p.M;
+  P.R = p.R;
+  P.alpha = 1.0f / (float)s->d.world_size;
+  P.gate_ar = gate ? 1 : 0;
+  P.pass = 0;
+  P.maps = s->dmaps;
+  P.ctr = s->ctr;
+  P.layers = s->dlayers;
+  P.cl = p.cl;
+  int first = 0;
+  double flops = 0;
+  for (int i = 1; i <= L; ++i) {
+    const LayerPlan &lp = p.layer[i - 1];
+    ooo::eng::Op &o = P.ops[i - 1];
+    o.kind = EPI_FWD;
+    o.act = (int16_t)lp.act;
+    o.bn = (int16_t)lp.ebn_fwd;
+    o.layer = (int16_t)i;
+    o.first = first;
+    o.mt = (int16_t)p.cl.MT;
+    o.nt = (int16_t)((lp.dout + lp.ebn_fwd - 1) / lp.ebn_fwd);
+    o.nkb = (int16_t)((lp.din + 63) / 64);
+    o.mapA = (int16_t)map_index(i, MS_FWD_A);
+    o.mapB = (int16_t)map_index(i, MS_FWD_B);
+    o.mapX = (int16_t)(i == L ? ooo::eng::MAP_Y : map_index(i, MS_FWD_X));
+    o.mapZ = (int16_t)(s->lr[i - 1].Z ? map_index(i, MS_FWD_Z) : ooo::eng::MAP_NONE);
+    first += o.mt * o.nt;
+    flops += 2.0 * p.M * lp.din * lp.dout;
+  }
+  P.nops = L;
+  P.ntasks = first;
+  CUtensorMap tmY;
+  OOO_TRY(make_map(&tmY, Y, p.layer[L - 1].dout, p.M, 64, 32));
+  TimedRec *tr;
+  OOO_TRY(begin_rec(s, s->hi, 7, 0, 0, &tr));
+  CU_TRY(ooo::eng::launch_engine(P, &tmY, &tmY, s->engine_ctas, s->hi, s->prio_hi));
+  OOO_TRY(end_rec(tr, s->hi, s->engine_ctas, flops, 0));
+  s->bwd_pending = false;
+  s->have_fwd = true;
+  return join_into(s, st);
+}
+
+ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, void *dX, cudaStream_t st) {
+  const Plan &p = s->p;
+  const int L = p.L;
+  OOO_TRY(fork_from(s, st));
+  CU_TRY(cudaMemsetAsync(s->ctr + p.cl.bwd_base, 0, (size_t)p.cl.bwd_size * 4, s->hi));
+  const bool comm = comm_active(s);
+  if (comm) {   // the comm stream's value-waits must observe the reset counters
+    CU_TRY(cudaEventRecord(s->ev_j_hi, s->hi));
+    CU_TRY(cudaStreamWaitEvent(s->comm, s->ev_j_hi, 0));
+  }
+  OOO_TRY(launch_seed_op(s, dY, s->hi, s->prio_hi));
+  // queue = D expanded to tiles; dW ops slotted right behind the next dO op so
+  // the critical chain is dispensed first (two-stream priority)
+  ooo::eng::Params P = {};
+  P.M = p.M;
+  P.R = p.R;
+  P.alpha = 1.0f / (float)s->d.world_size;
+  P.in_order = in_order ? 1 : 0;
+  P.pass = 1;
+  P.maps = s->dmaps;
+  P.ctr = s->ctr;
+  P.layers = s->dlayers;
+  P.cl = p.cl;
+  int nops = 0, first = 0;
+  double flops = 0;
+  auto add_op = [&](int op) {
+    const int i = op > 0 ? op : -op;
+    const LayerPlan &lp = p.layer[i - 1];
+    ooo::eng::Op &o = P.ops[nops++];
+    o.layer = (int16_t)i;
+    o.first = first;
+    if (op > 0) {
+      o.kind = EPI_DGRAD;
+      o.act = (int16_t)(i >= 2 ? p.layer[i - 2].act : OOO_ACT_IDENTITY);
+      o.bn = (int16_t)lp.ebn_dx;
+      o.mt = (int16_t)p.cl.MT;
+      o.nt = (int16_t)((lp.din + lp.ebn_dx - 1) / lp.ebn_dx);
+      o.nkb = (int16_t)((lp.dout + 63) / 64);
+      o.mapA = (int16_t)map_index(i, MS_DX_A);
+      o.mapB = (int16_t)map_index(i, MS_DX_B);
+      o.mapX = (int16_t)(i >= 2 ? map_index(i - 1, MS_DZ_X) : ooo::eng::MAP_DX);
+    } else {
+      o.kind = EPI_WGRAD;
+      o.act = OOO_ACT_IDENTITY;
+      o.bn = (int16_t)lp.ebn_dw;
+      o.mt = (int16_t)((lp.din + 127) / 128);
+      o.nt = (int16_t)((lp.dout + lp.ebn_dw - 1) / lp.ebn_dw);
+      o.nkb = (int16_t)((p.M + 63) / 64);
+      o.mapA = (int16_t)map_index(i, MS_DW_A);
+      o.mapB = (int16_t)map_index(i, MS_DW_B);
+      o.mapX = (int16_t)map_index(i, MS_GW_X);
+    }
+    o.mapZ = ooo::eng::MAP_NONE;
+    first += o.mt * o.nt;
+    flops += 2.0 * p.M * lp.din * lp.dout;
+  };
+  std::vector<int> pending;
+  for (int op : s->D) {
+    if (op > 0) {
+      add_op(op);
+      for (int w : pending) add_op(w);
+      pending.clear();
+    } else if (in_order) {
+      add_op(op);
+    } else {
+      pending.push_back(op);
+    }
+  }
+  for (int w : pending) add_op(w);
+  P.nops = nops;
+  P.ntasks = first;
+  CUtensorMap tmDX;
+  if (dX) OOO_TRY(make_map(&tmDX, dX, s->dims[0], p.M, 64, 32));
+  else tmDX = s->lr[0].dxA;   // unused placeholder
+  TimedRec *tr;
+  OOO_TRY(begin_rec(s, s->hi, 8, 0, 0, &tr));
+  CU_TRY(ooo::eng::launch_engine(P, &tmDX, &tmDX, s->engine_ctas, s->hi, s->prio_hi));
+  OOO_TRY(end_rec(tr, s->hi, s->engine_ctas, flops, 0));
+  if (comm) {
+    // S[dW] per bucket in D's dW order: the comm stream waits for the bucket's
+    // dW tiles (engine counter), all-reduces, and publishes ar_done for F_i.
+    static StreamValueFn wait_fn = stream_value_fn("cuStreamWaitValue32");
+    static StreamValueFn write_fn = stream_value_fn("cuStreamWriteValue32");
+    if (!wait_fn || !write_fn) return fail(OOO_ERR_CUDA, "stream memory operations unavailable");
+    std::vector<int> left(p.nbuckets), tiles(p.nbuckets, 0);
+    for (int b = 0; b < p.nbuckets; ++b) left[b] = p.bucket_last[b] - p.bucket_first[b] + 1;
+    for (int i = 1; i <= L; ++i) {
+      const LayerPlan &lp = p.layer[i - 1];
+      tiles[lp.bucket] += ((lp.din + 127) / 128) * ((lp.dout + lp.ebn_dw - 1) / lp.ebn_dw);
+    }
+    for (int op : s->D) {
+      if (op > 0) continue;
+      const int b = p.layer[-op - 1].bucket;
+      if (--left[b] != 0) continue;
+      CUresult r = wait_fn(s->comm, reinterpret_cast<CUdeviceptr>(s->ctr + p.cl.bucket_done + b),
+                           (cuuint32_t)tiles[b], CU_STREAM_WAIT_VALUE_GEQ);
+      if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWaitValue32 failed (%d)", (int)r);
+      OOO_TRY(launch_allreduce(s, b));
+      r = write_fn(s->comm, reinterpret_cast<CUdeviceptr>(s->ctr + p.cl.ar_done + b), 1, 0);
+      if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWriteValue32 failed (%d)", (int)r);
+    }
+  }
+  s->have_fwd = false;
+  s->bwd_pending = true;
+  return OOO_OK;
+}
+
 ooo_status enqueue_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st) {
+  if (s->p.engine) return engine_forward(s, X, Y, st);
   const int L = s->p.L;
   OOO_TRY(fork_from(s, st));
   const bool pend = s->bwd_pending;
@@ -594,6 +840,7 @@ ooo_status enqueue_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void
   }
   schedule_ops(L, sch.kind, k, s->d.need_input_grad != 0, s->D);
   if (s->timing) s->rec_cursor = 0;
+  if (s->p.engine) return engine_backward(s, dY, sch.kind == OOO_SCHED_IN_ORDER, dX, st);
   OOO_TRY(fork_from(s, st));
   const bool single = sch.kind == OOO_SCHED_IN_ORDER;
   cudaStream_t wst = single ? s->hi : s->lo;
@@ -762,9 +1009,72 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
           (st = make_map(&r.dxA, r.dZ, lp.dout, p.M, 64, 128)) != OOO_OK ||
           (st = make_map(&r.dxB, r.W, lp.dout, lp.din, 64, lp.dx.bn)) != OOO_OK ||
           (st = make_map(&r.dwA, r.X, lp.din, p.M, 64, 64)) != OOO_OK ||
-          (st = make_map(&r.dwB, r.dZ, lp.dout, p.M, 64, 64)) != OOO_OK)
+          (st = make_map(&r.dwB, r.dZ, lp.dout, p.M, 64, 64)) != OOO_OK ||
+          (st = make_map(&r.dzX, r.dZ, lp.dout, p.M, 64, 32)) != OOO_OK ||
+          (st = make_map(&r.gwX, r.gw, lp.dout, lp.din, 64, 32)) != OOO_OK ||
+          (r.Z && (st = make_map(&r.fwdZ, r.Z, lp.dout, p.M, 64, 32)) != OOO_OK) ||
+          (r.Xn && (st = make_map(&r.fwdX, r.Xn, lp.dout, p.M, 64, 32)) != OOO_OK))
         return cleanup_fail(st);
     }
+  }
+  if (p.engine) {
+    static std::once_flag eng_once;
+    static cudaError_t eng_err = cudaSuccess;
+    std::call_once(eng_once, [] { eng_err = ooo::eng::engine_init(); });
+    if (eng_err != cudaSuccess)
+      return cleanup_fail(fail(OOO_ERR_CUDA, "engine init: %s", cudaGetErrorString(eng_err)));
+    std::vector<CUtensorMap> maps((size_t)p.L * MS_COUNT);
+    std::vector<ooo::eng::LayerDev> ldev(p.L);
+    for (int i = 1; i <= p.L; ++i) {
+      const LayerPlan &lp = p.layer[i - 1];
+      LayerRt &r = s->lr[i - 1];
+      CUtensorMap *m = &maps[(size_t)(i - 1) * MS_COUNT];
+      memset(m, 0, sizeof(CUtensorMap) * MS_COUNT);
+      ooo_status st;
+      if ((st = make_map(&m[MS_FWD_A], r.X, lp.din, p.M, 64, 128)) != OOO_OK ||
+          (st = make_map(&m[MS_FWD_B], r.W, lp.dout, lp.din, 64, 64)) != OOO_OK ||
+          (r.Xn && (st = make_map(&m[MS_FWD_X], r.Xn, lp.dout, p.M, 64, 32)) != OOO_OK) ||
+          (r.Z && (st = make_map(&m[MS_FWD_Z], r.Z, lp.dout, p.M, 64, 32)) != OOO_OK) ||
+          (st = make_map(&m[MS_DX_A], r.dZ, lp.dout, p.M, 64, 128)) != OOO_OK ||
+          (st = make_map(&m[MS_DX_B], r.W, lp.dout, lp.din, 64, lp.ebn_dx)) != OOO_OK ||
+          (st = make_map(&m[MS_DZ_X], r.dZ, lp.dout, p.M, 64, 32)) != OOO_OK ||
+          (st = make_map(&m[MS_DW_A], r.X, lp.din, p.M, 64, 64)) != OOO_OK ||
+          (st = make_map(&m[MS_DW_B], r.dZ, lp.dout, p.M, 64, 64)) != OOO_OK ||
+          (st = make_map(&m[MS_GW_X], r.gw, lp.dout, lp.din, 64, 32)) != OOO_OK)
+        return cleanup_fail(st);
+      ooo::eng::LayerDev &L = ldev[i - 1];
+      memset(&L, 0, sizeof(L));
+      L.bias = r.b;
+      L.Z = r.Z;
+      L.dbpart = r.db;
+      L.db_out = r.gb;
+      L.din = lp.din;
+      L.dout = lp.dout;
+      L.act = lp.act;
+      L.bucket = lp.bucket;
+      L.fwd_nt = (lp.dout + lp.ebn_fwd - 1) / lp.ebn_fwd;
+      L.dx_nt = (lp.din + lp.ebn_dx - 1) / lp.ebn_dx;
+      L.dw_tiles = ((lp.din + 127) / 128) * ((lp.dout + lp.ebn_dw - 1) / lp.ebn_dw);
+    }
+    cudaError_t ce = cudaMemcpy(s->ws + p.off_maps, maps.data(), maps.size() * sizeof(CUtensorMap),
+                                cudaMemcpyHostToDevice);
+    if (ce == cudaSuccess)
+      ce = cudaMemcpy(s->ws + p.off_layers, ldev.data(), ldev.size() * sizeof(ooo::eng::LayerDev),
+                      cudaMemcpyHostToDevice);
+    if (ce == cudaSuccess)
+      ce = cudaMemset(s->ws + p.off_ctr, 0, (size_t)(p.cl.bwd_base + p.cl.bwd_size) * 4);
+    if (ce != cudaSuccess)
+      return cleanup_fail(fail(OOO_ERR_CUDA, "engine tables upload: %s", cudaGetErrorString(ce)));
+    s->dmaps = reinterpret_cast<const CUtensorMap *>(s->ws + p.off_maps);
+    s->dlayers = reinterpret_cast<const ooo::eng::LayerDev *>(s->ws + p.off_layers);
+    s->ctr = reinterpret_cast<int32_t *>(s->ws + p.off_ctr);
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    // N > 1: leave SMs for the NCCL kernels the engine's counters wait on
+    const int reserve = d->world_size > 1 ? (d->nccl_max_ctas > 0 ? d->nccl_max_ctas : 16) : 0;
+    s->engine_ctas = std::max(1, sms - reserve);
+    s->engine_ctas = std::min(s->engine_ctas, env_int("OOO_ENGINE_CTAS", s->engine_ctas));
   }
   int least = 0, greatest = 0;
   cudaError_t e = cudaDeviceGetStreamPriorityRange(&least, &greatest);
@@ -796,9 +1106,11 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
     ncclUniqueId id;
     memcpy(&id, d->nccl_unique_id, sizeof(id));
     ncclResult_t r;
-    if (s->api->CommInitRankConfig && d->nccl_max_ctas > 0) {
+    // engine: NCCL must fit in the SMs the persistent kernels leave free
+    const int max_ctas = d->nccl_max_ctas > 0 ? d->nccl_max_ctas : (p.engine ? 16 : 0);
+    if (s->api->CommInitRankConfig && max_ctas > 0) {
       ncclConfig_t cfg = NCCL_CONFIG_INITIALIZER;
-      cfg.maxCTAs = d->nccl_max_ctas;
+      cfg.maxCTAs = max_ctas;
       r = s->api->CommInitRankConfig(&s->nccl, d->world_size, id, d->rank, &cfg);
     } else {
       r = s->api->CommInitRank(&s->nccl, d->world_size, id, d->rank);
@@ -957,3 +1269,12 @@ ooo_status ooo_timing_read(ooo_stack *s, ooo_launch_record *out, int32_t cap, in
 }
 
 }  // extern "C"
+
+#ifdef OOO_TRACE
+// Debug builds only (libooo_trace.so): device buffer of [task][4] u64 stamps
+// filled by the engine kernels (tools/engine_trace.py).
+extern "C" ooo_status ooo_debug_set_trace(void *dev_ptr) {
+  CU_TRY(ooo::eng::engine_set_trace(dev_ptr));
+  return OOO_OK;
+}
+#endif

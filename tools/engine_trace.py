@@ -1,0 +1,113 @@
+"""Per-task timeline of the persistent engine (debug build libooo_trace.so).
+
+    python -m paper_conf_eurosys_ohlks22_b200.build --trace
+    python tools/engine_trace.py [C2] [k]
+
+For each op of the forward and backward queues: number of tiles, time from
+the pass start to its first dispense / first input-ready / last completion,
+mean per-tile durations (dispense->ready = dependency wait, ready->acc =
+mainloop, acc->done = epilogue) and the number of distinct CTAs.  A tuning
+aid, not part of the product path.
+"""
+import os
+import sys
+
+ROOT = __file__.rsplit("/tools/", 1)[0]
+os.environ.setdefault("OOO_LIB", os.path.join(ROOT, "paper_conf_eurosys_ohlks22_b200", "lib", "libooo_trace.so"))
+sys.path.insert(0, ROOT)
+
+import ctypes  # noqa: E402
+
+import torch  # noqa: E402
+
+from paper_conf_eurosys_ohlks22_b200 import _lib, configs, synth  # noqa: E402
+from paper_conf_eurosys_ohlks22_b200.stack import OooStack, schedule_order  # noqa: E402
+
+
+def ebn(n):
+    for b in (256, 192, 128):
+        if n % b == 0:
+            return b
+    return 64
+
+
+def queue(cfg, D, in_order):
+    """(kind, layer, ntiles) in engine queue order (mirrors engine_backward)."""
+    MT = (cfg.tokens + 127) // 128
+    ops, pending = [], []
+
+    def add(op):
+        i = abs(op)
+        din, dout = cfg.dims[i - 1], cfg.dims[i]
+        if op > 0:
+            ops.append(("dX", i, MT * ((din + ebn(din) - 1) // ebn(din))))
+        else:
+            ops.append(("dW", i, ((din + 127) // 128) * ((dout + ebn(dout) - 1) // ebn(dout))))
+    for op in D:
+        if op > 0:
+            add(op)
+            for w in pending:
+                add(w)
+            pending = []
+        elif in_order:
+            add(op)
+        else:
+            pending.append(op)
+    for w in pending:
+        add(w)
+    return ops
+
+
+def report(name, ops, buf):
+    import numpy as np
+    raw = buf.cpu().numpy().view(np.uint64).reshape(-1, 4)
+    cta = (raw >> np.uint64(48)).astype(np.int64)
+    t = (raw & np.uint64((1 << 48) - 1)).astype(np.float64)
+    valid = t[:, 3] > 0
+    t0 = t[valid, 0].min()
+    t = (t - t0) / 1e3
+    print(f"== {name}: {int(valid.sum())} tasks, span {t[valid, 3].max():.1f} us")
+    first = 0
+    for kind, layer, n in ops:
+        s = slice(first, first + n)
+        first += n
+        tt = t[s]
+        print(f"{kind} L{layer:3d} tiles {n:4d} disp {tt[:,0].min():8.1f} ready {tt[:,1].min():8.1f}"
+              f"..{tt[:,1].max():8.1f} done {tt[:,3].min():8.1f}..{tt[:,3].max():8.1f}"
+              f" wait {np.mean(tt[:,1]-tt[:,0]):6.1f} main {np.mean(tt[:,2]-tt[:,1]):6.1f}"
+              f" epi {np.mean(tt[:,3]-tt[:,2]):5.1f} ctas {len(set(cta[s, 3]))}")
+
+
+def main():
+    cfg = configs.get(sys.argv[1] if len(sys.argv) > 1 else "C2")
+    k = int(sys.argv[2]) if len(sys.argv) > 2 else 12
+    lib = _lib.load()
+    lib.ooo_debug_set_trace.restype = ctypes.c_int32
+    lib.ooo_debug_set_trace.argtypes = [ctypes.c_void_p]
+    dev = torch.device("cuda")
+    W, b = synth.weights_torch(cfg.dims, cfg.acts, cfg.dtype, dev)
+    stk = OooStack(cfg.dims, cfg.acts, cfg.tokens, W, b, dtype=cfg.dtype)
+    X = synth.activations_torch(cfg.tokens, cfg.dims[0], cfg.dtype, dev, 1, 0, 0)
+    dY = synth.activations_torch(cfg.tokens, cfg.dims[-1], cfg.dtype, dev, 1, 0, 1)
+    Y = stk.forward(X)
+    for _ in range(3):
+        stk.backward(dY, "first_k", k)
+        stk.forward(X, Y)
+    torch.cuda.synchronize()
+    buf = torch.zeros(200000 * 4, dtype=torch.int64, device=dev)
+    _lib.check(lib.ooo_debug_set_trace(buf.data_ptr()))
+    stk.backward(dY, "first_k", k)
+    torch.cuda.synchronize()
+    D = schedule_order(cfg.L, "first_k", k)
+    report(f"backward first_k({k})", queue(cfg, D, False), buf)
+    buf.zero_()
+    stk.forward(X, Y)
+    torch.cuda.synchronize()
+    MT = (cfg.tokens + 127) // 128
+    fops = [("F", i, MT * ((cfg.dims[i] + ebn(cfg.dims[i]) - 1) // ebn(cfg.dims[i]))) for i in range(1, cfg.L + 1)]
+    report("forward", fops, buf)
+    _lib.check(lib.ooo_debug_set_trace(None))
+
+
+if __name__ == "__main__":
+    main()
