@@ -48,11 +48,13 @@ __device__ __forceinline__ void etrace(int t, int slot) {
 __device__ __forceinline__ void etrace(int, int) {}
 #endif
 
-constexpr int kThreads = 192;
+constexpr int kEpiWarps = 8;
+constexpr int kEpiThreads = 32 * kEpiWarps;
+constexpr int kThreads = 64 + kEpiThreads;
 constexpr int kMaxBN = 256;
 constexpr int B_BYTES = kMaxBN * BK * 2;             // 32 KiB
 constexpr int STAGE = A_BYTES + B_BYTES;             // 48 KiB
-constexpr int STG_BYTES = 4 * 4096;
+constexpr int STG_BYTES = kEpiWarps * 2048;
 constexpr int STAGES = 4;
 constexpr int Q = 4;                                 // task ring depth
 constexpr int RING = STAGE * STAGES;
@@ -66,6 +68,8 @@ constexpr int RED_OFF = BIAS_OFF + kMaxBN * 4;
 constexpr int SMEM = RED_OFF + 4 * kMaxBN * 4 + 1024;
 static_assert(SMEM <= kSmemBudget, "engine smem budget");
 constexpr uint32_t TMEM_COLS = 512;
+
+__device__ __forceinline__ void ebar() { asm volatile("bar.sync 1, %0;" ::"n"(kEpiThreads) : "memory"); }
 
 __device__ __forceinline__ int ld_acquire(const int32_t *p) {
   int v;
@@ -157,7 +161,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     for (int a = 0; a < 2; ++a) {
       mbar_init(bar_tfull + 8 * a, 1);
-      mbar_init(bar_tempty + 8 * a, 4);   // one arrive per epilogue warp
+      mbar_init(bar_tempty + 8 * a, kEpiWarps);   // one arrive per epilogue warp
     }
     for (int s = 0; s < Q; ++s) {
       mbar_init(bar_qfull + 8 * s, 1);
@@ -280,15 +284,16 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     __syncwarp();
   } else {
-    // ============ epilogue (warps 2..5) ============
-    const int q = warp & 3;
-    const int et = threadIdx.x - 64;
-    const uint32_t stg = sbase + STG_OFF + q * 4096;
+    // ============ epilogue (warps 2..9: two per TMEM lane quarter) ============
+    const int q = warp & 3;                  // lane quarter (TMEM access restriction)
+    const int h = (warp - 2) >> 2;           // column half: 32-col chunks c = h, h+2, ...
+    const int et = threadIdx.x - 64;         // 0..255
+    const uint32_t stg = sbase + STG_OFF + (warp - 2) * 2048;
     for (int j = 0;; ++j) {
       const int slot = j % Q;
       mbar_wait(bar_qfull + 8 * slot, (j / Q) & 1);
       const int t = task_slot[slot];
-      epi_bar();                                   // everyone read the slot; previous task done with smem
+      ebar();                                   // everyone read the slot; previous task done with smem
       if (et == 0) mbar_arrive(bar_qempty + 8 * slot);
       if (t < 0) break;
       const TaskRt T = task_rt(p, t);
@@ -304,74 +309,59 @@ __global__ void __launch_bounds__(kThreads, 1)
       float *dbpart = nullptr;
       if (T.kind == EPI_FWD) {
         const __nv_bfloat16 *bias = reinterpret_cast<const __nv_bfloat16 *>(Ld.bias);
-        for (int c = et; c < T.bn; c += 128) {
+        for (int c = et; c < T.bn; c += kEpiThreads) {
           const int n = T.n0 + c;
           bias_s[c] = n < T.N ? __bfloat162float(bias[n]) : 0.f;
         }
-        epi_bar();
+        ebar();
       } else if (T.kind == EPI_DGRAD && T.layer >= 2) {
         const LayerDev &Lp = p.layers[T.layer - 2];
         zin = reinterpret_cast<const __nv_bfloat16 *>(Lp.Z);   // null for identity act_{i-1}
         dbpart = Lp.dbpart;
       }
+      const int nch = T.bn / 32;
+      const bool need_z = (T.kind == EPI_DGRAD) && o.act != ACT_ID && zin != nullptr && row_ok;
+      const __nv_bfloat16 *zrow = zin ? zin + (size_t)row * T.N + T.n0 : nullptr;
+      uint4 zr[4];
+      if (need_z && h < nch) ld_raw32(zrow + h * 32, zr);     // act' input, prefetched before the wait
       mbar_wait(bar_tfull + 8 * acc, (j >> 1) & 1);
       fence_after();
       if (et == 0) etrace(t, 2);
-      const bool need_z = (T.kind == EPI_DGRAD) && o.act != ACT_ID && zin != nullptr && row_ok;
-      const __nv_bfloat16 *zrow = zin ? zin + (size_t)row * T.N + T.n0 : nullptr;
-      uint4 zr0[4], zr1[4];
-      if (need_z) {
-        ld_raw32(zrow, zr0);
-        ld_raw32(zrow + 32, zr1);
-      }
-      for (int c = 0; c < T.bn / 64; ++c) {
-        const int col0 = T.n0 + c * 64;
+      for (int c = h; c < nch; c += 2) {
+        const int col0 = T.n0 + c * 32;
         if (col0 >= T.N) break;
-        float v[64];
+        float v[32];
         {
           uint32_t r[32];
-          const uint32_t ta = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * kMaxBN + c * 64);
-          tmem_ld32(ta, r);
+          tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * kMaxBN + c * 32), r);
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
-          tmem_ld32(ta + 32, r);
-#pragma unroll
-          for (int i = 0; i < 32; ++i) v[32 + i] = __uint_as_float(r[i]);
         }
         if (T.kind == EPI_FWD) {
 #pragma unroll
-          for (int i = 0; i < 64; ++i) v[i] = __bfloat162float(__float2bfloat16_rn(v[i] + bias_s[c * 64 + i]));
-          if (mZ) stage_store(mZ, stg, lane, v, col0, row0);             // Z_i
+          for (int i = 0; i < 32; ++i) v[i] = __bfloat162float(__float2bfloat16_rn(v[i] + bias_s[c * 32 + i]));
+          if (mZ) stage_store32(mZ, stg, lane, v, col0, row0);           // Z_i
           if (o.act != ACT_ID) {
 #pragma unroll
-            for (int i = 0; i < 64; ++i) v[i] = act_f(o.act, v[i]);
+            for (int i = 0; i < 32; ++i) v[i] = act_f(o.act, v[i]);
           }
-          stage_store(mX, stg, lane, v, col0, row0);                     // X_{i+1} (or Y)
+          stage_store32(mX, stg, lane, v, col0, row0);                   // X_{i+1} (or Y)
         } else if (T.kind == EPI_DGRAD) {
           if (need_z) {
-            float z[64];
-            unpack_bf16x32(zr0, *reinterpret_cast<float(*)[32]>(&z[0]));
-            unpack_bf16x32(zr1, *reinterpret_cast<float(*)[32]>(&z[32]));
-            if (c + 1 < T.bn / 64 && col0 + 64 < T.N) {
-              ld_raw32(zrow + (c + 1) * 64, zr0);
-              ld_raw32(zrow + (c + 1) * 64 + 32, zr1);
-            }
+            float z[32];
+            unpack_bf16x32(zr, z);
+            if (c + 2 < nch && col0 + 64 < T.N) ld_raw32(zrow + (c + 2) * 32, zr);
 #pragma unroll
-            for (int i = 0; i < 64; ++i) v[i] *= act_grad_f(o.act, z[i]);
+            for (int i = 0; i < 32; ++i) v[i] *= act_grad_f(o.act, z[i]);
           }
 #pragma unroll
-          for (int i = 0; i < 64; ++i) v[i] = row_ok ? __bfloat162float(__float2bfloat16_rn(v[i])) : 0.f;
-          stage_store(mX, stg, lane, v, col0, row0);                     // dZ_{i-1} (or dX)
-          if (dbpart) {
-            const float s0 = warp_colsum32(*reinterpret_cast<float(*)[32]>(&v[0]), lane);
-            const float s1 = warp_colsum32(*reinterpret_cast<float(*)[32]>(&v[32]), lane);
-            red[q * kMaxBN + c * 64 + lane] = s0;
-            red[q * kMaxBN + c * 64 + 32 + lane] = s1;
-          }
+          for (int i = 0; i < 32; ++i) v[i] = row_ok ? __bfloat162float(__float2bfloat16_rn(v[i])) : 0.f;
+          stage_store32(mX, stg, lane, v, col0, row0);                   // dZ_{i-1} (or dX)
+          if (dbpart) red[q * kMaxBN + c * 32 + lane] = warp_colsum32(v, lane);
         } else {  // EPI_WGRAD: one split, scaled bf16 straight into the gradient bucket
 #pragma unroll
-          for (int i = 0; i < 64; ++i) v[i] *= p.alpha;
-          stage_store(mX, stg, lane, v, col0, row0);
+          for (int i = 0; i < 32; ++i) v[i] *= p.alpha;
+          stage_store32(mX, stg, lane, v, col0, row0);
         }
       }
       // accumulator buffer free for task j+2
@@ -379,8 +369,8 @@ __global__ void __launch_bounds__(kThreads, 1)
       __syncwarp();
       if (lane == 0) mbar_arrive(bar_tempty + 8 * acc);
       if (T.kind == EPI_DGRAD && dbpart) {
-        epi_bar();
-        for (int cc = et; cc < T.bn; cc += 128) {
+        ebar();
+        for (int cc = et; cc < T.bn; cc += kEpiThreads) {
           const int col = T.n0 + cc;
           if (col < T.N) {
             const float s = ((red[cc] + red[kMaxBN + cc]) + red[2 * kMaxBN + cc]) + red[3 * kMaxBN + cc];
@@ -392,7 +382,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         // db_i = (1/N) sum over row blocks of the bias-grad partials (fixed order)
         if (T.layer < cl.L) wait_ge(ctr + cl.dz_total + (T.layer - 1), cl.MT * p.layers[T.layer].dx_nt);
         __nv_bfloat16 *db = reinterpret_cast<__nv_bfloat16 *>(Ld.db_out);
-        for (int cc = et; cc < T.bn; cc += 128) {
+        for (int cc = et; cc < T.bn; cc += kEpiThreads) {
           const int col = T.n0 + cc;
           if (col < T.N) {
             float s = 0.f;
@@ -404,7 +394,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       // ---- publish completion: all bulk stores of the tile are done
       if (lane == 0) tma_store_wait_all();
       __syncwarp();
-      epi_bar();
+      ebar();
       if (et == 0) {
         asm volatile("fence.proxy.async.global;" ::: "memory");
         __threadfence();

@@ -338,7 +338,7 @@ EncodeTiledFn get_encode() {
 
 // 2-D bf16 row-major tensor [outer][inner], 128-B swizzled box {box_inner, box_outer}.
 ooo_status make_map(CUtensorMap *m, const void *ptr, uint64_t inner, uint64_t outer,
-                    uint32_t box_inner, uint32_t box_outer) {
+                    uint32_t box_inner, uint32_t box_outer, int swizzle_bytes = 128) {
   EncodeTiledFn enc = get_encode();
   if (!enc) return fail(OOO_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
   cuuint64_t dims[2] = {inner, outer};
@@ -346,7 +346,8 @@ ooo_status make_map(CUtensorMap *m, const void *ptr, uint64_t inner, uint64_t ou
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t es[2] = {1, 1};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(ptr), dims, strides, box,
-                   es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                   es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   swizzle_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_128B,
                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuTensorMapEncodeTiled failed (%d)", (int)r);
   return OOO_OK;
@@ -673,7 +674,7 @@ ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st)
   P.nops = L;
   P.ntasks = first;
   CUtensorMap tmY;
-  OOO_TRY(make_map(&tmY, Y, p.layer[L - 1].dout, p.M, 64, 32));
+  OOO_TRY(make_map(&tmY, Y, p.layer[L - 1].dout, p.M, 32, 32, 64));
   TimedRec *tr;
   OOO_TRY(begin_rec(s, s->hi, 7, 0, 0, &tr));
   CU_TRY(ooo::eng::launch_engine(P, &tmY, &tmY, s->engine_ctas, s->hi, s->prio_hi));
@@ -755,7 +756,7 @@ ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, void *dX
   P.nops = nops;
   P.ntasks = first;
   CUtensorMap tmDX;
-  if (dX) OOO_TRY(make_map(&tmDX, dX, s->dims[0], p.M, 64, 32));
+  if (dX) OOO_TRY(make_map(&tmDX, dX, s->dims[0], p.M, 32, 32, 64));
   else tmDX = s->lr[0].dxA;   // unused placeholder
   TimedRec *tr;
   OOO_TRY(begin_rec(s, s->hi, 8, 0, 0, &tr));
@@ -1033,14 +1034,14 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
       ooo_status st;
       if ((st = make_map(&m[MS_FWD_A], r.X, lp.din, p.M, 64, 128)) != OOO_OK ||
           (st = make_map(&m[MS_FWD_B], r.W, lp.dout, lp.din, 64, 64)) != OOO_OK ||
-          (r.Xn && (st = make_map(&m[MS_FWD_X], r.Xn, lp.dout, p.M, 64, 32)) != OOO_OK) ||
-          (r.Z && (st = make_map(&m[MS_FWD_Z], r.Z, lp.dout, p.M, 64, 32)) != OOO_OK) ||
+          (r.Xn && (st = make_map(&m[MS_FWD_X], r.Xn, lp.dout, p.M, 32, 32, 64)) != OOO_OK) ||
+          (r.Z && (st = make_map(&m[MS_FWD_Z], r.Z, lp.dout, p.M, 32, 32, 64)) != OOO_OK) ||
           (st = make_map(&m[MS_DX_A], r.dZ, lp.dout, p.M, 64, 128)) != OOO_OK ||
           (st = make_map(&m[MS_DX_B], r.W, lp.dout, lp.din, 64, lp.ebn_dx)) != OOO_OK ||
-          (st = make_map(&m[MS_DZ_X], r.dZ, lp.dout, p.M, 64, 32)) != OOO_OK ||
+          (st = make_map(&m[MS_DZ_X], r.dZ, lp.dout, p.M, 32, 32, 64)) != OOO_OK ||
           (st = make_map(&m[MS_DW_A], r.X, lp.din, p.M, 64, 64)) != OOO_OK ||
           (st = make_map(&m[MS_DW_B], r.dZ, lp.dout, p.M, 64, 64)) != OOO_OK ||
-          (st = make_map(&m[MS_GW_X], r.gw, lp.dout, lp.din, 64, 32)) != OOO_OK)
+          (st = make_map(&m[MS_GW_X], r.gw, lp.dout, lp.din, 32, 32, 64)) != OOO_OK)
         return cleanup_fail(st);
       ooo::eng::LayerDev &L = ldev[i - 1];
       memset(&L, 0, sizeof(L));

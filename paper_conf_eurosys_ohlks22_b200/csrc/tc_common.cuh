@@ -215,6 +215,25 @@ __device__ __forceinline__ void stage_store(const CUtensorMap *map, uint32_t buf
   __syncwarp();
   if (lane == 0) tma_store_2d(map, buf, col0, row0);
 }
+// Same for 32 rows x 32 columns into a 2 KiB 64B-swizzled buffer (16-B chunk
+// c of 64-B row r at chunk c ^ ((r >> 1) & 3): conflict-free), box {32, 32}.
+__device__ __forceinline__ void stage_store32(const CUtensorMap *map, uint32_t buf, int lane,
+                                              const float (&v)[32], int col0, int row0) {
+  if (lane == 0) tma_store_wait_read();
+  __syncwarp();
+  const uint32_t rbase = buf + lane * 64;
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    const uint32_t a = rbase + ((c ^ ((lane >> 1) & 3)) << 4);
+    asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a),
+                 "r"(pack_bf2(v[8 * c + 0], v[8 * c + 1])), "r"(pack_bf2(v[8 * c + 2], v[8 * c + 3])),
+                 "r"(pack_bf2(v[8 * c + 4], v[8 * c + 5])), "r"(pack_bf2(v[8 * c + 6], v[8 * c + 7]))
+                 : "memory");
+  }
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  __syncwarp();
+  if (lane == 0) tma_store_2d(map, buf, col0, row0);
+}
 
 }  // namespace tc
 }  // namespace ooo
