@@ -76,6 +76,16 @@ __device__ __forceinline__ int ld_acquire(const int32_t *p) {
   asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+// Polls use relaxed loads: an acquire at gpu scope invalidates the SM's L1
+// (CCTL.IVALL) every time, which would hurt the epilogue warps' cached loads.
+__device__ __forceinline__ int ld_relaxed(const int32_t *p) {
+  int v;
+  asm volatile("ld.relaxed.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void red_release_add(int32_t *p, int v) {
+  asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
 __device__ __forceinline__ uint64_t gtimer() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -84,12 +94,14 @@ __device__ __forceinline__ uint64_t gtimer() {
 // Wait until *p >= target.  A dependency that is not met within 4 s means a
 // broken schedule: trap (the launch fails with an error) instead of hanging.
 __device__ __forceinline__ void wait_ge(const int32_t *p, int target) {
-  if (ld_acquire(p) >= target) return;
-  const uint64_t t0 = gtimer();
-  while (ld_acquire(p) < target) {
-    __nanosleep(32);
-    if (gtimer() - t0 > 4000000000ull) __trap();
+  if (ld_relaxed(p) < target) {
+    const uint64_t t0 = gtimer();
+    while (ld_relaxed(p) < target) {
+      __nanosleep(32);
+      if (gtimer() - t0 > 4000000000ull) __trap();
+    }
   }
+  (void)ld_acquire(p);   // one acquire orders the producer tiles' stores before our reads
 }
 
 __device__ __forceinline__ const CUtensorMap *map_of(int idx, const CUtensorMap *maps,
@@ -303,8 +315,17 @@ __global__ void __launch_bounds__(kThreads, 1)
       const int row0 = T.m0 + q * 32;
       const int row = row0 + lane;
       const bool row_ok = row < T.M;
-      const CUtensorMap *mX = map_of(o.mapX, p.maps, &tmY, &tmDX);
-      const CUtensorMap *mZ = o.mapZ != MAP_NONE ? map_of(o.mapZ, p.maps, &tmY, &tmDX) : nullptr;
+      // outputs (row-major, ldc = N): F_i -> X_{i+1} (+ Z_i), dO_i -> dZ_{i-1} (or dX), dW_i -> bucket
+      __nv_bfloat16 *out;
+      __nv_bfloat16 *zout = nullptr;
+      if (T.kind == EPI_FWD) {
+        out = reinterpret_cast<__nv_bfloat16 *>(T.layer == cl.L ? p.y_out : Ld.Xn);
+        zout = reinterpret_cast<__nv_bfloat16 *>(const_cast<void *>(Ld.Z));
+      } else if (T.kind == EPI_DGRAD) {
+        out = reinterpret_cast<__nv_bfloat16 *>(T.layer >= 2 ? p.layers[T.layer - 2].dZ : p.dx_out);
+      } else {
+        out = reinterpret_cast<__nv_bfloat16 *>(Ld.gw);
+      }
       const __nv_bfloat16 *zin = nullptr;
       float *dbpart = nullptr;
       if (T.kind == EPI_FWD) {
@@ -320,7 +341,11 @@ __global__ void __launch_bounds__(kThreads, 1)
         dbpart = Lp.dbpart;
       }
       const int nch = T.bn / 32;
-      const bool need_z = (T.kind == EPI_DGRAD) && o.act != ACT_ID && zin != nullptr && row_ok;
+      // param-space fields -> registers once per task (see act_chunk32)
+      const int act = o.act;
+      const int dbg = p.dbg;
+      const float alpha = p.alpha;
+      const bool need_z = (T.kind == EPI_DGRAD) && act != ACT_ID && zin != nullptr && row_ok;
       const __nv_bfloat16 *zrow = zin ? zin + (size_t)row * T.N + T.n0 : nullptr;
       uint4 zr[4];
       if (need_z && h < nch) ld_raw32(zrow + h * 32, zr);     // act' input, prefetched before the wait
@@ -340,28 +365,24 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (T.kind == EPI_FWD) {
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = __bfloat162float(__float2bfloat16_rn(v[i] + bias_s[c * 32 + i]));
-          if (mZ) stage_store32(mZ, stg, lane, v, col0, row0);           // Z_i
-          if (o.act != ACT_ID) {
-#pragma unroll
-            for (int i = 0; i < 32; ++i) v[i] = act_f(o.act, v[i]);
-          }
-          stage_store32(mX, stg, lane, v, col0, row0);                   // X_{i+1} (or Y)
+          if (zout && !(dbg & 2)) store32_rows(zout, T.N, stg, lane, v, col0, row0, T.M);   // Z_i
+          if (!(dbg & 1)) act_chunk32(act, v);
+          if (!(dbg & 2)) store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);  // X_{i+1} (or Y)
         } else if (T.kind == EPI_DGRAD) {
-          if (need_z) {
+          if (need_z && !(dbg & 1)) {
             float z[32];
             unpack_bf16x32(zr, z);
             if (c + 2 < nch && col0 + 64 < T.N) ld_raw32(zrow + (c + 2) * 32, zr);
-#pragma unroll
-            for (int i = 0; i < 32; ++i) v[i] *= act_grad_f(o.act, z[i]);
+            act_grad_mul_chunk32(act, v, z);
           }
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = row_ok ? __bfloat162float(__float2bfloat16_rn(v[i])) : 0.f;
-          stage_store32(mX, stg, lane, v, col0, row0);                   // dZ_{i-1} (or dX)
+          if (!(dbg & 2)) store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);  // dZ_{i-1} (or dX)
           if (dbpart) red[q * kMaxBN + c * 32 + lane] = warp_colsum32(v, lane);
         } else {  // EPI_WGRAD: one split, scaled bf16 straight into the gradient bucket
 #pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] *= p.alpha;
-          stage_store32(mX, stg, lane, v, col0, row0);
+          for (int i = 0; i < 32; ++i) v[i] *= alpha;
+          store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);
         }
       }
       // accumulator buffer free for task j+2
@@ -391,29 +412,25 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
         }
       }
-      // ---- publish completion: all bulk stores of the tile are done
-      if (lane == 0) tma_store_wait_all();
-      __syncwarp();
+      // ---- publish completion (release): the tile's global stores happen-before the counter
       ebar();
       if (et == 0) {
-        asm volatile("fence.proxy.async.global;" ::: "memory");
-        __threadfence();
+        // release reductions are cumulative: every store of the tile (all
+        // epilogue warps, ordered by the barrier above) is visible before the count
         if (T.kind == EPI_FWD) {
-          atomicAdd(ctr + cl.fwd_base + 1 + (T.layer - 1) * cl.MT + T.mblk, 1);
+          red_release_add(ctr + cl.fwd_base + 1 + (T.layer - 1) * cl.MT + T.mblk, 1);
         } else if (T.kind == EPI_DGRAD) {
           if (T.layer >= 2) {
-            atomicAdd(ctr + cl.dz_rows + (T.layer - 2) * cl.MT + T.mblk, 1);
-            atomicAdd(ctr + cl.dz_total + (T.layer - 2), 1);
+            red_release_add(ctr + cl.dz_rows + (T.layer - 2) * cl.MT + T.mblk, 1);
+            red_release_add(ctr + cl.dz_total + (T.layer - 2), 1);
           }
         } else {
-          atomicAdd(ctr + cl.dw_done + (T.layer - 1), 1);
-          atomicAdd(ctr + cl.bucket_done + Ld.bucket, 1);
+          red_release_add(ctr + cl.dw_done + (T.layer - 1), 1);
+          red_release_add(ctr + cl.bucket_done + Ld.bucket, 1);
         }
         etrace(t, 3);
       }
     }
-    if (lane == 0) tma_store_wait_all();
-    __syncwarp();
   }
   fence_before();
   __syncthreads();

@@ -48,13 +48,17 @@ struct LayerDev {
   const void *Z;           // Z_i (bf16) or null (identity: act' = 1)
   float *dbpart;           // bias-grad partials of layer i [R][d_i]
   void *db_out;            // bucket slot of db_i (bf16)
+  void *Xn;                // X_{i+1} store (null for i = L: the caller's Y)
+  void *dZ;                // dZ_i store
+  void *gw;                // bucket slot of dW_i (bf16)
+  void *pad0;
   int32_t din, dout, act, bucket;
   int32_t fwd_nt;          // n-tiles of F_i over d_i
   int32_t dx_nt;           // n-tiles of dO_i over d_{i-1}
   int32_t dw_tiles;        // tiles of dW_i
-  int32_t pad;
+  int32_t pad1[9];
 };
-static_assert(sizeof(LayerDev) == 64, "LayerDev layout");
+static_assert(sizeof(LayerDev) == 128, "LayerDev layout");
 
 // Counter layout (int32, in the workspace):
 //   fwd region : [0] dispenser, [1 + i*MT + m] rows of X_{i+1} done (i = 0..L-1)
@@ -73,9 +77,12 @@ struct Params {
   int32_t in_order;        // dO_i also waits for dW_{i+1} (conventional backprop)
   int32_t gate_ar;         // F_i waits ar_done[bucket(i)] (N > 1)
   int32_t pass;            // 0 forward, 1 backward
+  int32_t dbg;             // tuning experiments only (OOO_DBG): bit0 skip act math, bit1 skip stores
   const CUtensorMap *maps;
   int32_t *ctr;            // counter array base
   const LayerDev *layers;  // index i-1
+  void *y_out;             // caller's Y (F_L output)
+  void *dx_out;            // caller's dX (dO_1 output, need_input_grad)
   CounterLayout cl;
   Op ops[kMaxOps];
 };

@@ -647,6 +647,8 @@ ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st)
   P.alpha = 1.0f / (float)s->d.world_size;
   P.gate_ar = gate ? 1 : 0;
   P.pass = 0;
+  P.dbg = env_int("OOO_DBG", 0);
+  P.y_out = Y;
   P.maps = s->dmaps;
   P.ctr = s->ctr;
   P.layers = s->dlayers;
@@ -703,6 +705,8 @@ ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, void *dX
   P.alpha = 1.0f / (float)s->d.world_size;
   P.in_order = in_order ? 1 : 0;
   P.pass = 1;
+  P.dbg = env_int("OOO_DBG", 0);
+  P.dx_out = dX;
   P.maps = s->dmaps;
   P.ctr = s->ctr;
   P.layers = s->dlayers;
@@ -1049,6 +1053,9 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
       L.Z = r.Z;
       L.dbpart = r.db;
       L.db_out = r.gb;
+      L.Xn = r.Xn;
+      L.dZ = r.dZ;
+      L.gw = r.gw;
       L.din = lp.din;
       L.dout = lp.dout;
       L.act = lp.act;

@@ -115,17 +115,67 @@ __device__ __forceinline__ uint32_t idesc_rt(int bn, bool a_mn, bool b_mn) {
 }
 
 // ------------------------------------------------------------ epilogue math
+// Phi(z) (standard normal CDF) and e^{-z^2/2} with one exponential:
+// erf(x) = 1 - t (a1 + t (a2 + ...)) e^{-x^2}, t = 1 / (1 + p x), x = |z| / sqrt(2)
+// (Abramowitz & Stegun 7.1.26, |error| <= 1.5e-7 -- three orders below the
+// bf16 rounding applied to every GELU output).  Branch-free, unlike erff.
+__device__ __forceinline__ void gauss_cdf_exp(float z, float &Phi, float &ez) {
+  const float x = fabsf(z) * 0.70710678118654752f;
+  float t;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(t) : "f"(fmaf(0.3275911f, x, 1.f)));   // 1 ulp, no slow path
+  const float poly =
+      t * fmaf(t, fmaf(t, fmaf(t, fmaf(t, 1.061405429f, -1.453152027f), 1.421413741f), -0.284496736f),
+               0.254829592f);
+  ez = __expf(-0.5f * z * z);
+  const float erf_abs = fmaf(-poly, ez, 1.f);
+  Phi = 0.5f * (1.f + copysignf(erf_abs, z));
+}
 __device__ __forceinline__ float act_f(int act, float z) {
   if (act == ACT_RELU) return z > 0.f ? z : 0.f;
-  if (act == ACT_GELU) return z * 0.5f * (1.f + erff(z * 0.70710678118654752f));
+  if (act == ACT_GELU) {
+    float Phi, ez;
+    gauss_cdf_exp(z, Phi, ez);
+    return z * Phi;                                   // gelu(z) = z Phi(z)
+  }
   return z;
 }
 __device__ __forceinline__ float act_grad_f(int act, float z) {
   if (act == ACT_RELU) return z > 0.f ? 1.f : 0.f;
-  if (act == ACT_GELU)
-    return 0.5f * (1.f + erff(z * 0.70710678118654752f)) +
-           z * 0.39894228040143268f * __expf(-0.5f * z * z);
+  if (act == ACT_GELU) {
+    float Phi, ez;
+    gauss_cdf_exp(z, Phi, ez);
+    return fmaf(z * 0.39894228040143268f, ez, Phi);   // gelu'(z) = Phi(z) + z phi(z)
+  }
   return 1.f;
+}
+// Whole-chunk activation / activation-gradient with the act switch hoisted
+// out of the element loop (act must be a register value, not a param-space
+// reference: the asm memory clobbers elsewhere would force a reload per element).
+__device__ __forceinline__ void act_chunk32(int act, float (&v)[32]) {
+  if (act == ACT_GELU) {
+#pragma unroll
+    for (int i = 0; i < 32; ++i) {
+      float Phi, ez;
+      gauss_cdf_exp(v[i], Phi, ez);
+      v[i] *= Phi;
+    }
+  } else if (act == ACT_RELU) {
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = fmaxf(v[i], 0.f);
+  }
+}
+__device__ __forceinline__ void act_grad_mul_chunk32(int act, float (&v)[32], const float (&z)[32]) {
+  if (act == ACT_GELU) {
+#pragma unroll
+    for (int i = 0; i < 32; ++i) {
+      float Phi, ez;
+      gauss_cdf_exp(z[i], Phi, ez);
+      v[i] *= fmaf(z[i] * 0.39894228040143268f, ez, Phi);
+    }
+  } else if (act == ACT_RELU) {
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] = z[i] > 0.f ? v[i] : 0.f;
+  }
 }
 __device__ __forceinline__ float bf_lo(uint32_t u) { return __uint_as_float(u << 16); }
 __device__ __forceinline__ float bf_hi(uint32_t u) { return __uint_as_float(u & 0xFFFF0000u); }
@@ -214,6 +264,38 @@ __device__ __forceinline__ void stage_store(const CUtensorMap *map, uint32_t buf
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   __syncwarp();
   if (lane == 0) tma_store_2d(map, buf, col0, row0);
+}
+// Store one warp's 32 rows x 32 columns (bf16, lane = row) to a row-major
+// global tensor through a 2 KiB per-warp smem transpose: lanes write their
+// row (4 x 16 B, 64B-swizzled -> conflict-free), then read back so that
+// each group of 4 lanes owns one 64-B row segment -> fully coalesced
+// st.global.v4.  No async engine involved (TMA bulk stores would queue
+// behind the producer's TMA loads), so nothing to wait for.
+__device__ __forceinline__ void store32_rows(__nv_bfloat16 *g, int ldc, uint32_t buf, int lane,
+                                             const float (&v)[32], int col0, int row0, int M) {
+  __syncwarp();                            // previous read-back of buf finished
+  const uint32_t rbase = buf + lane * 64;
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    const uint32_t a = rbase + ((c ^ ((lane >> 1) & 3)) << 4);
+    asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a),
+                 "r"(pack_bf2(v[8 * c + 0], v[8 * c + 1])), "r"(pack_bf2(v[8 * c + 2], v[8 * c + 3])),
+                 "r"(pack_bf2(v[8 * c + 4], v[8 * c + 5])), "r"(pack_bf2(v[8 * c + 6], v[8 * c + 7]))
+                 : "memory");
+  }
+  __syncwarp();
+  const int c = lane & 3;
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int r = (lane >> 2) + 8 * k;
+    uint32_t x, y, z, w;
+    asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(x), "=r"(y), "=r"(z), "=r"(w)
+                 : "r"(buf + r * 64 + ((c ^ ((r >> 1) & 3)) << 4))
+                 : "memory");
+    const int grow = row0 + r;
+    if (grow < M) *reinterpret_cast<uint4 *>(g + (size_t)grow * ldc + col0 + c * 8) = make_uint4(x, y, z, w);
+  }
 }
 // Same for 32 rows x 32 columns into a 2 KiB 64B-swizzled buffer (16-B chunk
 // c of 64-B row r at chunk c ^ ((r >> 1) & 3): conflict-free), box {32, 32}.
