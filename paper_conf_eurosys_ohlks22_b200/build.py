@@ -64,19 +64,22 @@ def _digest() -> str:
     return h.hexdigest()
 
 
-def build(force: bool = False, verbose: bool = True, trace: bool = False) -> str:
+def build(force: bool = False, verbose: bool = True, trace: bool = False, variant: str = "",
+          defines: tuple = ()) -> str:
     """trace=True builds the debug variant lib/libooo_trace.so (-DOOO_TRACE:
-    per-task timestamps in the engine, tools/engine_trace.py)."""
-    lib = LIB if not trace else os.path.join(LIBDIR, "libooo_trace.so")
-    objdir = OBJDIR if not trace else OBJDIR + "_trace"
+    per-task timestamps in the engine, tools/engine_trace.py); `variant` +
+    `defines` build tuning variants lib/libooo_<variant>.so."""
+    name = "libooo_trace.so" if trace else (f"libooo_{variant}.so" if variant else "libooo.so")
+    lib = os.path.join(LIBDIR, name)
+    objdir = OBJDIR + ("_trace" if trace else "") + (f"_{variant}" if variant else "")
     os.makedirs(LIBDIR, exist_ok=True)
     os.makedirs(objdir, exist_ok=True)
     stamp = os.path.splitext(lib)[0] + ".sha256"
-    dig = _digest() + ("-trace" if trace else "")
+    dig = _digest() + ("-trace" if trace else "") + "".join(defines)
     if not force and os.path.exists(lib) and os.path.exists(stamp) and open(stamp).read() == dig:
         return lib
     nvcc = _nvcc()
-    flags = _flags() + (["-DOOO_TRACE"] if trace else [])
+    flags = _flags() + (["-DOOO_TRACE"] if trace else []) + [f"-D{d}" for d in defines]
 
     def compile_one(src):
         obj = os.path.join(objdir, src + ".o")
@@ -103,4 +106,6 @@ def build(force: bool = False, verbose: bool = True, trace: bool = False) -> str
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, trace="--trace" in sys.argv)
+    defs = tuple(a[2:] for a in sys.argv[1:] if a.startswith("-D"))
+    var = next((a.split("=", 1)[1] for a in sys.argv[1:] if a.startswith("--variant=")), "")
+    build(force="--force" in sys.argv, trace="--trace" in sys.argv, variant=var, defines=defs)

@@ -1,23 +1,32 @@
 // Persistent dataflow engine kernel (see engine.h for the design rationale).
 //
+// Template CG = CTAs per tile (tcgen05 cta_group):
+//   CG = 1 : one CTA per 128 x bn tile, B fully in its smem (48 KiB stages).
+//   CG = 2 : a CTA pair (cluster of 2) per 256 x bn tile; CTA rank r owns rows
+//            [m0 + 128 r, +128) and streams its own 128 rows of A and half of
+//            B (bn/2 columns); the leader's single thread issues
+//            tcgen05.mma.cta_group::2 (M = 256), reading A and B from both
+//            CTAs, so each SM moves 32 KiB per k-block and 6 stages fit.
+// Each CTA's TMEM holds its 128 accumulator rows (2 buffers x 256 columns).
+//
 // Roles per CTA (one CTA per SM, persistent):
-//   warp 0 lane 0 : dispenser + TMA producer.  Takes the next task index
-//                   (atomicAdd on the pass dispenser, so tiles are started in
-//                   queue = priority order), publishes it to the other roles
-//                   through a 4-deep smem task ring, waits until the task's
-//                   input rows are complete (acquire on a completion counter,
-//                   spin with timeout -> trap, never a silent hang), then
-//                   streams its A / B k-blocks with TMA into the smem ring.
-//   warp 1        : TMEM allocator; lane 0 issues tcgen05.mma (M=128, N=bn)
-//                   into accumulator j & 1 (double-buffered, 2 x 256 cols).
-//   warps 2..5    : epilogue of task j while task j+1's MMAs run: tcgen05.ld,
+//   warp 0 lane 0 : producer.  The leader also dispenses: atomicAdd on the
+//                   pass dispenser gives the next task (queue = priority
+//                   order), written to the 4-deep smem task ring(s).
+//                   Each producer waits until its input rows are complete
+//                   (acquire on a completion counter, timeout -> trap), then
+//                   issues its TMA loads, completing on the leader's barrier.
+//   warp 1        : TMEM allocator; the leader's lane 0 issues the MMAs into
+//                   accumulator j & 1 (double-buffered).
+//   warps 2..9    : epilogue of task j while task j+1's MMAs run: tcgen05.ld,
 //                   fused bias/act (F_i), act-grad + bias-grad partials (dO_i),
-//                   1/N scale + bias-grad reduction (dW_i), bf16 RNE, TMA bulk
+//                   1/N scale + bias-grad reduction (dW_i), bf16 RNE, coalesced
 //                   stores; then publish completion (release) to the counters.
 // Deadlock freedom: tasks are dispensed in increasing index and every
 // dependency of task t is a task with a smaller index, all CTAs are
 // co-resident (grid <= #SMs, 1 CTA/SM), and each role processes its tasks in
-// order; so the smallest unfinished task can always make progress.
+// order; so the smallest unfinished task can always make progress.  Every
+// wait is bounded (globaltimer) and traps instead of hanging.
 #include <cuda.h>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -33,43 +42,124 @@ namespace eng {
 using namespace ooo::tc;
 
 #ifdef OOO_TRACE
-// Debug builds only (libooo_trace.so): per-task %globaltimer stamps
-// [task][4] = dispensed, inputs ready (TMA issue starts), accumulator ready,
-// completion published; plus the CTA that ran it in [task][4] high bits.
+// Debug builds only (libooo_trace.so): per-task stamps [task][8]:
+// globaltimer at dispensed / inputs ready / accumulator ready / published
+// (leader CTA; CTA index in the top 16 bits), then clock64 at the same points.
 __device__ unsigned long long *g_etrace = nullptr;
 __device__ __forceinline__ void etrace(int t, int slot) {
   if (g_etrace && t >= 0) {
     unsigned long long v;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(v));
-    g_etrace[(size_t)t * 4 + slot] = (v & 0xFFFFFFFFFFFFull) | ((unsigned long long)blockIdx.x << 48);
+    g_etrace[(size_t)t * 8 + slot] = (v & 0xFFFFFFFFFFFFull) | ((unsigned long long)blockIdx.x << 48);
+    g_etrace[(size_t)t * 8 + 4 + slot] = clock64();
   }
+}
+// epilogue phase clocks [task][8] (leader CTA, epilogue thread 0)
+__device__ unsigned long long *g_etrace2 = nullptr;
+__device__ __forceinline__ void etrace2(int t, int slot) {
+  if (g_etrace2 && t >= 0) g_etrace2[(size_t)t * 8 + slot] = clock64();
 }
 #else
 __device__ __forceinline__ void etrace(int, int) {}
+__device__ __forceinline__ void etrace2(int, int) {}
 #endif
 
-constexpr int kEpiWarps = 8;
+#ifndef OOO_EPI_WARPS
+#define OOO_EPI_WARPS 8
+#endif
+constexpr int kEpiWarps = OOO_EPI_WARPS;             // multiple of 4 (TMEM lane quarters)
+constexpr int kEpiPerQ = kEpiWarps / 4;              // warps sharing a lane quarter (column split)
 constexpr int kEpiThreads = 32 * kEpiWarps;
 constexpr int kThreads = 64 + kEpiThreads;
 constexpr int kMaxBN = 256;
-constexpr int B_BYTES = kMaxBN * BK * 2;             // 32 KiB
-constexpr int STAGE = A_BYTES + B_BYTES;             // 48 KiB
 constexpr int STG_BYTES = kEpiWarps * 2048;
-constexpr int STAGES = 4;
 constexpr int Q = 4;                                 // task ring depth
-constexpr int RING = STAGE * STAGES;
-constexpr int STG_OFF = RING;
-constexpr int BAR_OFF = STG_OFF + STG_BYTES;
-// full[S] empty[S] tfull[2] tempty[2] taskfull[Q] taskempty[Q]
-constexpr int SLOT_OFF = BAR_OFF + (2 * STAGES + 4 + 2 * Q) * 8;
-constexpr int TASK_OFF = SLOT_OFF + 16;
-constexpr int BIAS_OFF = (TASK_OFF + 4 * Q + 15) / 16 * 16;
-constexpr int RED_OFF = BIAS_OFF + kMaxBN * 4;
-constexpr int SMEM = RED_OFF + 4 * kMaxBN * 4 + 1024;
-static_assert(SMEM <= kSmemBudget, "engine smem budget");
 constexpr uint32_t TMEM_COLS = 512;
+constexpr uint64_t kTimeoutNs = 4000000000ull;
+
+template <int CG> struct Cfg {
+  static constexpr int B_BYTES = (kMaxBN / CG) * BK * 2;   // this CTA's share of B
+  static constexpr int STAGE = A_BYTES + B_BYTES;
+  static constexpr int STAGES = CG == 2 ? 6 : 4;
+  static constexpr int RING = STAGE * STAGES;
+  static constexpr int STG_OFF = RING;
+  static constexpr int BAR_OFF = STG_OFF + STG_BYTES;
+  // full[S] empty[S] tfull[2] tempty[2] taskfull[Q] taskempty[Q]
+  static constexpr int SLOT_OFF = BAR_OFF + (2 * STAGES + 4 + 2 * Q) * 8;
+  static constexpr int TASK_OFF = SLOT_OFF + 16;
+  static constexpr int BIAS_OFF = (TASK_OFF + 4 * Q + 15) / 16 * 16;
+  static constexpr int RED_OFF = BIAS_OFF + kMaxBN * 4;
+  static constexpr int SMEM = RED_OFF + 4 * kMaxBN * 4 + 1024;
+  static_assert(SMEM <= kSmemBudget, "engine smem budget");
+  static_assert(STAGE % 1024 == 0, "stage alignment");
+};
 
 __device__ __forceinline__ void ebar() { asm volatile("bar.sync 1, %0;" ::"n"(kEpiThreads) : "memory"); }
+
+__device__ __forceinline__ uint64_t gtimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// ---- cluster (CTA pair) helpers
+__device__ __forceinline__ uint32_t cta_rank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+__device__ __forceinline__ uint32_t mapa(uint32_t addr, uint32_t rank) {
+  uint32_t r;
+  asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(r) : "r"(addr), "r"(rank));
+  return r;
+}
+__device__ __forceinline__ void cluster_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+__device__ __forceinline__ void st_cluster_u32(uint32_t cluster_addr, int v) {
+  asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(cluster_addr), "r"(v) : "memory");
+}
+// Bounded mbarrier wait with the default (CTA-scope) semantics.  Spinning
+// with .acquire.cluster would emit an L1 invalidation (CCTL.IVALL) on every
+// poll -- measured at 2/3 of all warp samples.
+__device__ __forceinline__ void mbar_wait_b(uint32_t bar, uint32_t parity) {
+  if (mbar_try_wait(bar, parity)) return;
+  const uint64_t t0 = gtimer();
+  while (!mbar_try_wait(bar, parity))
+    if (gtimer() - t0 > kTimeoutNs) __trap();
+}
+// For barriers that receive arrivals from the peer CTA (release.cluster):
+// one cluster-scope acquire fence after the wait, not one per poll.
+__device__ __forceinline__ void mbar_wait_cl(uint32_t bar, uint32_t parity) {
+  mbar_wait_b(bar, parity);
+  asm volatile("fence.acq_rel.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void tma_load_2d_pair(uint32_t dst, const CUtensorMap *map, uint32_t leader_bar,
+                                                 int c0, int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
+      " [%0], [%1, {%3, %4}], [%2];" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(leader_bar), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void umma_bf16_pair(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc, uint32_t idesc,
+                                               uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
+}
+// completion of the leader's MMAs arrives on the same barrier in both CTAs
+__device__ __forceinline__ void umma_commit_pair(uint32_t bar) {
+  asm volatile(
+      "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+          bar),
+      "h"((unsigned short)3)
+      : "memory");
+}
 
 __device__ __forceinline__ int ld_acquire(const int32_t *p) {
   int v;
@@ -86,11 +176,6 @@ __device__ __forceinline__ int ld_relaxed(const int32_t *p) {
 __device__ __forceinline__ void red_release_add(int32_t *p, int v) {
   asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
-__device__ __forceinline__ uint64_t gtimer() {
-  uint64_t t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
-}
 // Wait until *p >= target.  A dependency that is not met within 4 s means a
 // broken schedule: trap (the launch fails with an error) instead of hanging.
 __device__ __forceinline__ void wait_ge(const int32_t *p, int target) {
@@ -98,7 +183,7 @@ __device__ __forceinline__ void wait_ge(const int32_t *p, int target) {
     const uint64_t t0 = gtimer();
     while (ld_relaxed(p) < target) {
       __nanosleep(32);
-      if (gtimer() - t0 > 4000000000ull) __trap();
+      if (gtimer() - t0 > kTimeoutNs) __trap();
     }
   }
   (void)ld_acquire(p);   // one acquire orders the producer tiles' stores before our reads
@@ -121,8 +206,9 @@ __device__ __forceinline__ int op_of(const Params &p, int t) {
 }
 
 struct TaskRt {
-  int op, kind, layer, bn, nkb, m0, n0, M, N, mblk;
+  int op, kind, layer, bn, nkb, m0, n0, M, N, mblk0;   // m0 / mblk0: first row (block) of the tile
 };
+template <int CG>
 __device__ __forceinline__ TaskRt task_rt(const Params &p, int t) {
   TaskRt r;
   r.op = op_of(p, t);
@@ -132,8 +218,8 @@ __device__ __forceinline__ TaskRt task_rt(const Params &p, int t) {
   r.layer = o.layer;
   r.bn = o.bn;
   r.nkb = o.nkb;
-  r.mblk = rel / o.nt;
-  r.m0 = r.mblk * BM;
+  r.mblk0 = o.m_off + CG * (rel / o.nt);
+  r.m0 = r.mblk0 * BM;
   r.n0 = (rel % o.nt) * o.bn;
   const LayerDev &L = p.layers[o.layer - 1];
   if (o.kind == EPI_FWD) { r.M = p.M; r.N = L.dout; }
@@ -142,86 +228,119 @@ __device__ __forceinline__ TaskRt task_rt(const Params &p, int t) {
   return r;
 }
 
+template <int CG>
 __global__ void __launch_bounds__(kThreads, 1)
     engine_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constant__ CUtensorMap tmDX,
                   const __grid_constant__ Params p) {
+  using C = Cfg<CG>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                               ~static_cast<uintptr_t>(1023));
   const uint32_t sbase = smem_u32(smem);
-  const uint32_t bar_full = sbase + BAR_OFF;
-  const uint32_t bar_empty = bar_full + 8 * STAGES;
-  const uint32_t bar_tfull = bar_empty + 8 * STAGES;
+  const uint32_t bar_full = sbase + C::BAR_OFF;
+  const uint32_t bar_empty = bar_full + 8 * C::STAGES;
+  const uint32_t bar_tfull = bar_empty + 8 * C::STAGES;
   const uint32_t bar_tempty = bar_tfull + 16;
   const uint32_t bar_qfull = bar_tempty + 16;
   const uint32_t bar_qempty = bar_qfull + 8 * Q;
-  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(smem + SLOT_OFF);
-  volatile int *task_slot = reinterpret_cast<volatile int *>(smem + TASK_OFF);
-  float *bias_s = reinterpret_cast<float *>(smem + BIAS_OFF);
-  float *red = reinterpret_cast<float *>(smem + RED_OFF);
+  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(smem + C::SLOT_OFF);
+  volatile int *task_slot = reinterpret_cast<volatile int *>(smem + C::TASK_OFF);
+  float *bias_s = reinterpret_cast<float *>(smem + C::BIAS_OFF);
+  float *red = reinterpret_cast<float *>(smem + C::RED_OFF);
   int32_t *ctr = p.ctr;
   const CounterLayout &cl = p.cl;
   int32_t *dispenser = ctr + (p.pass == 0 ? cl.fwd_base : cl.bwd_base);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
+  const uint32_t rank = CG == 2 ? cta_rank() : 0;   // 0 = leader (issues the MMAs)
+  const bool leader = rank == 0;
 
   if (warp == 0 && lane == 0) {
-    for (int s = 0; s < STAGES; ++s) {
-      mbar_init(bar_full + 8 * s, 1);
-      mbar_init(bar_empty + 8 * s, 1);
+    for (int s = 0; s < C::STAGES; ++s) {
+      mbar_init(bar_full + 8 * s, 1);           // leader's expect_tx arrival (+ the CTAs' bytes)
+      mbar_init(bar_empty + 8 * s, 1);          // leader's MMA commit
     }
     for (int a = 0; a < 2; ++a) {
-      mbar_init(bar_tfull + 8 * a, 1);
-      mbar_init(bar_tempty + 8 * a, kEpiWarps);   // one arrive per epilogue warp
+      mbar_init(bar_tfull + 8 * a, 1);          // leader's MMA commit
+      mbar_init(bar_tempty + 8 * a, CG * kEpiWarps);   // epilogue warps of all CTAs (leader's copy)
     }
     for (int s = 0; s < Q; ++s) {
-      mbar_init(bar_qfull + 8 * s, 1);
-      mbar_init(bar_qempty + 8 * s, 2);   // MMA lane + epilogue leader
+      mbar_init(bar_qfull + 8 * s, 1);          // leader's producer
+      mbar_init(bar_qempty + 8 * s, 2 * CG);    // MMA + epi (+ peer producer + peer epi)
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   }
   if (warp == 1) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
-                     smem_u32(tmem_slot)),
-                 "r"(TMEM_COLS)
-                 : "memory");
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    if (CG == 2) {
+      asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                       smem_u32(tmem_slot)),
+                   "r"(TMEM_COLS)
+                   : "memory");
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;" ::: "memory");
+    } else {
+      asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                       smem_u32(tmem_slot)),
+                   "r"(TMEM_COLS)
+                   : "memory");
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+    }
   }
   fence_before();
-  __syncthreads();
+  if (CG == 2) cluster_sync(); else __syncthreads();
   fence_after();
   const uint32_t tmem = *tmem_slot;
   pdl_wait();
+  // the leader's barriers as seen from this CTA (== local ones for CG = 1)
+  const uint32_t L_full = CG == 2 ? mapa(bar_full, 0) : bar_full;
+  const uint32_t L_tempty = CG == 2 ? mapa(bar_tempty, 0) : bar_tempty;
+  const uint32_t L_qempty = CG == 2 ? mapa(bar_qempty, 0) : bar_qempty;
 
   if (warp == 0) {
-    // ============ dispenser + TMA producer ============
+    // ============ dispenser (leader) + TMA producer ============
     if (lane == 0) {
+      const uint32_t P_qfull = CG == 2 ? mapa(bar_qfull, 1) : 0;
+      const uint32_t P_slot = CG == 2 ? mapa(smem_u32(const_cast<int *>(task_slot)), 1) : 0;
       int it = 0;
       for (int j = 0;; ++j) {
-        int t = atomicAdd(dispenser, 1);
-        if (t >= p.ntasks) t = -1;
-        etrace(t, 0);
         const int slot = j % Q;
-        if (j >= Q) mbar_wait(bar_qempty + 8 * slot, ((j / Q) - 1) & 1);
-        task_slot[slot] = t;
-        mbar_arrive(bar_qfull + 8 * slot);
+        int t;
+        if (leader) {
+          t = atomicAdd(dispenser, 1);
+          if (t >= p.ntasks) t = -1;
+          etrace(t, 0);
+          if (j >= Q) {
+            if (CG == 2) mbar_wait_cl(bar_qempty + 8 * slot, ((j / Q) - 1) & 1);
+            else mbar_wait_b(bar_qempty + 8 * slot, ((j / Q) - 1) & 1);
+          }
+          task_slot[slot] = t;
+          mbar_arrive(bar_qfull + 8 * slot);
+          if (CG == 2) {
+            st_cluster_u32(P_slot + 4 * slot, t);
+            mbar_arrive_cluster(P_qfull + 8 * slot);
+          }
+        } else {
+          mbar_wait_cl(bar_qfull + 8 * slot, (j / Q) & 1);
+          t = task_slot[slot];
+          mbar_arrive_cluster(L_qempty + 8 * slot);
+        }
         if (t < 0) break;
-        const TaskRt T = task_rt(p, t);
+        const TaskRt T = task_rt<CG>(p, t);
         const Op &o = p.ops[T.op];
         const LayerDev &Ld = p.layers[T.layer - 1];
+        const int mblk = T.mblk0 + (int)rank;    // this CTA's row block
         // ---- dependencies (all on tasks with smaller indices)
         if (T.kind == EPI_FWD) {
-          if (T.layer > 1) {
+          if (T.layer > 1 && mblk < cl.MT) {
             const LayerDev &Lp = p.layers[T.layer - 2];
-            wait_ge(ctr + cl.fwd_base + 1 + (T.layer - 2) * cl.MT + T.mblk, Lp.fwd_nt);
+            wait_ge(ctr + cl.fwd_base + 1 + (T.layer - 2) * cl.MT + mblk, Lp.fwd_nt);
           }
           if (p.gate_ar) wait_ge(ctr + cl.ar_done + Ld.bucket, 1);
         } else if (T.kind == EPI_DGRAD) {
           if (T.layer < cl.L) {
             const LayerDev &Ln = p.layers[T.layer];
-            wait_ge(ctr + cl.dz_rows + (T.layer - 1) * cl.MT + T.mblk, Ln.dx_nt);
+            if (mblk < cl.MT) wait_ge(ctr + cl.dz_rows + (T.layer - 1) * cl.MT + mblk, Ln.dx_nt);
             if (p.in_order) wait_ge(ctr + cl.dw_done + T.layer, Ln.dw_tiles);
           }
         } else {
@@ -231,88 +350,120 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
         }
         asm volatile("fence.proxy.async.global;" ::: "memory");   // TMA reads see the producers' data
-        etrace(t, 1);
+        if (leader) etrace(t, 1);
         const CUtensorMap *mA = map_of(o.mapA, p.maps, &tmY, &tmDX);
         const CUtensorMap *mB = map_of(o.mapB, p.maps, &tmY, &tmDX);
+        tma_prefetch(mA);      // descriptors live in global memory: warm the TMA descriptor cache
+        tma_prefetch(mB);
         const bool a_mn = T.kind == EPI_WGRAD;
         const bool b_mn = T.kind != EPI_DGRAD;
-        const uint32_t bytes = A_BYTES + T.bn * BK * 2;
+        const int bh = T.bn / CG;                                 // this CTA's B columns
+        const uint32_t bytes = CG * (A_BYTES + bh * BK * 2);      // all CTAs, on the leader's barrier
+        const int am = T.m0 + BM * (int)rank;
+        const int bn0 = T.n0 + bh * (int)rank;
         for (int kb = 0; kb < T.nkb; ++kb, ++it) {
-          const int s = it % STAGES;
-          if (it >= STAGES) mbar_wait(bar_empty + 8 * s, ((it / STAGES) - 1) & 1);
-          const uint32_t fb = bar_full + 8 * s;
-          mbar_expect_tx(fb, bytes);
-          const uint32_t sa = sbase + s * STAGE;
+          const int s = it % C::STAGES;
+          if (it >= C::STAGES) mbar_wait_b(bar_empty + 8 * s, ((it / C::STAGES) - 1) & 1);
+          if (leader) mbar_expect_tx(bar_full + 8 * s, bytes);
+          const uint32_t lb = L_full + 8 * s;
+          const uint32_t sa = sbase + s * C::STAGE;
           const uint32_t sb = sa + A_BYTES;
           const int k0 = kb * BK;
-          if (!a_mn) {
-            tma_load_2d(sa, mA, fb, k0, T.m0);                 // box {64 K, 128 M}
+          if (CG == 2) {
+            if (!a_mn) {
+              tma_load_2d_pair(sa, mA, lb, k0, am);                // box {64 K, 128 M}
+            } else {
+              tma_load_2d_pair(sa, mA, lb, am, k0);                // box {64 M, 64 K}
+              tma_load_2d_pair(sa + 8192, mA, lb, am + 64, k0);
+            }
+            if (!b_mn) {
+              tma_load_2d_pair(sb, mB, lb, k0, bn0);               // box {64 K, bn/2 N}
+            } else {
+              for (int c = 0; c < bh / 64; ++c) tma_load_2d_pair(sb + 8192 * c, mB, lb, bn0 + 64 * c, k0);
+            }
           } else {
-            tma_load_2d(sa, mA, fb, T.m0, k0);                 // box {64 M, 64 K}
-            tma_load_2d(sa + 8192, mA, fb, T.m0 + 64, k0);
-          }
-          if (!b_mn) {
-            tma_load_2d(sb, mB, fb, k0, T.n0);                 // box {64 K, bn N}
-          } else {
-            for (int c = 0; c < T.bn / 64; ++c) tma_load_2d(sb + 8192 * c, mB, fb, T.n0 + 64 * c, k0);
+            if (!a_mn) {
+              tma_load_2d(sa, mA, lb, k0, am);
+            } else {
+              tma_load_2d(sa, mA, lb, am, k0);
+              tma_load_2d(sa + 8192, mA, lb, am + 64, k0);
+            }
+            if (!b_mn) {
+              tma_load_2d(sb, mB, lb, k0, bn0);                    // box {64 K, bn N}
+            } else {
+              for (int c = 0; c < bh / 64; ++c) tma_load_2d(sb + 8192 * c, mB, lb, bn0 + 64 * c, k0);
+            }
           }
         }
       }
     }
   } else if (warp == 1) {
-    // ============ MMA issuer ============
-    if (lane == 0) {
+    // ============ MMA issuer (leader CTA only) ============
+    if (leader && lane == 0) {
       int it = 0;
       for (int j = 0;; ++j) {
         const int slot = j % Q;
-        mbar_wait(bar_qfull + 8 * slot, (j / Q) & 1);
+        mbar_wait_b(bar_qfull + 8 * slot, (j / Q) & 1);
         const int t = task_slot[slot];
         mbar_arrive(bar_qempty + 8 * slot);
         if (t < 0) break;
-        const TaskRt T = task_rt(p, t);
+        const TaskRt T = task_rt<CG>(p, t);
         const bool a_mn = T.kind == EPI_WGRAD;
         const bool b_mn = T.kind != EPI_DGRAD;
-        const uint32_t ID = idesc_rt(T.bn, a_mn, b_mn);
+        // M = 128 * CG across the CTAs, N = bn
+        const uint32_t ID = (1u << 4) | (1u << 7) | (1u << 10) | ((a_mn ? 1u : 0u) << 15) |
+                            ((b_mn ? 1u : 0u) << 16) | ((uint32_t)(T.bn >> 3) << 17) |
+                            ((uint32_t)((BM * CG) >> 4) << 24);
         const int acc = j & 1;
-        if (j >= 2) mbar_wait(bar_tempty + 8 * acc, ((j >> 1) - 1) & 1);
+        if (j >= 2) {
+          if (CG == 2) mbar_wait_cl(bar_tempty + 8 * acc, ((j >> 1) - 1) & 1);
+          else mbar_wait_b(bar_tempty + 8 * acc, ((j >> 1) - 1) & 1);
+        }
         fence_after();
         const uint32_t dtm = tmem + (uint32_t)(acc * kMaxBN);
         for (int kb = 0; kb < T.nkb; ++kb, ++it) {
-          const int s = it % STAGES;
-          mbar_wait(bar_full + 8 * s, (it / STAGES) & 1);
+          const int s = it % C::STAGES;
+          mbar_wait_b(bar_full + 8 * s, (it / C::STAGES) & 1);
           fence_after();
-          const uint32_t sa = sbase + s * STAGE;
+          const uint32_t sa = sbase + s * C::STAGE;
           const uint32_t sb = sa + A_BYTES;
 #pragma unroll
           for (int kk = 0; kk < BK / 16; ++kk) {
             const uint64_t ad = a_mn ? sdesc(sa + kk * 2048, 8192, 1024) : sdesc(sa + kk * 32, 16, 1024);
             const uint64_t bd = b_mn ? sdesc(sb + kk * 2048, 8192, 1024) : sdesc(sb + kk * 32, 16, 1024);
-            umma_bf16(dtm, ad, bd, ID, (kb | kk) != 0 ? 1u : 0u);
+            if (CG == 2) umma_bf16_pair(dtm, ad, bd, ID, (kb | kk) != 0 ? 1u : 0u);
+            else umma_bf16(dtm, ad, bd, ID, (kb | kk) != 0 ? 1u : 0u);
           }
-          umma_commit(bar_empty + 8 * s);
+          if (CG == 2) umma_commit_pair(bar_empty + 8 * s); else umma_commit(bar_empty + 8 * s);
         }
-        umma_commit(bar_tfull + 8 * acc);
+        if (CG == 2) umma_commit_pair(bar_tfull + 8 * acc); else umma_commit(bar_tfull + 8 * acc);
       }
     }
     __syncwarp();
   } else {
     // ============ epilogue (warps 2..9: two per TMEM lane quarter) ============
     const int q = warp & 3;                  // lane quarter (TMEM access restriction)
-    const int h = (warp - 2) >> 2;           // column half: 32-col chunks c = h, h+2, ...
+    const int h = (warp - 2) >> 2;           // column slot: 32-col chunks c = h, h + kEpiPerQ, ...
     const int et = threadIdx.x - 64;         // 0..255
-    const uint32_t stg = sbase + STG_OFF + (warp - 2) * 2048;
+    const uint32_t stg = sbase + C::STG_OFF + (warp - 2) * 2048;
     for (int j = 0;; ++j) {
       const int slot = j % Q;
-      mbar_wait(bar_qfull + 8 * slot, (j / Q) & 1);
+      if (leader) mbar_wait_b(bar_qfull + 8 * slot, (j / Q) & 1);
+      else mbar_wait_cl(bar_qfull + 8 * slot, (j / Q) & 1);
       const int t = task_slot[slot];
       ebar();                                   // everyone read the slot; previous task done with smem
-      if (et == 0) mbar_arrive(bar_qempty + 8 * slot);
+      if (et == 0) {
+        if (leader) mbar_arrive(bar_qempty + 8 * slot);
+        else mbar_arrive_cluster(L_qempty + 8 * slot);
+      }
       if (t < 0) break;
-      const TaskRt T = task_rt(p, t);
+      const TaskRt T = task_rt<CG>(p, t);
       const Op &o = p.ops[T.op];
       const LayerDev &Ld = p.layers[T.layer - 1];
       const int acc = j & 1;
-      const int row0 = T.m0 + q * 32;
+      const int mblk = T.mblk0 + (int)rank;
+      const int mrow0 = T.m0 + BM * (int)rank;  // this CTA's first row
+      const int row0 = mrow0 + q * 32;
       const int row = row0 + lane;
       const bool row_ok = row < T.M;
       // outputs (row-major, ldc = N): F_i -> X_{i+1} (+ Z_i), dO_i -> dZ_{i-1} (or dX), dW_i -> bucket
@@ -349,10 +500,12 @@ __global__ void __launch_bounds__(kThreads, 1)
       const __nv_bfloat16 *zrow = zin ? zin + (size_t)row * T.N + T.n0 : nullptr;
       uint4 zr[4];
       if (need_z && h < nch) ld_raw32(zrow + h * 32, zr);     // act' input, prefetched before the wait
-      mbar_wait(bar_tfull + 8 * acc, (j >> 1) & 1);
+      mbar_wait_b(bar_tfull + 8 * acc, (j >> 1) & 1);
       fence_after();
-      if (et == 0) etrace(t, 2);
-      for (int c = h; c < nch; c += 2) {
+      if (et == 0 && leader) etrace(t, 2);
+      const bool tr2 = et == 0 && leader;
+      if (tr2) etrace2(t, 0);
+      for (int c = h; c < ((dbg & 4) ? 0 : nch); c += kEpiPerQ) {
         const int col0 = T.n0 + c * 32;
         if (col0 >= T.N) break;
         float v[32];
@@ -362,6 +515,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
         }
+        if (tr2 && c == h) etrace2(t, 1);
         if (T.kind == EPI_FWD) {
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = __bfloat162float(__float2bfloat16_rn(v[i] + bias_s[c * 32 + i]));
@@ -372,7 +526,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (need_z && !(dbg & 1)) {
             float z[32];
             unpack_bf16x32(zr, z);
-            if (c + 2 < nch && col0 + 64 < T.N) ld_raw32(zrow + (c + 2) * 32, zr);
+            if (c + kEpiPerQ < nch && col0 + 32 * kEpiPerQ < T.N) ld_raw32(zrow + (c + kEpiPerQ) * 32, zr);
             act_grad_mul_chunk32(act, v, z);
           }
 #pragma unroll
@@ -384,22 +538,27 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int i = 0; i < 32; ++i) v[i] *= alpha;
           store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);
         }
+        if (tr2 && c == h) etrace2(t, 2);
       }
-      // accumulator buffer free for task j+2
+      if (tr2) etrace2(t, 3);
+      // accumulator buffer free for task j+2 (the leader's barrier counts all CTAs)
       fence_before();
       __syncwarp();
-      if (lane == 0) mbar_arrive(bar_tempty + 8 * acc);
-      if (T.kind == EPI_DGRAD && dbpart) {
+      if (lane == 0) {
+        if (leader) mbar_arrive(bar_tempty + 8 * acc);
+        else mbar_arrive_cluster(L_tempty + 8 * acc);
+      }
+      if (T.kind == EPI_DGRAD && dbpart && mblk < cl.MT) {
         ebar();
         for (int cc = et; cc < T.bn; cc += kEpiThreads) {
           const int col = T.n0 + cc;
           if (col < T.N) {
             const float s = ((red[cc] + red[kMaxBN + cc]) + red[2 * kMaxBN + cc]) + red[3 * kMaxBN + cc];
-            dbpart[(size_t)T.mblk * T.N + col] = s;
+            dbpart[(size_t)mblk * T.N + col] = s;
           }
         }
       }
-      if (T.kind == EPI_WGRAD && T.m0 == 0) {
+      if (T.kind == EPI_WGRAD && mrow0 == 0) {
         // db_i = (1/N) sum over row blocks of the bias-grad partials (fixed order)
         if (T.layer < cl.L) wait_ge(ctr + cl.dz_total + (T.layer - 1), cl.MT * p.layers[T.layer].dx_nt);
         __nv_bfloat16 *db = reinterpret_cast<__nv_bfloat16 *>(Ld.db_out);
@@ -412,58 +571,84 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
         }
       }
-      // ---- publish completion (release): the tile's global stores happen-before the counter
+      // ---- publish completion of this CTA's rows (release)
+      if (tr2) etrace2(t, 4);
       ebar();
-      if (et == 0) {
+      if (tr2) etrace2(t, 5);
+      if (et == 0 && mrow0 < T.M) {
         // release reductions are cumulative: every store of the tile (all
         // epilogue warps, ordered by the barrier above) is visible before the count
         if (T.kind == EPI_FWD) {
-          red_release_add(ctr + cl.fwd_base + 1 + (T.layer - 1) * cl.MT + T.mblk, 1);
+          red_release_add(ctr + cl.fwd_base + 1 + (T.layer - 1) * cl.MT + mblk, 1);
         } else if (T.kind == EPI_DGRAD) {
           if (T.layer >= 2) {
-            red_release_add(ctr + cl.dz_rows + (T.layer - 2) * cl.MT + T.mblk, 1);
+            red_release_add(ctr + cl.dz_rows + (T.layer - 2) * cl.MT + mblk, 1);
             red_release_add(ctr + cl.dz_total + (T.layer - 2), 1);
           }
         } else {
           red_release_add(ctr + cl.dw_done + (T.layer - 1), 1);
           red_release_add(ctr + cl.bucket_done + Ld.bucket, 1);
         }
-        etrace(t, 3);
+        if (leader) etrace(t, 3);
       }
     }
   }
   fence_before();
-  __syncthreads();
+  if (CG == 2) cluster_sync(); else __syncthreads();   // no CTA leaves while its peer may still signal it
   if (warp == 1) {
     fence_after();
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS)
-                 : "memory");
+    if (CG == 2)
+      asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS)
+                   : "memory");
+    else
+      asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS)
+                   : "memory");
   }
 }
 
-int engine_smem_bytes() { return SMEM; }
+int engine_smem_bytes(int cg) { return cg == 2 ? Cfg<2>::SMEM : Cfg<1>::SMEM; }
 
 #ifdef OOO_TRACE
-cudaError_t engine_set_trace(void *p) { return cudaMemcpyToSymbol(g_etrace, &p, sizeof(p)); }
+cudaError_t engine_set_trace(void *p) {
+  // [task][8] phase stamps, followed by [task][8] epilogue clocks (same buffer, second half)
+  void *p2 = p ? static_cast<char *>(p) + (size_t)200000 * 8 * 8 : nullptr;
+  cudaError_t e = cudaMemcpyToSymbol(g_etrace, &p, sizeof(p));
+  if (e == cudaSuccess) e = cudaMemcpyToSymbol(g_etrace2, &p2, sizeof(p2));
+  return e;
+}
 #endif
 
 cudaError_t engine_init() {
-  return cudaFuncSetAttribute(engine_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+  cudaError_t e = cudaFuncSetAttribute(engine_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<1>::SMEM);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(engine_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<2>::SMEM);
+  return e;
 }
 
-cudaError_t launch_engine(const Params &p, const CUtensorMap *tmY, const CUtensorMap *tmDX, int ctas,
+cudaError_t launch_engine(int cg, const Params &p, const CUtensorMap *tmY, const CUtensorMap *tmDX, int ctas,
                           cudaStream_t stream, int priority) {
   cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = dim3(ctas, 1, 1);
   cfg.blockDim = dim3(kThreads, 1, 1);
-  cfg.dynamicSmemBytes = SMEM;
   cfg.stream = stream;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributePriority;
   attr[0].val.priority = priority;
+  if (cg == 2) {
+    cfg.gridDim = dim3((ctas / 2) * 2, 1, 1);   // whole CTA pairs
+    cfg.dynamicSmemBytes = Cfg<2>::SMEM;
+    attr[1].id = cudaLaunchAttributeClusterDimension;
+    attr[1].val.clusterDim.x = 2;
+    attr[1].val.clusterDim.y = 1;
+    attr[1].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 2;
+    return cudaLaunchKernelEx(&cfg, engine_kernel<2>, *tmY, *tmDX, p);
+  }
+  cfg.gridDim = dim3(ctas, 1, 1);
+  cfg.dynamicSmemBytes = Cfg<1>::SMEM;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  return cudaLaunchKernelEx(&cfg, engine_kernel, *tmY, *tmDX, p);
+  return cudaLaunchKernelEx(&cfg, engine_kernel<1>, *tmY, *tmDX, p);
 }
 
 }  // namespace eng

@@ -96,6 +96,7 @@ struct Plan {
   int64_t grad_elems = 0;
   // engine (bf16): map table, layer table, completion counters
   bool engine = false;
+  int cg = 2;                      // engine CTAs per tile (2 = CTA pairs, cta_group::2)
   size_t off_maps = 0, off_layers = 0, off_ctr = 0;
   ooo::eng::CounterLayout cl{};
 };
@@ -160,8 +161,8 @@ GemmPlan plan_tc_mn(int M, int N, int K, bool weight_grad) {
 int engine_bn(int N) {
   const int forced = env_int("OOO_EBN", 0);
   if (forced && N % forced == 0) return forced;
-  for (int bn : {256, 192, 128}) if (N % bn == 0) return bn;
-  return 64;
+  // CTA pairs split B in halves of >= 64 columns: bn in {128, 256}
+  return N % 256 == 0 ? 256 : 128;
 }
 
 GemmPlan plan_simt(int M, int N, int K, bool weight_grad) {
@@ -264,6 +265,7 @@ Plan make_plan(const ooo_stack_desc *d) {
   // persistent dataflow engine (bf16): map table, layer table, counters
   p.engine = p.dtype == OOO_BF16 && 2 * p.L <= ooo::eng::kMaxOps && env_int("OOO_ENGINE", 1) != 0;
   if (p.engine) {
+    p.cg = env_int("OOO_CG", 2) == 1 ? 1 : 2;
     for (int i = 1; i <= p.L; ++i) {
       LayerPlan &lp = p.layer[i - 1];
       lp.ebn_fwd = engine_bn(lp.dout);
@@ -626,6 +628,14 @@ StreamValueFn stream_value_fn(const char *name) {
 
 int map_index(int layer, int slot) { return (layer - 1) * MS_COUNT + slot; }
 
+// Row groups per row-local op for the wavefront queue: as many as the op
+// table allows (kernel-parameter size), at most MT, default cap 8.
+int engine_groups(int MT, int grouped_ops, int other_ops) {
+  int G = std::min(MT, env_int("OOO_GROUPS", 1));
+  if (grouped_ops > 0) G = std::min(G, (ooo::eng::kMaxOps - other_ops) / grouped_ops);
+  return std::max(G, 1);
+}
+
 bool comm_active(const ooo_stack *s) { return s->nccl != nullptr && s->d.comm_enabled; }
 
 ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st) {
@@ -653,33 +663,42 @@ ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st)
   P.ctr = s->ctr;
   P.layers = s->dlayers;
   P.cl = p.cl;
-  int first = 0;
+  int first = 0, nops = 0;
   double flops = 0;
-  for (int i = 1; i <= L; ++i) {
-    const LayerPlan &lp = p.layer[i - 1];
-    ooo::eng::Op &o = P.ops[i - 1];
-    o.kind = EPI_FWD;
-    o.act = (int16_t)lp.act;
-    o.bn = (int16_t)lp.ebn_fwd;
-    o.layer = (int16_t)i;
-    o.first = first;
-    o.mt = (int16_t)p.cl.MT;
-    o.nt = (int16_t)((lp.dout + lp.ebn_fwd - 1) / lp.ebn_fwd);
-    o.nkb = (int16_t)((lp.din + 63) / 64);
-    o.mapA = (int16_t)map_index(i, MS_FWD_A);
-    o.mapB = (int16_t)map_index(i, MS_FWD_B);
-    o.mapX = (int16_t)(i == L ? ooo::eng::MAP_Y : map_index(i, MS_FWD_X));
-    o.mapZ = (int16_t)(s->lr[i - 1].Z ? map_index(i, MS_FWD_Z) : ooo::eng::MAP_NONE);
-    first += o.mt * o.nt;
-    flops += 2.0 * p.M * lp.din * lp.dout;
+  // wavefront over (layer, row group): group g of layer i+1 is queued right
+  // behind group g of layer i, deeper layers first within a diagonal
+  const int PT = (p.cl.MT + p.cg - 1) / p.cg;   // 128*cg-row tiles
+  const int G = engine_groups(PT, L, 0);
+  for (int sdiag = 0; sdiag < L + G - 1; ++sdiag) {
+    for (int g = 0; g < G; ++g) {
+      const int i = sdiag - g + 1;
+      if (i < 1 || i > L) continue;
+      const LayerPlan &lp = p.layer[i - 1];
+      ooo::eng::Op &o = P.ops[nops++];
+      o.kind = EPI_FWD;
+      o.act = (int16_t)lp.act;
+      o.bn = (int16_t)lp.ebn_fwd;
+      o.layer = (int16_t)i;
+      o.first = first;
+      o.m_off = (int16_t)(p.cg * (g * PT / G));
+      o.mt = (int16_t)((g + 1) * PT / G - g * PT / G);
+      o.nt = (int16_t)((lp.dout + lp.ebn_fwd - 1) / lp.ebn_fwd);
+      o.nkb = (int16_t)((lp.din + 63) / 64);
+      o.mapA = (int16_t)map_index(i, MS_FWD_A);
+      o.mapB = (int16_t)map_index(i, MS_FWD_B);
+      o.mapX = (int16_t)(i == L ? ooo::eng::MAP_Y : map_index(i, MS_FWD_X));
+      o.mapZ = (int16_t)(s->lr[i - 1].Z ? map_index(i, MS_FWD_Z) : ooo::eng::MAP_NONE);
+      first += o.mt * o.nt;
+      if (g == 0) flops += 2.0 * p.M * lp.din * lp.dout;
+    }
   }
-  P.nops = L;
+  P.nops = nops;
   P.ntasks = first;
   CUtensorMap tmY;
   OOO_TRY(make_map(&tmY, Y, p.layer[L - 1].dout, p.M, 32, 32, 64));
   TimedRec *tr;
   OOO_TRY(begin_rec(s, s->hi, 7, 0, 0, &tr));
-  CU_TRY(ooo::eng::launch_engine(P, &tmY, &tmY, s->engine_ctas, s->hi, s->prio_hi));
+  CU_TRY(ooo::eng::launch_engine(p.cg, P, &tmY, &tmY, s->engine_ctas, s->hi, s->prio_hi));
   OOO_TRY(end_rec(tr, s->hi, s->engine_ctas, flops, 0));
   s->bwd_pending = false;
   s->have_fwd = true;
@@ -713,17 +732,24 @@ ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, void *dX
   P.cl = p.cl;
   int nops = 0, first = 0;
   double flops = 0;
-  auto add_op = [&](int op) {
+  // dO ops are row-local -> split into G row groups (wavefront order below)
+  int ndo = 0;
+  for (int op : s->D) ndo += op > 0;
+  const int PT = (p.cl.MT + p.cg - 1) / p.cg;   // 128*cg-row tiles
+  const int G = in_order ? 1 : engine_groups(PT, ndo, L);
+  auto add_op = [&](int op, int g) {
     const int i = op > 0 ? op : -op;
     const LayerPlan &lp = p.layer[i - 1];
     ooo::eng::Op &o = P.ops[nops++];
     o.layer = (int16_t)i;
     o.first = first;
+    o.m_off = 0;
     if (op > 0) {
       o.kind = EPI_DGRAD;
       o.act = (int16_t)(i >= 2 ? p.layer[i - 2].act : OOO_ACT_IDENTITY);
       o.bn = (int16_t)lp.ebn_dx;
-      o.mt = (int16_t)p.cl.MT;
+      o.m_off = (int16_t)(p.cg * (g * PT / G));
+      o.mt = (int16_t)((g + 1) * PT / G - g * PT / G);
       o.nt = (int16_t)((lp.din + lp.ebn_dx - 1) / lp.ebn_dx);
       o.nkb = (int16_t)((lp.dout + 63) / 64);
       o.mapA = (int16_t)map_index(i, MS_DX_A);
@@ -733,7 +759,7 @@ ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, void *dX
       o.kind = EPI_WGRAD;
       o.act = OOO_ACT_IDENTITY;
       o.bn = (int16_t)lp.ebn_dw;
-      o.mt = (int16_t)((lp.din + 127) / 128);
+      o.mt = (int16_t)(((lp.din + 127) / 128 + p.cg - 1) / p.cg);
       o.nt = (int16_t)((lp.dout + lp.ebn_dw - 1) / lp.ebn_dw);
       o.nkb = (int16_t)((p.M + 63) / 64);
       o.mapA = (int16_t)map_index(i, MS_DW_A);
@@ -742,21 +768,46 @@ ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, void *dX
     }
     o.mapZ = ooo::eng::MAP_NONE;
     first += o.mt * o.nt;
-    flops += 2.0 * p.M * lp.din * lp.dout;
+    if (g == 0) flops += 2.0 * p.M * lp.din * lp.dout;
   };
-  std::vector<int> pending;
-  for (int op : s->D) {
-    if (op > 0) {
-      add_op(op);
-      for (int w : pending) add_op(w);
-      pending.clear();
-    } else if (in_order) {
-      add_op(op);
-    } else {
-      pending.push_back(op);
+  if (in_order) {
+    // conventional backprop: D as is, each op whole; the kernel adds
+    // the dW_{i+1} -> dO_i dependency
+    for (int op : s->D) add_op(op, 0);
+  } else {
+    // Alg. 2 order with the dO chain as a wavefront over row groups; dW_i
+    // (i > k) is queued right behind the last group of the dO op that
+    // completes its input, the reversed first-k dW ops stay at the end (l.6)
+    std::vector<int> dos, tail;
+    std::vector<char> is_tail(L + 1, 0);
+    for (int op : s->D)
+      if (op > 0) dos.push_back(op);
+    // dW ops after the last dO op in D are the reversed first-k tail
+    int last_do = -1;
+    for (int j = 0; j < (int)s->D.size(); ++j) if (s->D[j] > 0) last_do = j;
+    for (int j = last_do + 1; j < (int)s->D.size(); ++j) {
+      tail.push_back(s->D[j]);
+      is_tail[-s->D[j]] = 1;
     }
+    const int nd = (int)dos.size();
+    std::vector<char> has_do(L + 2, 0);
+    for (int op : dos) has_do[op] = 1;
+    for (int sdiag = 0; sdiag < nd + G - 1; ++sdiag) {
+      for (int g = 0; g < G; ++g) {
+        const int jj = sdiag - g;
+        if (jj < 0 || jj >= nd) continue;
+        const int i = dos[jj];
+        add_op(+i, g);
+        if (g == G - 1) {
+          // release dW ops whose input dZ is now fully produced
+          if (!is_tail[i]) add_op(-i, 0);
+          if (i == 2 && !has_do[1] && !is_tail[1]) add_op(-1, 0);
+        }
+      }
+    }
+    if (nd == 0 && !is_tail[1]) add_op(-1, 0);   // L == 1 without input grad
+    for (int w : tail) add_op(w, 0);
   }
-  for (int w : pending) add_op(w);
   P.nops = nops;
   P.ntasks = first;
   CUtensorMap tmDX;
@@ -764,7 +815,7 @@ ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, void *dX
   else tmDX = s->lr[0].dxA;   // unused placeholder
   TimedRec *tr;
   OOO_TRY(begin_rec(s, s->hi, 8, 0, 0, &tr));
-  CU_TRY(ooo::eng::launch_engine(P, &tmDX, &tmDX, s->engine_ctas, s->hi, s->prio_hi));
+  CU_TRY(ooo::eng::launch_engine(p.cg, P, &tmDX, &tmDX, s->engine_ctas, s->hi, s->prio_hi));
   OOO_TRY(end_rec(tr, s->hi, s->engine_ctas, flops, 0));
   if (comm) {
     // S[dW] per bucket in D's dW order: the comm stream waits for the bucket's
@@ -1041,7 +1092,7 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
           (r.Xn && (st = make_map(&m[MS_FWD_X], r.Xn, lp.dout, p.M, 32, 32, 64)) != OOO_OK) ||
           (r.Z && (st = make_map(&m[MS_FWD_Z], r.Z, lp.dout, p.M, 32, 32, 64)) != OOO_OK) ||
           (st = make_map(&m[MS_DX_A], r.dZ, lp.dout, p.M, 64, 128)) != OOO_OK ||
-          (st = make_map(&m[MS_DX_B], r.W, lp.dout, lp.din, 64, lp.ebn_dx)) != OOO_OK ||
+          (st = make_map(&m[MS_DX_B], r.W, lp.dout, lp.din, 64, lp.ebn_dx / p.cg)) != OOO_OK ||
           (st = make_map(&m[MS_DZ_X], r.dZ, lp.dout, p.M, 32, 32, 64)) != OOO_OK ||
           (st = make_map(&m[MS_DW_A], r.X, lp.din, p.M, 64, 64)) != OOO_OK ||
           (st = make_map(&m[MS_DW_B], r.dZ, lp.dout, p.M, 64, 64)) != OOO_OK ||

@@ -25,15 +25,15 @@ from paper_conf_eurosys_ohlks22_b200.stack import OooStack, schedule_order  # no
 
 
 def ebn(n):
-    for b in (256, 192, 128):
-        if n % b == 0:
-            return b
-    return 64
+    f = int(os.environ.get("OOO_EBN", "0"))
+    if f and n % f == 0:
+        return f
+    return 256 if n % 256 == 0 else 128
 
 
 def queue(cfg, D, in_order):
     """(kind, layer, ntiles) in engine queue order (mirrors engine_backward)."""
-    MT = (cfg.tokens + 127) // 128
+    MT = ((cfg.tokens + 127) // 128 + 1) // 2      # 256-row pair tiles
     ops, pending = [], []
 
     def add(op):
@@ -42,7 +42,7 @@ def queue(cfg, D, in_order):
         if op > 0:
             ops.append(("dX", i, MT * ((din + ebn(din) - 1) // ebn(din))))
         else:
-            ops.append(("dW", i, ((din + 127) // 128) * ((dout + ebn(dout) - 1) // ebn(dout))))
+            ops.append(("dW", i, (((din + 127) // 128 + 1) // 2) * ((dout + ebn(dout) - 1) // ebn(dout))))
     for op in D:
         if op > 0:
             add(op)
@@ -60,13 +60,22 @@ def queue(cfg, D, in_order):
 
 def report(name, ops, buf):
     import numpy as np
-    raw = buf.cpu().numpy().view(np.uint64).reshape(-1, 4)
+    allb = buf.cpu().numpy().view(np.uint64)
+    raw8 = allb[: 200000 * 8].reshape(-1, 8)
+    epi = allb[200000 * 8:].reshape(-1, 8).astype(np.float64)   # epilogue phase clocks
+    raw = raw8[:, :4]
+    clk = raw8[:, 4:].astype(np.float64)
     cta = (raw >> np.uint64(48)).astype(np.int64)
     t = (raw & np.uint64((1 << 48) - 1)).astype(np.float64)
     valid = t[:, 3] > 0
     t0 = t[valid, 0].min()
     t = (t - t0) / 1e3
-    print(f"== {name}: {int(valid.sum())} tasks, span {t[valid, 3].max():.1f} us")
+    # SM clock: cycles between "ready" and "acc ready" over the same interval in ns
+    dc = clk[valid, 2] - clk[valid, 1]
+    dt = (t[valid, 2] - t[valid, 1])
+    ok = dt > 1.0
+    mhz = np.median(dc[ok] / (dt[ok] * 1e3) * 1e3) if ok.any() else float("nan")
+    print(f"== {name}: {int(valid.sum())} tasks, span {t[valid, 3].max():.1f} us, SM clock ~{mhz:.0f} MHz")
     first = 0
     for kind, layer, n in ops:
         s = slice(first, first + n)
@@ -76,6 +85,11 @@ def report(name, ops, buf):
               f"..{tt[:,1].max():8.1f} done {tt[:,3].min():8.1f}..{tt[:,3].max():8.1f}"
               f" wait {np.mean(tt[:,1]-tt[:,0]):6.1f} main {np.mean(tt[:,2]-tt[:,1]):6.1f}"
               f" epi {np.mean(tt[:,3]-tt[:,2]):5.1f} ctas {len(set(cta[s, 3]))}")
+        e = epi[s]
+        if e[:, 5].max() > 0:
+            d = lambda a, b: np.median(e[:, b] - e[:, a])  # noqa: E731
+            print(f"     epi cycles: tmem_ld {d(0, 1):6.0f} chunk0 {d(1, 2):6.0f} loop {d(0, 3):6.0f}"
+                  f" tail {d(3, 4):6.0f} bar {d(4, 5):6.0f}")
 
 
 def main():
@@ -85,6 +99,7 @@ def main():
     lib.ooo_debug_set_trace.restype = ctypes.c_int32
     lib.ooo_debug_set_trace.argtypes = [ctypes.c_void_p]
     dev = torch.device("cuda")
+    os.environ["OOO_GROUPS"] = "1"     # the report assumes layer-major queues
     W, b = synth.weights_torch(cfg.dims, cfg.acts, cfg.dtype, dev)
     stk = OooStack(cfg.dims, cfg.acts, cfg.tokens, W, b, dtype=cfg.dtype)
     X = synth.activations_torch(cfg.tokens, cfg.dims[0], cfg.dtype, dev, 1, 0, 0)
@@ -94,7 +109,7 @@ def main():
         stk.backward(dY, "first_k", k)
         stk.forward(X, Y)
     torch.cuda.synchronize()
-    buf = torch.zeros(200000 * 4, dtype=torch.int64, device=dev)
+    buf = torch.zeros(2 * 200000 * 8, dtype=torch.int64, device=dev)
     _lib.check(lib.ooo_debug_set_trace(buf.data_ptr()))
     stk.backward(dY, "first_k", k)
     torch.cuda.synchronize()
@@ -103,7 +118,7 @@ def main():
     buf.zero_()
     stk.forward(X, Y)
     torch.cuda.synchronize()
-    MT = (cfg.tokens + 127) // 128
+    MT = ((cfg.tokens + 127) // 128 + 1) // 2
     fops = [("F", i, MT * ((cfg.dims[i] + ebn(cfg.dims[i]) - 1) // ebn(cfg.dims[i]))) for i in range(1, cfg.L + 1)]
     report("forward", fops, buf)
     _lib.check(lib.ooo_debug_set_trace(None))
