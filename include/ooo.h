@@ -42,10 +42,12 @@
  * Stream semantics: every call is stream-ordered after prior work on the
  * caller's stream `st`.  ooo_backward returns with work still in flight on
  * the library's internal streams (hi priority: dO ops; lo priority: dW ops;
- * comm: all-reduces).  The next ooo_forward joins it per layer (F_i waits for
- * layer i's synchronised gradient) and finally joins everything into
- * `st`; ooo_join joins it explicitly.  Gradients in `grads` are valid only
- * after one of those.  No call synchronises the host or allocates, so the
+ * comm: all-reduces) -- or, on the bf16 engine path, with its kernel
+ * deferred: the next ooo_forward then runs backward(t) and forward(t+1) as
+ * ONE persistent kernel whose F_i tiles start as soon as S[dW_i] and
+ * dW_{i+1} are done (Fig. 4(c)).  ooo_forward finally joins everything into
+ * `st`; ooo_join runs/joins an outstanding backward explicitly.  Gradients in
+ * `grads` and dX are valid only after one of those.  No call synchronises the host or allocates, so the
  * sequence ooo_backward; ooo_forward is CUDA-graph capturable on `st`.
  *
  * Errors: argument/shape errors are detected before anything is enqueued;
@@ -161,6 +163,18 @@ int32_t ooo_max_k(int32_t L, int64_t m_fwd, const int64_t *m_dO, const int64_t *
  * deferral, §3; E8 at P:352-354): sum_{i=2..k} |dZ_i|. */
 int64_t ooo_deferral_bytes(const ooo_stack_desc *d, int32_t k);
 
+/* Host only (no GPU): the tile queue the bf16 engine dispenses for one step,
+ * as planned from the two priority chains (critical: dO ops in D's order,
+ * then -- if `fused` -- the X -> X_1 copy and F_1..F_L of the next forward;
+ * deferred: dW ops in D's order; §4.1, Alg. 2) for
+ * `workers` concurrently resident tiles (<= 0: 148 / CTAs per tile).
+ * Writes up to `cap` ops as 5 int32 each: kind (0 F, 1 dO, 2 dW, 3 copy),
+ * layer i, first tile row, tile rows, column tiles; *n receives the count.
+ * *topological = 1 iff every op follows all ops it depends on (the engine's
+ * deadlock-freedom condition).  OOO_ERR_UNSUPPORTED for fp32 stacks. */
+ooo_status ooo_engine_plan(const ooo_stack_desc *d, ooo_schedule sch, int32_t fused, int32_t workers,
+                           int32_t *out, int32_t cap, int32_t *n, int32_t *topological);
+
 /* NCCL bootstrap id (rank 0 calls, caller broadcasts).  Needs libnccl.so.2. */
 ooo_status ooo_get_unique_id(void *out /* OOO_UNIQUE_ID_BYTES */);
 
@@ -207,7 +221,8 @@ ooo_status ooo_tensor(ooo_stack *s, int32_t kind, int32_t layer, void **ptr, int
  * replay of a timed region), ooo_timing_read fills up to `cap` records
  * describing the most recent execution of each bracketed launch. */
 typedef struct {
-  int32_t kind;       /* 0 fwd GEMM, 1 dX GEMM, 2 dW GEMM, 3 seed act-grad, 4 pack, 5 all-reduce, 6 copy */
+  int32_t kind;       /* 0 fwd GEMM, 1 dX GEMM, 2 dW GEMM, 3 seed act-grad, 4 pack, 5 all-reduce, 6 copy,
+                         7 engine forward, 8 engine backward, 9 engine step (backward + next forward) */
   int32_t layer;
   int32_t stream;     /* 0 hi, 1 lo, 2 comm */
   int32_t grid;       /* CTAs launched */

@@ -62,13 +62,14 @@ class LaunchRecord(ctypes.Structure):
 
 
 KIND_NAMES = {0: "fwd_gemm", 1: "dx_gemm", 2: "dw_gemm", 3: "seed", 4: "pack", 5: "allreduce", 6: "copy",
-              7: "engine_fwd", 8: "engine_bwd"}
+              7: "engine_fwd", 8: "engine_bwd", 9: "engine_step"}
 
 EXPORTS = [
     "ooo_abi_version", "ooo_last_error", "ooo_status_string", "ooo_query_sizes", "ooo_grad_offsets",
     "ooo_schedule_order", "ooo_max_k", "ooo_deferral_bytes", "ooo_get_unique_id", "ooo_create_stack",
     "ooo_forward", "ooo_backward", "ooo_join", "ooo_graph_create", "ooo_graph_launch",
     "ooo_graph_destroy", "ooo_destroy", "ooo_tensor", "ooo_set_timing", "ooo_timing_read",
+    "ooo_engine_plan",
 ]
 
 _lib = None
@@ -104,6 +105,9 @@ def load() -> ctypes.CDLL:
     lib.ooo_max_k.argtypes = [c_int32, c_int64, POINTER(c_int64), POINTER(c_int64), c_int64]
     lib.ooo_deferral_bytes.restype = c_int64
     lib.ooo_deferral_bytes.argtypes = [POINTER(StackDesc), c_int32]
+    lib.ooo_engine_plan.restype = S
+    lib.ooo_engine_plan.argtypes = [POINTER(StackDesc), Schedule, c_int32, c_int32, POINTER(c_int32), c_int32,
+                                    POINTER(c_int32), POINTER(c_int32)]
     lib.ooo_get_unique_id.restype = S
     lib.ooo_get_unique_id.argtypes = [c_void_p]
     lib.ooo_create_stack.restype = S

@@ -11,19 +11,22 @@
 //
 // Roles per CTA (one CTA per SM, persistent):
 //   warp 0 lane 0 : producer.  The leader also dispenses: atomicAdd on the
-//                   pass dispenser gives the next task (queue = priority
+//                   launch's dispenser gives the next task (queue = priority
 //                   order), written to the 4-deep smem task ring(s).
+//                   X -> X_1 copy tasks (EPI_COPY) have no loads and no MMA:
+//                   only the epilogue warps run them.
 //                   Each producer waits until its input rows are complete
 //                   (acquire on a completion counter, timeout -> trap), then
 //                   issues its TMA loads, completing on the leader's barrier.
 //   warp 1        : TMEM allocator; the leader's lane 0 issues the MMAs into
-//                   accumulator j & 1 (double-buffered).
+//                   accumulator j & 1 of its j-th GEMM task (double-buffered).
 //   warps 2..9    : epilogue of task j while task j+1's MMAs run: tcgen05.ld,
 //                   fused bias/act (F_i), act-grad + bias-grad partials (dO_i),
 //                   1/N scale + bias-grad reduction (dW_i), bf16 RNE, coalesced
 //                   stores; then publish completion (release) to the counters.
 // Deadlock freedom: tasks are dispensed in increasing index and every
-// dependency of task t is a task with a smaller index, all CTAs are
+// dependency of task t is a task with a smaller index (or, for F_i at N > 1,
+// the comm stream's all-reduce of a bucket whose dW tasks all precede t), all CTAs are
 // co-resident (grid <= #SMs, 1 CTA/SM), and each role processes its tasks in
 // order; so the smallest unfinished task can always make progress.  Every
 // wait is bounded (globaltimer) and traps instead of hanging.
@@ -223,9 +226,49 @@ __device__ __forceinline__ TaskRt task_rt(const Params &p, int t) {
   r.n0 = (rel % o.nt) * o.bn;
   const LayerDev &L = p.layers[o.layer - 1];
   if (o.kind == EPI_FWD) { r.M = p.M; r.N = L.dout; }
-  else if (o.kind == EPI_DGRAD) { r.M = p.M; r.N = L.din; }
+  else if (o.kind == EPI_DGRAD || o.kind == EPI_COPY) { r.M = p.M; r.N = L.din; }
   else { r.M = L.din; r.N = L.dout; }
   return r;
+}
+
+// Dependencies of task T for row block mblk: all on tasks earlier in the
+// queue (the host planner emits ops in a topological order), or on the comm
+// stream's all-reduce of a bucket whose dW tasks all precede T.  kWait: block
+// until met (bounded); else: report whether met now.
+template <bool kWait>
+__device__ __forceinline__ bool dep_ge(const int32_t *c, int target) {
+  if (kWait) { wait_ge(c, target); return true; }
+  return ld_relaxed(c) >= target;
+}
+template <bool kWait>
+__device__ __forceinline__ bool deps(const Params &p, const TaskRt &T, int mblk) {
+  const CounterLayout &cl = p.cl;
+  const int32_t *ctr = p.ctr;
+  const LayerDev &Ld = p.layers[T.layer - 1];
+  bool ok = true;
+  if (T.kind == EPI_FWD) {
+    if (mblk < cl.MT) {
+      if (T.layer > 1)
+        ok = dep_ge<kWait>(ctr + cl.fwd_rows + (T.layer - 2) * cl.MT + mblk, p.layers[T.layer - 2].fwd_nt);
+      else
+        ok = dep_ge<kWait>(ctr + cl.xcopy + mblk, p.copy_nt);
+    }
+    if (ok && p.fwd_gate == 1) ok = dep_ge<kWait>(ctr + cl.dw_done + (T.layer - 1), Ld.dw_tiles);   // P:84, N = 1
+    else if (ok && p.fwd_gate == 2) ok = dep_ge<kWait>(ctr + cl.ar_done + Ld.bucket, 1);          // P:84, S[dW_i]
+    if (ok && p.fwd_gate && T.layer < cl.L)      // WAR: dW_{i+1} reads X_{i+1}
+      ok = dep_ge<kWait>(ctr + cl.dw_done + T.layer, p.layers[T.layer].dw_tiles);
+  } else if (T.kind == EPI_DGRAD) {
+    if (T.layer < cl.L) {
+      const LayerDev &Ln = p.layers[T.layer];
+      if (mblk < cl.MT) ok = dep_ge<kWait>(ctr + cl.dz_rows + (T.layer - 1) * cl.MT + mblk, Ln.dx_nt);
+      if (ok && p.in_order) ok = dep_ge<kWait>(ctr + cl.dw_done + T.layer, Ln.dw_tiles);
+    }
+  } else if (T.kind == EPI_WGRAD) {
+    if (T.layer < cl.L) ok = dep_ge<kWait>(ctr + cl.dz_total + (T.layer - 1), cl.MT * p.layers[T.layer].dx_nt);
+  } else {   // EPI_COPY: dW_1 of the pending backward still reads X_1
+    if (p.fwd_gate) ok = dep_ge<kWait>(ctr + cl.dw_done, p.layers[0].dw_tiles);
+  }
+  return ok;
 }
 
 template <int CG>
@@ -249,7 +292,6 @@ __global__ void __launch_bounds__(kThreads, 1)
   float *red = reinterpret_cast<float *>(smem + C::RED_OFF);
   int32_t *ctr = p.ctr;
   const CounterLayout &cl = p.cl;
-  int32_t *dispenser = ctr + (p.pass == 0 ? cl.fwd_base : cl.bwd_base);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -307,7 +349,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int slot = j % Q;
         int t;
         if (leader) {
-          t = atomicAdd(dispenser, 1);
+          t = atomicAdd(ctr, 1);
           if (t >= p.ntasks) t = -1;
           etrace(t, 0);
           if (j >= Q) {
@@ -327,28 +369,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         if (t < 0) break;
         const TaskRt T = task_rt<CG>(p, t);
+        if (T.kind == EPI_COPY) continue;        // epilogue warps only
         const Op &o = p.ops[T.op];
         const LayerDev &Ld = p.layers[T.layer - 1];
-        const int mblk = T.mblk0 + (int)rank;    // this CTA's row block
-        // ---- dependencies (all on tasks with smaller indices)
-        if (T.kind == EPI_FWD) {
-          if (T.layer > 1 && mblk < cl.MT) {
-            const LayerDev &Lp = p.layers[T.layer - 2];
-            wait_ge(ctr + cl.fwd_base + 1 + (T.layer - 2) * cl.MT + mblk, Lp.fwd_nt);
-          }
-          if (p.gate_ar) wait_ge(ctr + cl.ar_done + Ld.bucket, 1);
-        } else if (T.kind == EPI_DGRAD) {
-          if (T.layer < cl.L) {
-            const LayerDev &Ln = p.layers[T.layer];
-            if (mblk < cl.MT) wait_ge(ctr + cl.dz_rows + (T.layer - 1) * cl.MT + mblk, Ln.dx_nt);
-            if (p.in_order) wait_ge(ctr + cl.dw_done + T.layer, Ln.dw_tiles);
-          }
-        } else {
-          if (T.layer < cl.L) {
-            const LayerDev &Ln = p.layers[T.layer];
-            wait_ge(ctr + cl.dz_total + (T.layer - 1), cl.MT * Ln.dx_nt);
-          }
-        }
+        deps<true>(p, T, T.mblk0 + (int)rank);    // this CTA's row block (no-op after a ready claim)
         asm volatile("fence.proxy.async.global;" ::: "memory");   // TMA reads see the producers' data
         if (leader) etrace(t, 1);
         const CUtensorMap *mA = map_of(o.mapA, p.maps, &tmY, &tmDX);
@@ -400,7 +424,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   } else if (warp == 1) {
     // ============ MMA issuer (leader CTA only) ============
     if (leader && lane == 0) {
-      int it = 0;
+      int it = 0, ja = 0;   // k-block stages, accumulator uses (GEMM tasks only)
       for (int j = 0;; ++j) {
         const int slot = j % Q;
         mbar_wait_b(bar_qfull + 8 * slot, (j / Q) & 1);
@@ -408,17 +432,19 @@ __global__ void __launch_bounds__(kThreads, 1)
         mbar_arrive(bar_qempty + 8 * slot);
         if (t < 0) break;
         const TaskRt T = task_rt<CG>(p, t);
+        if (T.kind == EPI_COPY) continue;        // no accumulator
         const bool a_mn = T.kind == EPI_WGRAD;
         const bool b_mn = T.kind != EPI_DGRAD;
         // M = 128 * CG across the CTAs, N = bn
         const uint32_t ID = (1u << 4) | (1u << 7) | (1u << 10) | ((a_mn ? 1u : 0u) << 15) |
                             ((b_mn ? 1u : 0u) << 16) | ((uint32_t)(T.bn >> 3) << 17) |
                             ((uint32_t)((BM * CG) >> 4) << 24);
-        const int acc = j & 1;
-        if (j >= 2) {
-          if (CG == 2) mbar_wait_cl(bar_tempty + 8 * acc, ((j >> 1) - 1) & 1);
-          else mbar_wait_b(bar_tempty + 8 * acc, ((j >> 1) - 1) & 1);
+        const int acc = ja & 1;
+        if (ja >= 2) {
+          if (CG == 2) mbar_wait_cl(bar_tempty + 8 * acc, ((ja >> 1) - 1) & 1);
+          else mbar_wait_b(bar_tempty + 8 * acc, ((ja >> 1) - 1) & 1);
         }
+        ++ja;
         fence_after();
         const uint32_t dtm = tmem + (uint32_t)(acc * kMaxBN);
         for (int kb = 0; kb < T.nkb; ++kb, ++it) {
@@ -446,7 +472,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int h = (warp - 2) >> 2;           // column slot: 32-col chunks c = h, h + kEpiPerQ, ...
     const int et = threadIdx.x - 64;         // 0..255
     const uint32_t stg = sbase + C::STG_OFF + (warp - 2) * 2048;
-    for (int j = 0;; ++j) {
+    for (int j = 0, ja = 0;; ++j) {
       const int slot = j % Q;
       if (leader) mbar_wait_b(bar_qfull + 8 * slot, (j / Q) & 1);
       else mbar_wait_cl(bar_qfull + 8 * slot, (j / Q) & 1);
@@ -458,11 +484,33 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       if (t < 0) break;
       const TaskRt T = task_rt<CG>(p, t);
-      const Op &o = p.ops[T.op];
-      const LayerDev &Ld = p.layers[T.layer - 1];
-      const int acc = j & 1;
       const int mblk = T.mblk0 + (int)rank;
       const int mrow0 = T.m0 + BM * (int)rank;  // this CTA's first row
+      if (T.kind == EPI_COPY) {
+        // caller's X rows [mrow0, +128) x [n0, +bn) -> X_1 store (dW_1 of the
+        // pending backward reads X_1: WAR wait first)
+        if (mrow0 < T.M) {
+          if (p.fwd_gate && et == 0) wait_ge(ctr + cl.dw_done, p.layers[0].dw_tiles);
+          ebar();
+          const int rows = min(BM, T.M - mrow0);
+          const int vpr = min(T.bn, T.N - T.n0) / 8;     // 16-byte vectors per row
+          const uint4 *src = reinterpret_cast<const uint4 *>(p.x_in);
+          uint4 *dst = reinterpret_cast<uint4 *>(p.layers[0].X);
+          const size_t ld = (size_t)T.N / 8;
+          for (int v = et; v < rows * vpr; v += kEpiThreads) {
+            const size_t e = (size_t)(mrow0 + v / vpr) * ld + T.n0 / 8 + v % vpr;
+            dst[e] = __ldg(src + e);
+          }
+          ebar();
+          if (et == 0) red_release_add(ctr + cl.xcopy + mblk, 1);
+        }
+        if (et == 0 && leader) { etrace(t, 1); etrace(t, 2); etrace(t, 3); }
+        continue;
+      }
+      const Op &o = p.ops[T.op];
+      const LayerDev &Ld = p.layers[T.layer - 1];
+      const int acc = ja & 1;
+      const int jacc = ja++;
       const int row0 = mrow0 + q * 32;
       const int row = row0 + lane;
       const bool row_ok = row < T.M;
@@ -500,7 +548,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const __nv_bfloat16 *zrow = zin ? zin + (size_t)row * T.N + T.n0 : nullptr;
       uint4 zr[4];
       if (need_z && h < nch) ld_raw32(zrow + h * 32, zr);     // act' input, prefetched before the wait
-      mbar_wait_b(bar_tfull + 8 * acc, (j >> 1) & 1);
+      mbar_wait_b(bar_tfull + 8 * acc, (jacc >> 1) & 1);
       fence_after();
       if (et == 0 && leader) etrace(t, 2);
       const bool tr2 = et == 0 && leader;
@@ -579,7 +627,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         // release reductions are cumulative: every store of the tile (all
         // epilogue warps, ordered by the barrier above) is visible before the count
         if (T.kind == EPI_FWD) {
-          red_release_add(ctr + cl.fwd_base + 1 + (T.layer - 1) * cl.MT + mblk, 1);
+          red_release_add(ctr + cl.fwd_rows + (T.layer - 1) * cl.MT + mblk, 1);
         } else if (T.kind == EPI_DGRAD) {
           if (T.layer >= 2) {
             red_release_add(ctr + cl.dz_rows + (T.layer - 2) * cl.MT + mblk, 1);

@@ -1,20 +1,23 @@
-// Persistent dataflow engine: one kernel per pass (forward / backward) that
-// runs the whole pass as a priority-ordered queue of 128 x BN output tiles.
+// Persistent dataflow engine: one kernel per training step (backward(t) fused
+// with forward(t+1)) that runs the whole step as a priority-ordered queue of
+// output tiles.
 //
 // Why (paper §2, §4.1, §5.1): the paper schedules
 // dO_i / dW_i ops of a layer stack so that the critical chain (dO, then the
 // next forward) is never delayed and the deferrable dW ops fill idle
-// resources, in Algorithm 2's order.  On B200 a BERT-sized layer GEMM is only
-// 3-20 us of tensor work, so per-kernel launch, first-load latency, exposed
-// epilogue and wave tails cost as much as the math.  The engine removes those
+// resources, in Algorithm 2's order; the next forward F_i may start as soon
+// as S[dW_i] is done.  On B200 a BERT-sized layer GEMM is only 3-20 us
+// of tensor work, so per-kernel launch, first-load latency, exposed epilogue
+// and wave tails cost as much as the math.  The engine removes those
 // boundaries: CTAs take tiles in queue order (the schedule D expanded to
-// tiles), a tile starts as soon as the row block it reads is complete
-// (dO_i and F_i are row-local: output row block m needs only input row
-// block m), and dW_i tiles are slotted into the queue behind the critical
-// dO tiles (reverse first-k keeps dW_1..dW_k at the end).  Completion
-// counters in global memory replace stream events; they also drive the
-// per-bucket all-reduce (the comm stream waits on them with
-// cuStreamWaitValue32) and gate the next forward (F_i waits for its bucket).
+// tiles, then the next forward), a tile starts as soon as the rows it reads
+// are complete (dO_i and F_i are row-local: output row block m needs only
+// input row block m), dW_i tiles are slotted into the queue behind the
+// critical dO tiles (reverse first-k keeps dW_1..dW_k at the end), and F_i
+// starts as soon as dW_i is done -- the Fig. 4(c) overlap, inside one kernel.
+// Completion counters in global memory replace stream events; they also
+// drive the per-bucket all-reduce (the comm stream waits on them with
+// cuStreamWaitValue32) and gate F_i on its bucket's all-reduce for N > 1.
 #pragma once
 #include <cuda.h>
 #include <cuda_runtime.h>
@@ -23,22 +26,25 @@
 namespace ooo {
 namespace eng {
 
-constexpr int kMaxOps = 512;
+constexpr int kMaxOps = 768;     // op table travels as a kernel parameter (<= 32 KiB)
 constexpr int MAP_NONE = -1;
 constexpr int MAP_Y = -2;    // kernel-parameter map of the caller's Y
 constexpr int MAP_DX = -3;   // kernel-parameter map of the caller's dX
+constexpr int EPI_COPY = 3;  // task kind: copy the caller's X rows into the X_1 store (no MMA)
 
-// One op of the pass = one layer GEMM (F_i, dO_i or dW_i) = mt x nt tiles.
+// One op of the queue = one row group of a layer GEMM (F_i, dO_i or dW_i), or
+// the X -> X_1 copy = mt x nt tiles starting at row block m_off.
 struct Op {
-  int16_t kind;     // EPI_FWD / EPI_DGRAD / EPI_WGRAD
+  int16_t kind;     // EPI_FWD / EPI_DGRAD / EPI_WGRAD / EPI_COPY
   int16_t act;      // epilogue activation (act_i for F_i, act_{i-1} for dO_i)
   int16_t bn;       // tile width (64..256, % 64 == 0)
   int16_t layer;    // i (1-based)
   int32_t first;    // first task index of this op in the queue
-  int16_t mt, nt;   // tiles: rows (128) x cols (bn)
-  int16_t nkb;      // K / 64
+  int16_t mt, nt;   // tiles: rows (128 * cg) x cols (bn)
+  int16_t nkb;      // K / 64 (0 for EPI_COPY)
   int16_t mapA, mapB, mapX, mapZ;   // indices into the map table (or MAP_*)
-  int16_t pad[3];
+  int16_t m_off;    // first row block of the group
+  int16_t pad[2];
 };
 static_assert(sizeof(Op) == 32, "Op layout");
 
@@ -51,48 +57,51 @@ struct LayerDev {
   void *Xn;                // X_{i+1} store (null for i = L: the caller's Y)
   void *dZ;                // dZ_i store
   void *gw;                // bucket slot of dW_i (bf16)
-  void *pad0;
+  void *X;                 // X_i store (layer 1: the copy of the caller's X)
   int32_t din, dout, act, bucket;
   int32_t fwd_nt;          // n-tiles of F_i over d_i
   int32_t dx_nt;           // n-tiles of dO_i over d_{i-1}
-  int32_t dw_tiles;        // tiles of dW_i
+  int32_t dw_tiles;        // 128-row tiles of dW_i (completion count)
   int32_t pad1[9];
 };
 static_assert(sizeof(LayerDev) == 128, "LayerDev layout");
 
-// Counter layout (int32, in the workspace):
-//   fwd region : [0] dispenser, [1 + i*MT + m] rows of X_{i+1} done (i = 0..L-1)
-//   bwd region : [0] dispenser, dz_rows[i][m], dz_total[i], dw_done[i],
-//                bucket_done[b], ar_done[b]   (i = 1..L, index i-1)
+// Counter layout (int32, one region in the workspace; indices are absolute):
+//   [0] dispenser | [1] unused | fwd_rows[L][MT]: tiles done of row block m of X_{i+1} |
+//   xcopy[MT]: X_1 rows copied | dz_rows[L][MT] | dz_total[L] | dw_done[L] |
+//   bucket_done[nb] | ar_done[nb]
+// A forward-only launch resets [0, fwd_end); a backward resets [0, total).
 struct CounterLayout {
   int L, MT, nb;
-  int fwd_base, fwd_size;
-  int bwd_base, bwd_size;
-  int dz_rows, dz_total, dw_done, bucket_done, ar_done;   // absolute indices
+  int fwd_rows, xcopy, fwd_end;
+  int dz_rows, dz_total, dw_done, bucket_done, ar_done, total;
 };
 
 struct Params {
   int32_t nops, ntasks, M, R;
   float alpha;
   int32_t in_order;        // dO_i also waits for dW_{i+1} (conventional backprop)
-  int32_t gate_ar;         // F_i waits ar_done[bucket(i)] (N > 1)
-  int32_t pass;            // 0 forward, 1 backward
-  int32_t dbg;             // tuning experiments only (OOO_DBG): bit0 skip act math, bit1 skip stores
+  int32_t fwd_gate;        // 0: none; 1: F_i waits dW_i (N = 1); 2: F_i waits ar_done[bucket(i)]
+                           // (N > 1); both also wait dW_{i+1} (it reads X_{i+1}, which F_i overwrites)
+  int32_t dbg;             // tuning experiments only (OOO_DBG): bit0 skip act math, bit1 skip stores, bit2 skip epilogue
+  int32_t copy_nt;         // column tiles per row block of the X -> X_1 copy
   const CUtensorMap *maps;
   int32_t *ctr;            // counter array base
   const LayerDev *layers;  // index i-1
   void *y_out;             // caller's Y (F_L output)
   void *dx_out;            // caller's dX (dO_1 output, need_input_grad)
+  const void *x_in;        // caller's X (source of the X_1 copy tasks)
   CounterLayout cl;
   Op ops[kMaxOps];
 };
 
-int engine_smem_bytes();
+// cg = CTAs per tile: 1 (128-row tiles) or 2 (CTA pairs, 256-row tiles, cta_group::2)
+int engine_smem_bytes(int cg);
 cudaError_t engine_init();
 #ifdef OOO_TRACE
 cudaError_t engine_set_trace(void *p);   // debug builds: per-task timestamps buffer
 #endif
-cudaError_t launch_engine(const Params &p, const CUtensorMap *tmY, const CUtensorMap *tmDX, int ctas,
+cudaError_t launch_engine(int cg, const Params &p, const CUtensorMap *tmY, const CUtensorMap *tmDX, int ctas,
                           cudaStream_t stream, int priority);
 
 }  // namespace eng

@@ -29,6 +29,7 @@
 #include "engine.h"
 #include "kernels.h"
 #include "nccl_dyn.h"
+#include "planner.h"
 
 using namespace ooo;
 
@@ -278,16 +279,16 @@ Plan make_plan(const ooo_stack_desc *d) {
     cl.L = p.L;
     cl.MT = (p.M + 127) / 128;
     cl.nb = p.nbuckets;
-    cl.fwd_base = 0;
-    cl.fwd_size = 1 + p.L * cl.MT;
-    cl.bwd_base = align_up(cl.fwd_size, 64);
-    cl.dz_rows = cl.bwd_base + 1;
+    cl.fwd_rows = 2;
+    cl.xcopy = cl.fwd_rows + p.L * cl.MT;
+    cl.fwd_end = cl.xcopy + cl.MT;
+    cl.dz_rows = (int)align_up(cl.fwd_end, 32);
     cl.dz_total = cl.dz_rows + p.L * cl.MT;
     cl.dw_done = cl.dz_total + p.L;
     cl.bucket_done = cl.dw_done + p.L;
     cl.ar_done = cl.bucket_done + p.nbuckets;
-    cl.bwd_size = cl.ar_done + p.nbuckets - cl.bwd_base;
-    p.off_ctr = take((size_t)(cl.bwd_base + cl.bwd_size) * 4);
+    cl.total = cl.ar_done + p.nbuckets;
+    p.off_ctr = take((size_t)cl.total * 4);
   }
   p.workspace_bytes = std::max<size_t>(off, 256);
   p.grad_elems = goff;
@@ -397,6 +398,14 @@ struct ooo_stack {
   const CUtensorMap *dmaps = nullptr;         // map table (workspace)
   const ooo::eng::LayerDev *dlayers = nullptr;
   int engine_ctas = 148;
+  bool eng_pending = false;                   // ooo_backward enqueued, its kernel deferred
+  std::vector<ooo::plan::Unit> eng_crit, eng_defer;   // the deferred backward's chains
+  double eng_flops = 0;
+  void *eng_dX = nullptr;
+  bool eng_in_order = false;
+#ifdef OOO_TRACE
+  std::vector<ooo::eng::Op> last_queue;       // debug: the most recent engine launch's ops
+#endif
 };
 
 struct ooo_graph {
@@ -628,195 +637,220 @@ StreamValueFn stream_value_fn(const char *name) {
 
 int map_index(int layer, int slot) { return (layer - 1) * MS_COUNT + slot; }
 
-// Row groups per row-local op for the wavefront queue: as many as the op
-// table allows (kernel-parameter size), at most MT, default cap 8.
-int engine_groups(int MT, int grouped_ops, int other_ops) {
-  int G = std::min(MT, env_int("OOO_GROUPS", 1));
-  if (grouped_ops > 0) G = std::min(G, (ooo::eng::kMaxOps - other_ops) / grouped_ops);
-  return std::max(G, 1);
+bool comm_active(const ooo_stack *s) { return s->nccl != nullptr && s->d.comm_enabled; }
+
+namespace pl = ooo::plan;
+static_assert(pl::FWD == EPI_FWD && pl::DGRAD == EPI_DGRAD && pl::WGRAD == EPI_WGRAD &&
+                  pl::COPY == ooo::eng::EPI_COPY, "planner kinds = engine task kinds");
+
+// Planner timing model (tuning knob for experiments: OOO_PLAN_SLACK).
+pl::Model plan_model() {
+  pl::Model m;
+  if (const char *v = getenv("OOO_PLAN_SLACK")) m.slack = atof(v);
+  return m;
 }
 
-bool comm_active(const ooo_stack *s) { return s->nccl != nullptr && s->d.comm_enabled; }
+int copy_bn(int d0) { return d0 % 256 == 0 ? 256 : (d0 % 128 == 0 ? 128 : 64); }
+
+// Whole-op planner units.  Row-local ops (F_i, dO_i, copy) span the PT =
+// ceil(MT / cg) token tile rows; dW_i spans the ceil(d_{i-1} / (128 cg)) rows
+// of its weight-gradient tile grid.
+pl::Unit unit_of(const ooo_stack *s, int kind, int i) {
+  const Plan &p = s->p;
+  const int PT = (p.cl.MT + p.cg - 1) / p.cg;
+  pl::Unit u = {};
+  u.kind = kind;
+  u.layer = i;
+  u.m_off = 0;
+  if (kind == pl::COPY) {
+    u.layer = 1;
+    u.bn = copy_bn(s->dims[0]);
+    u.mt = PT;
+    u.nt = (s->dims[0] + u.bn - 1) / u.bn;
+    u.nkb = 0;
+    return u;
+  }
+  const LayerPlan &lp = p.layer[i - 1];
+  if (kind == pl::FWD) {
+    u.act = lp.act;
+    u.bn = lp.ebn_fwd;
+    u.mt = PT;
+    u.nt = (lp.dout + u.bn - 1) / u.bn;
+    u.nkb = (lp.din + 63) / 64;
+  } else if (kind == pl::DGRAD) {
+    u.act = i >= 2 ? p.layer[i - 2].act : OOO_ACT_IDENTITY;
+    u.bn = lp.ebn_dx;
+    u.mt = PT;
+    u.nt = (lp.din + u.bn - 1) / u.bn;
+    u.nkb = (lp.dout + 63) / 64;
+  } else {
+    u.act = OOO_ACT_IDENTITY;
+    u.bn = lp.ebn_dw;
+    u.mt = ((lp.din + 127) / 128 + p.cg - 1) / p.cg;
+    u.nt = (lp.dout + u.bn - 1) / u.bn;
+    u.nkb = (p.M + 63) / 64;
+  }
+  return u;
+}
+
+ooo::eng::Op op_of_unit(const ooo_stack *s, const pl::Unit &u) {
+  const Plan &p = s->p;
+  const int i = u.layer;
+  ooo::eng::Op o = {};
+  o.kind = (int16_t)u.kind;
+  o.layer = (int16_t)i;
+  o.act = (int16_t)u.act;
+  o.bn = (int16_t)u.bn;
+  o.m_off = (int16_t)(p.cg * u.m_off);   // 128-row blocks
+  o.mt = (int16_t)u.mt;
+  o.nt = (int16_t)u.nt;
+  o.nkb = (int16_t)u.nkb;
+  o.mapA = o.mapB = o.mapX = o.mapZ = ooo::eng::MAP_NONE;
+  if (u.kind == pl::FWD) {
+    o.mapA = (int16_t)map_index(i, MS_FWD_A);
+    o.mapB = (int16_t)map_index(i, MS_FWD_B);
+    o.mapX = (int16_t)(i == p.L ? ooo::eng::MAP_Y : map_index(i, MS_FWD_X));
+    o.mapZ = (int16_t)(s->lr[i - 1].Z ? map_index(i, MS_FWD_Z) : ooo::eng::MAP_NONE);
+  } else if (u.kind == pl::DGRAD) {
+    o.mapA = (int16_t)map_index(i, MS_DX_A);
+    o.mapB = (int16_t)map_index(i, MS_DX_B);
+    o.mapX = (int16_t)(i >= 2 ? map_index(i - 1, MS_DZ_X) : ooo::eng::MAP_DX);
+  } else if (u.kind == pl::WGRAD) {
+    o.mapA = (int16_t)map_index(i, MS_DW_A);
+    o.mapB = (int16_t)map_index(i, MS_DW_B);
+    o.mapX = (int16_t)map_index(i, MS_GW_X);
+  }
+  return o;
+}
+
+// Backward chains.  ooo schedules: critical = the dO chain in D's order,
+// deferred = the dW ops in D's order (Alg. 2: dW_L..dW_{k+1}, then the
+// reversed first-k dW_1..dW_k); the planner interleaves them (two priority
+// streams).  in_order (conventional backprop): one chain =
+// D, and the kernel adds the dW_{i+1} -> dO_i dependency.
+void engine_bwd_units(const ooo_stack *s, bool in_order, std::vector<pl::Unit> &crit,
+                      std::vector<pl::Unit> &defer, double &flops) {
+  const Plan &p = s->p;
+  for (int op : s->D) {
+    const int i = op > 0 ? op : -op;
+    const pl::Unit u = unit_of(s, op > 0 ? pl::DGRAD : pl::WGRAD, i);
+    (op < 0 && !in_order ? defer : crit).push_back(u);
+    flops += 2.0 * p.M * p.layer[i - 1].din * p.layer[i - 1].dout;
+  }
+}
+
+// Plans the FIFO order (planner.h) and launches the engine on it.
+ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const std::vector<pl::Unit> &defer,
+                         void *Y, void *dX, const void *X, bool in_order, int fwd_gate, int rec_kind, double flops) {
+  const Plan &p = s->p;
+  pl::Problem pb;
+  pb.L = p.L;
+  pb.rows = (p.cl.MT + p.cg - 1) / p.cg;
+  pb.workers = std::max(1, s->engine_ctas / p.cg);
+  pb.in_order = in_order;
+  pb.fwd_gate = fwd_gate;
+  pb.bucket.resize(p.L);
+  for (int i = 1; i <= p.L; ++i) pb.bucket[i - 1] = p.layer[i - 1].bucket;
+  pb.crit = crit;
+  pb.defer = defer;
+  const std::vector<pl::Unit> order = pl::schedule(pb, plan_model(), ooo::eng::kMaxOps);
+  if (order.empty()) return fail(OOO_ERR_UNSUPPORTED, "engine queue does not fit the op table (%d ops)", ooo::eng::kMaxOps);
+  ooo::eng::Params P = {};
+  P.M = p.M;
+  P.R = p.R;
+  P.alpha = 1.0f / (float)s->d.world_size;
+  P.in_order = in_order ? 1 : 0;
+  P.fwd_gate = fwd_gate;
+  P.dbg = env_int("OOO_DBG", 0);
+  P.copy_nt = (s->dims[0] + copy_bn(s->dims[0]) - 1) / copy_bn(s->dims[0]);
+  P.maps = s->dmaps;
+  P.ctr = s->ctr;
+  P.layers = s->dlayers;
+  P.y_out = Y;
+  P.dx_out = dX;
+  P.x_in = X;
+  P.cl = p.cl;
+  int first = 0;
+  for (size_t j = 0; j < order.size(); ++j) {
+    P.ops[j] = op_of_unit(s, order[j]);
+    P.ops[j].first = first;
+    first += order[j].mt * order[j].nt;
+  }
+  P.nops = (int)order.size();
+  P.ntasks = first;
+#ifdef OOO_TRACE
+  s->last_queue.assign(P.ops, P.ops + P.nops);
+#endif
+  CUtensorMap tmY, tmDX;
+  if (Y) OOO_TRY(make_map(&tmY, Y, p.layer[p.L - 1].dout, p.M, 32, 32, 64));
+  else tmY = s->lr[0].dxA;    // unused placeholder
+  if (dX) OOO_TRY(make_map(&tmDX, dX, s->dims[0], p.M, 32, 32, 64));
+  else tmDX = s->lr[0].dxA;
+  TimedRec *tr;
+  OOO_TRY(begin_rec(s, s->hi, rec_kind, 0, 0, &tr));
+  CU_TRY(ooo::eng::launch_engine(p.cg, P, &tmY, &tmDX, s->engine_ctas, s->hi, s->prio_hi));
+  return end_rec(tr, s->hi, s->engine_ctas, flops, 0);
+}
+
+// A backward whose kernel is still deferred (engine): run it alone.
+ooo_status engine_flush(ooo_stack *s) {
+  if (!s->eng_pending) return OOO_OK;
+  s->eng_pending = false;
+  return engine_launch(s, s->eng_crit, s->eng_defer, nullptr, s->eng_dX, nullptr, s->eng_in_order, 0, 8,
+                       s->eng_flops);
+}
 
 ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st) {
   const Plan &p = s->p;
   const int L = p.L;
   OOO_TRY(fork_from(s, st));
-  const bool gate = s->bwd_pending && comm_active(s);
-  CU_TRY(cudaMemsetAsync(s->ctr + p.cl.fwd_base, 0, (size_t)p.cl.fwd_size * 4, s->hi));
-  {
-    TimedRec *tr;
-    OOO_TRY(begin_rec(s, s->hi, 6, 1, 0, &tr));
-    const size_t bytes = (size_t)p.M * s->dims[0] * p.elt;
-    CU_TRY(cudaMemcpyAsync(s->lr[0].X, X, bytes, cudaMemcpyDeviceToDevice, s->hi));
-    OOO_TRY(end_rec(tr, s->hi, 0, 0, 2.0 * bytes));
-  }
-  ooo::eng::Params P = {};
-  P.M = p.M;
-  P.R = p.R;
-  P.alpha = 1.0f / (float)s->d.world_size;
-  P.gate_ar = gate ? 1 : 0;
-  P.pass = 0;
-  P.dbg = env_int("OOO_DBG", 0);
-  P.y_out = Y;
-  P.maps = s->dmaps;
-  P.ctr = s->ctr;
-  P.layers = s->dlayers;
-  P.cl = p.cl;
-  int first = 0, nops = 0;
   double flops = 0;
-  // wavefront over (layer, row group): group g of layer i+1 is queued right
-  // behind group g of layer i, deeper layers first within a diagonal
-  const int PT = (p.cl.MT + p.cg - 1) / p.cg;   // 128*cg-row tiles
-  const int G = engine_groups(PT, L, 0);
-  for (int sdiag = 0; sdiag < L + G - 1; ++sdiag) {
-    for (int g = 0; g < G; ++g) {
-      const int i = sdiag - g + 1;
-      if (i < 1 || i > L) continue;
-      const LayerPlan &lp = p.layer[i - 1];
-      ooo::eng::Op &o = P.ops[nops++];
-      o.kind = EPI_FWD;
-      o.act = (int16_t)lp.act;
-      o.bn = (int16_t)lp.ebn_fwd;
-      o.layer = (int16_t)i;
-      o.first = first;
-      o.m_off = (int16_t)(p.cg * (g * PT / G));
-      o.mt = (int16_t)((g + 1) * PT / G - g * PT / G);
-      o.nt = (int16_t)((lp.dout + lp.ebn_fwd - 1) / lp.ebn_fwd);
-      o.nkb = (int16_t)((lp.din + 63) / 64);
-      o.mapA = (int16_t)map_index(i, MS_FWD_A);
-      o.mapB = (int16_t)map_index(i, MS_FWD_B);
-      o.mapX = (int16_t)(i == L ? ooo::eng::MAP_Y : map_index(i, MS_FWD_X));
-      o.mapZ = (int16_t)(s->lr[i - 1].Z ? map_index(i, MS_FWD_Z) : ooo::eng::MAP_NONE);
-      first += o.mt * o.nt;
-      if (g == 0) flops += 2.0 * p.M * lp.din * lp.dout;
-    }
+  for (int i = 1; i <= L; ++i) flops += 2.0 * p.M * p.layer[i - 1].din * p.layer[i - 1].dout;
+  // the next forward: copy X -> X_1, then F_1..F_L (critical chain)
+  std::vector<pl::Unit> fwd;
+  fwd.push_back(unit_of(s, pl::COPY, 1));
+  for (int i = 1; i <= L; ++i) fwd.push_back(unit_of(s, pl::FWD, i));
+  if (s->eng_pending && env_int("OOO_FUSE", 1) == 0) OOO_TRY(engine_flush(s));   // experiments: unfused
+  if (s->eng_pending) {
+    // backward(t) + forward(t+1) in one launch (Fig. 4(c)); counters were
+    // reset by ooo_backward.  F_i is gated on dW_i (N = 1) or on its bucket's
+    // all-reduce (N > 1) and on dW_{i+1} (it reads X_{i+1}).
+    s->eng_pending = false;
+    const bool ar = comm_active(s);
+    std::vector<pl::Unit> crit = s->eng_crit;
+    crit.insert(crit.end(), fwd.begin(), fwd.end());
+    OOO_TRY(engine_launch(s, crit, s->eng_defer, Y, s->eng_dX, X, s->eng_in_order, ar ? 2 : 1, 9,
+                          s->eng_flops + flops));
+  } else {
+    CU_TRY(cudaMemsetAsync(s->ctr, 0, (size_t)p.cl.fwd_end * 4, s->hi));
+    OOO_TRY(engine_launch(s, fwd, {}, Y, nullptr, X, false, 0, 7, flops));
   }
-  P.nops = nops;
-  P.ntasks = first;
-  CUtensorMap tmY;
-  OOO_TRY(make_map(&tmY, Y, p.layer[L - 1].dout, p.M, 32, 32, 64));
-  TimedRec *tr;
-  OOO_TRY(begin_rec(s, s->hi, 7, 0, 0, &tr));
-  CU_TRY(ooo::eng::launch_engine(p.cg, P, &tmY, &tmY, s->engine_ctas, s->hi, s->prio_hi));
-  OOO_TRY(end_rec(tr, s->hi, s->engine_ctas, flops, 0));
   s->bwd_pending = false;
   s->have_fwd = true;
   return join_into(s, st);
 }
 
+// Enqueues the counter reset, the seed and the comm stream's all-reduces; the
+// engine kernel itself is deferred to the next ooo_forward (fused step) or
+// ooo_join (backward alone).
 ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, void *dX, cudaStream_t st) {
   const Plan &p = s->p;
   const int L = p.L;
   OOO_TRY(fork_from(s, st));
-  CU_TRY(cudaMemsetAsync(s->ctr + p.cl.bwd_base, 0, (size_t)p.cl.bwd_size * 4, s->hi));
+  CU_TRY(cudaMemsetAsync(s->ctr, 0, (size_t)p.cl.total * 4, s->hi));
   const bool comm = comm_active(s);
   if (comm) {   // the comm stream's value-waits must observe the reset counters
     CU_TRY(cudaEventRecord(s->ev_j_hi, s->hi));
     CU_TRY(cudaStreamWaitEvent(s->comm, s->ev_j_hi, 0));
   }
   OOO_TRY(launch_seed_op(s, dY, s->hi, s->prio_hi));
-  // queue = D expanded to tiles; dW ops slotted right behind the next dO op so
-  // the critical chain is dispensed first (two-stream priority)
-  ooo::eng::Params P = {};
-  P.M = p.M;
-  P.R = p.R;
-  P.alpha = 1.0f / (float)s->d.world_size;
-  P.in_order = in_order ? 1 : 0;
-  P.pass = 1;
-  P.dbg = env_int("OOO_DBG", 0);
-  P.dx_out = dX;
-  P.maps = s->dmaps;
-  P.ctr = s->ctr;
-  P.layers = s->dlayers;
-  P.cl = p.cl;
-  int nops = 0, first = 0;
-  double flops = 0;
-  // dO ops are row-local -> split into G row groups (wavefront order below)
-  int ndo = 0;
-  for (int op : s->D) ndo += op > 0;
-  const int PT = (p.cl.MT + p.cg - 1) / p.cg;   // 128*cg-row tiles
-  const int G = in_order ? 1 : engine_groups(PT, ndo, L);
-  auto add_op = [&](int op, int g) {
-    const int i = op > 0 ? op : -op;
-    const LayerPlan &lp = p.layer[i - 1];
-    ooo::eng::Op &o = P.ops[nops++];
-    o.layer = (int16_t)i;
-    o.first = first;
-    o.m_off = 0;
-    if (op > 0) {
-      o.kind = EPI_DGRAD;
-      o.act = (int16_t)(i >= 2 ? p.layer[i - 2].act : OOO_ACT_IDENTITY);
-      o.bn = (int16_t)lp.ebn_dx;
-      o.m_off = (int16_t)(p.cg * (g * PT / G));
-      o.mt = (int16_t)((g + 1) * PT / G - g * PT / G);
-      o.nt = (int16_t)((lp.din + lp.ebn_dx - 1) / lp.ebn_dx);
-      o.nkb = (int16_t)((lp.dout + 63) / 64);
-      o.mapA = (int16_t)map_index(i, MS_DX_A);
-      o.mapB = (int16_t)map_index(i, MS_DX_B);
-      o.mapX = (int16_t)(i >= 2 ? map_index(i - 1, MS_DZ_X) : ooo::eng::MAP_DX);
-    } else {
-      o.kind = EPI_WGRAD;
-      o.act = OOO_ACT_IDENTITY;
-      o.bn = (int16_t)lp.ebn_dw;
-      o.mt = (int16_t)(((lp.din + 127) / 128 + p.cg - 1) / p.cg);
-      o.nt = (int16_t)((lp.dout + lp.ebn_dw - 1) / lp.ebn_dw);
-      o.nkb = (int16_t)((p.M + 63) / 64);
-      o.mapA = (int16_t)map_index(i, MS_DW_A);
-      o.mapB = (int16_t)map_index(i, MS_DW_B);
-      o.mapX = (int16_t)map_index(i, MS_GW_X);
-    }
-    o.mapZ = ooo::eng::MAP_NONE;
-    first += o.mt * o.nt;
-    if (g == 0) flops += 2.0 * p.M * lp.din * lp.dout;
-  };
-  if (in_order) {
-    // conventional backprop: D as is, each op whole; the kernel adds
-    // the dW_{i+1} -> dO_i dependency
-    for (int op : s->D) add_op(op, 0);
-  } else {
-    // Alg. 2 order with the dO chain as a wavefront over row groups; dW_i
-    // (i > k) is queued right behind the last group of the dO op that
-    // completes its input, the reversed first-k dW ops stay at the end (l.6)
-    std::vector<int> dos, tail;
-    std::vector<char> is_tail(L + 1, 0);
-    for (int op : s->D)
-      if (op > 0) dos.push_back(op);
-    // dW ops after the last dO op in D are the reversed first-k tail
-    int last_do = -1;
-    for (int j = 0; j < (int)s->D.size(); ++j) if (s->D[j] > 0) last_do = j;
-    for (int j = last_do + 1; j < (int)s->D.size(); ++j) {
-      tail.push_back(s->D[j]);
-      is_tail[-s->D[j]] = 1;
-    }
-    const int nd = (int)dos.size();
-    std::vector<char> has_do(L + 2, 0);
-    for (int op : dos) has_do[op] = 1;
-    for (int sdiag = 0; sdiag < nd + G - 1; ++sdiag) {
-      for (int g = 0; g < G; ++g) {
-        const int jj = sdiag - g;
-        if (jj < 0 || jj >= nd) continue;
-        const int i = dos[jj];
-        add_op(+i, g);
-        if (g == G - 1) {
-          // release dW ops whose input dZ is now fully produced
-          if (!is_tail[i]) add_op(-i, 0);
-          if (i == 2 && !has_do[1] && !is_tail[1]) add_op(-1, 0);
-        }
-      }
-    }
-    if (nd == 0 && !is_tail[1]) add_op(-1, 0);   // L == 1 without input grad
-    for (int w : tail) add_op(w, 0);
-  }
-  P.nops = nops;
-  P.ntasks = first;
-  CUtensorMap tmDX;
-  if (dX) OOO_TRY(make_map(&tmDX, dX, s->dims[0], p.M, 32, 32, 64));
-  else tmDX = s->lr[0].dxA;   // unused placeholder
-  TimedRec *tr;
-  OOO_TRY(begin_rec(s, s->hi, 8, 0, 0, &tr));
-  CU_TRY(ooo::eng::launch_engine(p.cg, P, &tmDX, &tmDX, s->engine_ctas, s->hi, s->prio_hi));
-  OOO_TRY(end_rec(tr, s->hi, s->engine_ctas, flops, 0));
+  s->eng_crit.clear();
+  s->eng_defer.clear();
+  s->eng_flops = 0;
+  engine_bwd_units(s, in_order, s->eng_crit, s->eng_defer, s->eng_flops);
+  s->eng_dX = dX;
+  s->eng_in_order = in_order;
+  s->eng_pending = true;
   if (comm) {
     // S[dW] per bucket in D's dW order: the comm stream waits for the bucket's
     // dW tiles (engine counter), all-reduces, and publishes ar_done for F_i.
@@ -1007,6 +1041,49 @@ int64_t ooo_deferral_bytes(const ooo_stack_desc *d, int32_t k) {
   return s;
 }
 
+ooo_status ooo_engine_plan(const ooo_stack_desc *d, ooo_schedule sch, int32_t fused, int32_t workers,
+                           int32_t *out, int32_t cap, int32_t *n, int32_t *topological) {
+  OOO_TRY(validate_desc(d, false));
+  if (!n || !topological || (cap > 0 && !out)) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL output");
+  if (sch.kind != OOO_SCHED_IN_ORDER && sch.kind != OOO_SCHED_FIRST_K)
+    return fail(OOO_ERR_INVALID_ARGUMENT, "schedule kind %d invalid", sch.kind);
+  if (sch.k < 0) return fail(OOO_ERR_INVALID_ARGUMENT, "k must be >= 0");
+  ooo_stack tmp;
+  tmp.d = *d;
+  tmp.dims.assign(d->dims, d->dims + d->num_layers + 1);
+  tmp.p = make_plan(d);
+  if (!tmp.p.engine) return fail(OOO_ERR_UNSUPPORTED, "no engine for this stack (fp32 or OOO_ENGINE=0)");
+  const bool in_order = sch.kind == OOO_SCHED_IN_ORDER;
+  schedule_ops(tmp.p.L, sch.kind, sch.k, d->need_input_grad != 0, tmp.D);
+  std::vector<pl::Unit> crit, defer;
+  double flops = 0;
+  engine_bwd_units(&tmp, in_order, crit, defer, flops);
+  if (fused) {
+    crit.push_back(unit_of(&tmp, pl::COPY, 1));
+    for (int i = 1; i <= tmp.p.L; ++i) crit.push_back(unit_of(&tmp, pl::FWD, i));
+  }
+  pl::Problem pb;
+  pb.L = tmp.p.L;
+  pb.rows = (tmp.p.cl.MT + tmp.p.cg - 1) / tmp.p.cg;
+  pb.workers = workers > 0 ? workers : std::max(1, kSMs / tmp.p.cg);
+  pb.in_order = in_order;
+  pb.fwd_gate = fused ? (d->world_size > 1 && d->comm_enabled ? 2 : 1) : 0;
+  pb.bucket.resize(pb.L);
+  for (int i = 1; i <= pb.L; ++i) pb.bucket[i - 1] = tmp.p.layer[i - 1].bucket;
+  pb.crit = crit;
+  pb.defer = defer;
+  const std::vector<pl::Unit> order = pl::schedule(pb, plan_model(), ooo::eng::kMaxOps);
+  if (order.empty()) return fail(OOO_ERR_UNSUPPORTED, "queue does not fit the op table");
+  for (size_t j = 0; j < order.size() && (int32_t)j < cap; ++j) {
+    const pl::Unit &u = order[j];
+    int32_t *o = out + 5 * j;
+    o[0] = u.kind; o[1] = u.layer; o[2] = u.m_off; o[3] = u.mt; o[4] = u.nt;
+  }
+  *n = (int32_t)order.size();
+  *topological = pl::topological(pb, order) ? 1 : 0;
+  return OOO_OK;
+}
+
 ooo_status ooo_get_unique_id(void *out) {
   if (!out) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL output");
   const char *why = nullptr;
@@ -1104,6 +1181,7 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
       L.Z = r.Z;
       L.dbpart = r.db;
       L.db_out = r.gb;
+      L.X = r.X;
       L.Xn = r.Xn;
       L.dZ = r.dZ;
       L.gw = r.gw;
@@ -1121,7 +1199,7 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
       ce = cudaMemcpy(s->ws + p.off_layers, ldev.data(), ldev.size() * sizeof(ooo::eng::LayerDev),
                       cudaMemcpyHostToDevice);
     if (ce == cudaSuccess)
-      ce = cudaMemset(s->ws + p.off_ctr, 0, (size_t)(p.cl.bwd_base + p.cl.bwd_size) * 4);
+      ce = cudaMemset(s->ws + p.off_ctr, 0, (size_t)p.cl.total * 4);
     if (ce != cudaSuccess)
       return cleanup_fail(fail(OOO_ERR_CUDA, "engine tables upload: %s", cudaGetErrorString(ce)));
     s->dmaps = reinterpret_cast<const CUtensorMap *>(s->ws + p.off_maps);
@@ -1203,6 +1281,7 @@ ooo_status ooo_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void *dX
 
 ooo_status ooo_join(ooo_stack *s, void *stream) {
   if (!s) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL stack");
+  OOO_TRY(engine_flush(s));
   OOO_TRY(join_into(s, static_cast<cudaStream_t>(stream)));
   return check_async(s);
 }
@@ -1264,6 +1343,7 @@ ooo_status ooo_graph_destroy(ooo_graph *g) {
 
 ooo_status ooo_destroy(ooo_stack *s) {
   if (!s) return OOO_OK;
+  if (s->eng_pending) (void)engine_flush(s);   // the comm stream may be waiting on its counters
   if (s->hi) cudaStreamSynchronize(s->hi);
   if (s->lo) cudaStreamSynchronize(s->lo);
   if (s->comm) cudaStreamSynchronize(s->comm);
@@ -1335,5 +1415,20 @@ ooo_status ooo_timing_read(ooo_stack *s, ooo_launch_record *out, int32_t cap, in
 extern "C" ooo_status ooo_debug_set_trace(void *dev_ptr) {
   CU_TRY(ooo::eng::engine_set_trace(dev_ptr));
   return OOO_OK;
+}
+
+// the most recent engine launch's queue as (kind, layer,
+// tiles) triples; returns the number of ops.
+extern "C" int32_t ooo_debug_last_queue(ooo_stack *s, int32_t *out, int32_t cap) {
+  int32_t n = 0;
+  for (const auto &o : s->last_queue) {
+    if (n < cap) {
+      out[3 * n] = o.kind;
+      out[3 * n + 1] = o.layer;
+      out[3 * n + 2] = o.mt * o.nt;
+    }
+    ++n;
+  }
+  return n;
 }
 #endif

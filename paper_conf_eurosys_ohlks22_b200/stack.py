@@ -77,6 +77,24 @@ def deferral_bytes(dims, acts, tokens, dtype, k) -> int:
     return int(load().ooo_deferral_bytes(ctypes.byref(d), int(k)))
 
 
+def engine_plan(dims, acts, tokens, kind="first_k", k=0, fused=True, workers=0, need_input_grad=False,
+                bucket_layers=1, world_size=1):
+    """The engine's planned tile queue for one step (host only): list of
+    (kind, layer, first_row, rows, col_tiles) with kind 'F'/'dO'/'dW'/'copy',
+    and whether it is a topological order of the step's dependencies."""
+    d, _keep = _desc(dims, acts, tokens, "bf16", need_input_grad=need_input_grad,
+                     bucket_layers=bucket_layers, world_size=world_size)
+    cap = 4096
+    out = (c_int32 * (5 * cap))()
+    n, topo = c_int32(), c_int32()
+    check(load().ooo_engine_plan(ctypes.byref(d), _lib.schedule(kind, k), int(bool(fused)), int(workers), out, cap,
+                                 ctypes.byref(n), ctypes.byref(topo)))
+    names = {0: "F", 1: "dO", 2: "dW", 3: "copy"}
+    ops = [(names[out[5 * j]], out[5 * j + 1], out[5 * j + 2], out[5 * j + 3], out[5 * j + 4])
+           for j in range(min(n.value, cap))]
+    return ops, bool(topo.value)
+
+
 def get_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(_lib.UNIQUE_ID_BYTES)
     check(load().ooo_get_unique_id(buf))

@@ -11,7 +11,8 @@ import pytest
 import torch
 
 from paper_conf_eurosys_ohlks22_b200 import configs
-from tests.gpu_helpers import Case, bf16_floor, max_err
+from oracle.layers import rel_fro
+from tests.gpu_helpers import TDT, Case, bf16_floor, max_err, to_dev, to_np
 
 pytestmark = pytest.mark.gpu
 
@@ -138,3 +139,47 @@ def test_bf16_bert_base_full_config_end_to_end():
     errs = max_err(out, ref)
     print("bert_base full-size errors", errs, "floor", bf16_floor(c.L))
     _check(errs, max(BF16_TOL, 2 * bf16_floor(c.L)))
+
+
+# ------------------------------- fused step: backward(t) + forward(t+1)
+@pytest.mark.parametrize("kind,k,tokens,need_dx", [("first_k", 2, 400, False), ("first_k", 5, 264, True),
+                                                   ("in_order", 0, 512, False), ("first_k", 0, 136, False)])
+def test_bf16_fused_step_across_iterations(kind, k, tokens, need_dx):
+    """ooo_backward(t); ooo_forward(X_{t+1}) runs as one engine launch whose
+    F_i tiles overlap the deferred dW tiles (Fig. 4(c)).  Over three
+    iterations with fresh inputs per step, check against the oracle the
+    gradients of step t and Y of step t+1 (which must see the new X and no
+    partially overwritten activations), and bit-exactness against the
+    unfused sequence (backward; join; forward) on a second stack."""
+    dims, acts = [192, 320, 256, 448, 256, 192], ["gelu", "id", "gelu", "gelu", "id"]
+    cases = [Case(dims, acts, tokens, "bf16", need_dx=need_dx, step=t) for t in range(3)]
+    fused = cases[0].stack(bucket_layers=2)
+    plain = cases[0].stack(bucket_layers=2)
+    Xs = [to_dev(c.X, "bf16") for c in cases]
+    dYs = [to_dev(c.dY, "bf16") for c in cases]
+    dXa = torch.empty(tokens, dims[0], dtype=TDT["bf16"], device="cuda") if need_dx else None
+    dXb = torch.empty_like(dXa) if need_dx else None
+    Ya = fused.forward(Xs[0])
+    Yb = plain.forward(Xs[0])
+    for t in range(3):
+        ref = cases[t].oracle(k if kind == "first_k" else 0)
+        torch.cuda.synchronize()
+        assert rel_fro(to_np(Ya), ref.Y[0]) <= BF16_TOL, t
+        assert torch.equal(Ya, Yb), t
+        fused.backward(dYs[t], kind, k, dXa)
+        plain.backward(dYs[t], kind, k, dXb)
+        plain.join()
+        if t < 2:
+            Ya = fused.forward(Xs[t + 1])       # fused launch
+            Yb = plain.forward(Xs[t + 1])
+        else:
+            fused.join()
+        torch.cuda.synchronize()
+        assert torch.equal(fused.grads_buf, plain.grads_buf), t
+        if need_dx:
+            assert torch.equal(dXa, dXb), t
+        out = {"Y": ref.Y[0], "dW": [to_np(w) for w in fused.dW], "db": [to_np(v) for v in fused.db],
+               "dX": to_np(dXa) if need_dx else None}
+        _check(max_err(out, ref), BF16_TOL)
+    fused.close()
+    plain.close()

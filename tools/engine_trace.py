@@ -3,7 +3,7 @@
     python -m paper_conf_eurosys_ohlks22_b200.build --trace
     python tools/engine_trace.py [C2] [k]
 
-For each op of the forward and backward queues: number of tiles, time from
+For each op of the backward-alone, forward-alone and fused-step queues: number of tiles, time from
 the pass start to its first dispense / first input-ready / last completion,
 mean per-tile durations (dispense->ready = dependency wait, ready->acc =
 mainloop, acc->done = epilogue) and the number of distinct CTAs.  A tuning
@@ -24,38 +24,16 @@ from paper_conf_eurosys_ohlks22_b200 import _lib, configs, synth  # noqa: E402
 from paper_conf_eurosys_ohlks22_b200.stack import OooStack, schedule_order  # noqa: E402
 
 
-def ebn(n):
-    f = int(os.environ.get("OOO_EBN", "0"))
-    if f and n % f == 0:
-        return f
-    return 256 if n % 256 == 0 else 128
+KIND = {0: "F", 1: "dX", 2: "dW", 3: "cp"}
 
 
-def queue(cfg, D, in_order):
-    """(kind, layer, ntiles) in engine queue order (mirrors engine_backward)."""
-    MT = ((cfg.tokens + 127) // 128 + 1) // 2      # 256-row pair tiles
-    ops, pending = [], []
-
-    def add(op):
-        i = abs(op)
-        din, dout = cfg.dims[i - 1], cfg.dims[i]
-        if op > 0:
-            ops.append(("dX", i, MT * ((din + ebn(din) - 1) // ebn(din))))
-        else:
-            ops.append(("dW", i, (((din + 127) // 128 + 1) // 2) * ((dout + ebn(dout) - 1) // ebn(dout))))
-    for op in D:
-        if op > 0:
-            add(op)
-            for w in pending:
-                add(w)
-            pending = []
-        elif in_order:
-            add(op)
-        else:
-            pending.append(op)
-    for w in pending:
-        add(w)
-    return ops
+def last_queue(lib, stk):
+    """(kind, layer, ntiles) of the most recent engine launch (debug export)."""
+    lib.ooo_debug_last_queue.restype = ctypes.c_int32
+    lib.ooo_debug_last_queue.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32]
+    buf = (ctypes.c_int32 * (3 * 1024))()
+    n = lib.ooo_debug_last_queue(stk._h, buf, 1024)
+    return [(KIND[buf[3 * j]], buf[3 * j + 1], buf[3 * j + 2]) for j in range(n)]
 
 
 def report(name, ops, buf):
@@ -99,7 +77,6 @@ def main():
     lib.ooo_debug_set_trace.restype = ctypes.c_int32
     lib.ooo_debug_set_trace.argtypes = [ctypes.c_void_p]
     dev = torch.device("cuda")
-    os.environ["OOO_GROUPS"] = "1"     # the report assumes layer-major queues
     W, b = synth.weights_torch(cfg.dims, cfg.acts, cfg.dtype, dev)
     stk = OooStack(cfg.dims, cfg.acts, cfg.tokens, W, b, dtype=cfg.dtype)
     X = synth.activations_torch(cfg.tokens, cfg.dims[0], cfg.dtype, dev, 1, 0, 0)
@@ -112,15 +89,18 @@ def main():
     buf = torch.zeros(2 * 200000 * 8, dtype=torch.int64, device=dev)
     _lib.check(lib.ooo_debug_set_trace(buf.data_ptr()))
     stk.backward(dY, "first_k", k)
+    stk.join()
     torch.cuda.synchronize()
-    D = schedule_order(cfg.L, "first_k", k)
-    report(f"backward first_k({k})", queue(cfg, D, False), buf)
+    report(f"backward first_k({k}) alone", last_queue(lib, stk), buf)
     buf.zero_()
     stk.forward(X, Y)
     torch.cuda.synchronize()
-    MT = ((cfg.tokens + 127) // 128 + 1) // 2
-    fops = [("F", i, MT * ((cfg.dims[i] + ebn(cfg.dims[i]) - 1) // ebn(cfg.dims[i]))) for i in range(1, cfg.L + 1)]
-    report("forward", fops, buf)
+    report("forward alone", last_queue(lib, stk), buf)
+    buf.zero_()
+    stk.backward(dY, "first_k", k)
+    stk.forward(X, Y)
+    torch.cuda.synchronize()
+    report(f"fused step first_k({k})", last_queue(lib, stk), buf)
     _lib.check(lib.ooo_debug_set_trace(None))
 
 
