@@ -62,9 +62,20 @@ __device__ unsigned long long *g_etrace2 = nullptr;
 __device__ __forceinline__ void etrace2(int t, int slot) {
   if (g_etrace2 && t >= 0) g_etrace2[(size_t)t * 8 + slot] = clock64();
 }
+// pipeline globaltimer stamps [task][8] (third region): 4 accumulator free
+// (MMA may start), 5 last MMA issued, 6 first k-block load issued, 7 last
+__device__ unsigned long long *g_etrace3 = nullptr;
+__device__ __forceinline__ void etrace_gt(int t, int slot) {
+  if (g_etrace3 && t >= 0) {
+    unsigned long long v;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(v));
+    g_etrace3[(size_t)t * 8 + slot] = v;
+  }
+}
 #else
 __device__ __forceinline__ void etrace(int, int) {}
 __device__ __forceinline__ void etrace2(int, int) {}
+__device__ __forceinline__ void etrace_gt(int, int) {}
 #endif
 
 #ifndef OOO_EPI_WARPS
@@ -83,7 +94,7 @@ constexpr uint64_t kTimeoutNs = 4000000000ull;
 template <int CG> struct Cfg {
   static constexpr int B_BYTES = (kMaxBN / CG) * BK * 2;   // this CTA's share of B
   static constexpr int STAGE = A_BYTES + B_BYTES;
-  static constexpr int STAGES = CG == 2 ? 6 : 4;
+  static constexpr int STAGES = CG == 2 ? (kEpiWarps > 8 ? 5 : 6) : (kEpiWarps > 8 ? 3 : 4);
   static constexpr int RING = STAGE * STAGES;
   static constexpr int STG_OFF = RING;
   static constexpr int BAR_OFF = STG_OFF + STG_BYTES;
@@ -277,8 +288,9 @@ __global__ void __launch_bounds__(kThreads, 1)
                   const __grid_constant__ Params p) {
   using C = Cfg<CG>;
   extern __shared__ uint8_t smem_raw[];
-  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
-                                              ~static_cast<uintptr_t>(1023));
+  // 1 KiB alignment by pointer arithmetic on the __shared__ array, so that the
+  // compiler keeps the shared address space (LDS/STS, not generic LD/ST)
+  uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   const uint32_t sbase = smem_u32(smem);
   const uint32_t bar_full = sbase + C::BAR_OFF;
   const uint32_t bar_empty = bar_full + 8 * C::STAGES;
@@ -388,6 +400,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         for (int kb = 0; kb < T.nkb; ++kb, ++it) {
           const int s = it % C::STAGES;
           if (it >= C::STAGES) mbar_wait_b(bar_empty + 8 * s, ((it / C::STAGES) - 1) & 1);
+          if (leader && (kb == 0 || kb == T.nkb - 1)) etrace_gt(t, kb == 0 ? 6 : 7);
           if (leader) mbar_expect_tx(bar_full + 8 * s, bytes);
           const uint32_t lb = L_full + 8 * s;
           const uint32_t sa = sbase + s * C::STAGE;
@@ -446,6 +459,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         }
         ++ja;
         fence_after();
+        etrace_gt(t, 4);                         // accumulator free: MMA may start
         const uint32_t dtm = tmem + (uint32_t)(acc * kMaxBN);
         for (int kb = 0; kb < T.nkb; ++kb, ++it) {
           const int s = it % C::STAGES;
@@ -463,6 +477,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (CG == 2) umma_commit_pair(bar_empty + 8 * s); else umma_commit(bar_empty + 8 * s);
         }
         if (CG == 2) umma_commit_pair(bar_tfull + 8 * acc); else umma_commit(bar_tfull + 8 * acc);
+        etrace_gt(t, 5);                         // last MMA issued
       }
     }
     __syncwarp();
@@ -566,7 +581,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (tr2 && c == h) etrace2(t, 1);
         if (T.kind == EPI_FWD) {
 #pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = __bfloat162float(__float2bfloat16_rn(v[i] + bias_s[c * 32 + i]));
+          for (int i = 0; i < 32; ++i) v[i] += bias_s[c * 32 + i];
+          round_bf16x32(v);
           if (zout && !(dbg & 2)) store32_rows(zout, T.N, stg, lane, v, col0, row0, T.M);   // Z_i
           if (!(dbg & 1)) act_chunk32(act, v);
           if (!(dbg & 2)) store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);  // X_{i+1} (or Y)
@@ -577,8 +593,9 @@ __global__ void __launch_bounds__(kThreads, 1)
             if (c + kEpiPerQ < nch && col0 + 32 * kEpiPerQ < T.N) ld_raw32(zrow + (c + kEpiPerQ) * 32, zr);
             act_grad_mul_chunk32(act, v, z);
           }
+          round_bf16x32(v);
 #pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = row_ok ? __bfloat162float(__float2bfloat16_rn(v[i])) : 0.f;
+          for (int i = 0; i < 32; ++i) v[i] = row_ok ? v[i] : 0.f;
           if (!(dbg & 2)) store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);  // dZ_{i-1} (or dX)
           if (dbpart) red[q * kMaxBN + c * 32 + lane] = warp_colsum32(v, lane);
         } else {  // EPI_WGRAD: one split, scaled bf16 straight into the gradient bucket
@@ -658,10 +675,12 @@ int engine_smem_bytes(int cg) { return cg == 2 ? Cfg<2>::SMEM : Cfg<1>::SMEM; }
 
 #ifdef OOO_TRACE
 cudaError_t engine_set_trace(void *p) {
-  // [task][8] phase stamps, followed by [task][8] epilogue clocks (same buffer, second half)
+  // [task][8] phase stamps, [task][8] epilogue clocks, [task][8] pipeline stamps (same buffer)
   void *p2 = p ? static_cast<char *>(p) + (size_t)200000 * 8 * 8 : nullptr;
+  void *p3 = p ? static_cast<char *>(p) + (size_t)2 * 200000 * 8 * 8 : nullptr;
   cudaError_t e = cudaMemcpyToSymbol(g_etrace, &p, sizeof(p));
   if (e == cudaSuccess) e = cudaMemcpyToSymbol(g_etrace2, &p2, sizeof(p2));
+  if (e == cudaSuccess) e = cudaMemcpyToSymbol(g_etrace3, &p3, sizeof(p3));
   return e;
 }
 #endif

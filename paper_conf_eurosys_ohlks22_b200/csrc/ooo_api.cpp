@@ -1417,15 +1417,17 @@ extern "C" ooo_status ooo_debug_set_trace(void *dev_ptr) {
   return OOO_OK;
 }
 
-// the most recent engine launch's queue as (kind, layer,
-// tiles) triples; returns the number of ops.
+// the most recent engine launch's queue as (kind, layer, m_off in 128-row
+// blocks, tile rows, column tiles) per op; returns the number of ops.
 extern "C" int32_t ooo_debug_last_queue(ooo_stack *s, int32_t *out, int32_t cap) {
   int32_t n = 0;
   for (const auto &o : s->last_queue) {
     if (n < cap) {
-      out[3 * n] = o.kind;
-      out[3 * n + 1] = o.layer;
-      out[3 * n + 2] = o.mt * o.nt;
+      out[5 * n] = o.kind;
+      out[5 * n + 1] = o.layer;
+      out[5 * n + 2] = o.m_off;
+      out[5 * n + 3] = o.mt;
+      out[5 * n + 4] = o.nt;
     }
     ++n;
   }

@@ -210,9 +210,15 @@ __device__ __forceinline__ void st_bf16x32(__nv_bfloat16 *p, const float (&f)[32
     q[j] = u;
   }
 }
+// RNE to bf16 and back, two values per F2FP.PACK_AB (the scalar
+// __float2bfloat16_rn compiles to the slower F2F.BF16.F32 on sm_100).
 __device__ __forceinline__ void round_bf16x32(float (&f)[32]) {
 #pragma unroll
-  for (int j = 0; j < 32; ++j) f[j] = __bfloat162float(__float2bfloat16_rn(f[j]));
+  for (int j = 0; j < 16; ++j) {
+    const uint32_t u = pack_bf2(f[2 * j], f[2 * j + 1]);
+    f[2 * j] = __uint_as_float(u << 16);
+    f[2 * j + 1] = __uint_as_float(u & 0xFFFF0000u);
+  }
 }
 // Column sums over the 32 lanes of a warp: on return lane l holds the sum of
 // column l (fixed butterfly order -> deterministic).

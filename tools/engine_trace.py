@@ -31,16 +31,20 @@ def last_queue(lib, stk):
     """(kind, layer, ntiles) of the most recent engine launch (debug export)."""
     lib.ooo_debug_last_queue.restype = ctypes.c_int32
     lib.ooo_debug_last_queue.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int32]
-    buf = (ctypes.c_int32 * (3 * 1024))()
+    buf = (ctypes.c_int32 * (5 * 1024))()
     n = lib.ooo_debug_last_queue(stk._h, buf, 1024)
-    return [(KIND[buf[3 * j]], buf[3 * j + 1], buf[3 * j + 2]) for j in range(n)]
+    return [(KIND[buf[5 * j]], buf[5 * j + 1], buf[5 * j + 3] * buf[5 * j + 4], buf[5 * j + 2], buf[5 * j + 4])
+            for j in range(n)]
 
 
 def report(name, ops, buf):
     import numpy as np
     allb = buf.cpu().numpy().view(np.uint64)
+    out = os.path.join(ROOT, "gpurun_out", "trace_" + name.split()[0] + "_" + name.split()[1] + ".npz")
+    os.makedirs(os.path.dirname(out), exist_ok=True)
+    np.savez_compressed(out, raw=allb[: 3 * 200000 * 8], ops=np.array([list(o) for o in ops], dtype=object))
     raw8 = allb[: 200000 * 8].reshape(-1, 8)
-    epi = allb[200000 * 8:].reshape(-1, 8).astype(np.float64)   # epilogue phase clocks
+    epi = allb[200000 * 8: 2 * 200000 * 8].reshape(-1, 8).astype(np.float64)   # epilogue phase clocks
     raw = raw8[:, :4]
     clk = raw8[:, 4:].astype(np.float64)
     cta = (raw >> np.uint64(48)).astype(np.int64)
@@ -55,7 +59,7 @@ def report(name, ops, buf):
     mhz = np.median(dc[ok] / (dt[ok] * 1e3) * 1e3) if ok.any() else float("nan")
     print(f"== {name}: {int(valid.sum())} tasks, span {t[valid, 3].max():.1f} us, SM clock ~{mhz:.0f} MHz")
     first = 0
-    for kind, layer, n in ops:
+    for kind, layer, n, *_ in ops:
         s = slice(first, first + n)
         first += n
         tt = t[s]
@@ -63,6 +67,14 @@ def report(name, ops, buf):
               f"..{tt[:,1].max():8.1f} done {tt[:,3].min():8.1f}..{tt[:,3].max():8.1f}"
               f" wait {np.mean(tt[:,1]-tt[:,0]):6.1f} main {np.mean(tt[:,2]-tt[:,1]):6.1f}"
               f" epi {np.mean(tt[:,3]-tt[:,2]):5.1f} ctas {len(set(cta[s, 3]))}")
+        g = allb[2 * 200000 * 8:].reshape(-1, 8)[s]
+        if g[:, 7].max() > 0:
+            m48 = np.uint64((1 << 48) - 1)
+            f6 = ((g[:, 6] & m48).astype(np.float64) - t0) / 1e3
+            f7 = ((g[:, 7] & m48).astype(np.float64) - t0) / 1e3
+            ok = g[:, 7] > 0
+            print(f"     loads: first {np.mean(f6[ok] - tt[ok, 1]):6.1f} after ready, last {np.mean(f7[ok] - tt[ok, 1]):6.1f};"
+                  f" acc {np.mean(tt[ok, 2] - f7[ok]):6.1f} after last; last-load range {f7[ok].min():8.1f}..{f7[ok].max():8.1f}")
         e = epi[s]
         if e[:, 5].max() > 0:
             d = lambda a, b: np.median(e[:, b] - e[:, a])  # noqa: E731
@@ -86,7 +98,7 @@ def main():
         stk.backward(dY, "first_k", k)
         stk.forward(X, Y)
     torch.cuda.synchronize()
-    buf = torch.zeros(2 * 200000 * 8, dtype=torch.int64, device=dev)
+    buf = torch.zeros(3 * 200000 * 8, dtype=torch.int64, device=dev)
     _lib.check(lib.ooo_debug_set_trace(buf.data_ptr()))
     stk.backward(dY, "first_k", k)
     stk.join()
