@@ -643,10 +643,11 @@ namespace pl = ooo::plan;
 static_assert(pl::FWD == EPI_FWD && pl::DGRAD == EPI_DGRAD && pl::WGRAD == EPI_WGRAD &&
                   pl::COPY == ooo::eng::EPI_COPY, "planner kinds = engine task kinds");
 
-// Planner timing model (tuning knob for experiments: OOO_PLAN_SLACK).
+// Planner timing model (tuning knobs for experiments: OOO_PLAN_LEAD, OOO_PLAN_RESERVE).
 pl::Model plan_model() {
   pl::Model m;
-  if (const char *v = getenv("OOO_PLAN_SLACK")) m.slack = atof(v);
+  if (const char *v = getenv("OOO_PLAN_LEAD")) m.lead = atof(v);
+  if (const char *v = getenv("OOO_PLAN_RESERVE")) m.reserve = atof(v);
   return m;
 }
 

@@ -3,9 +3,6 @@
 
 #include <algorithm>
 #include <limits>
-#ifdef PLAN_DEBUG
-#include <cstdio>
-#endif
 
 namespace ooo {
 namespace plan {
@@ -39,6 +36,7 @@ class Sim {
     mma_.assign(W, 0.0);
     epi_.assign(W, 0.0);
     epi_prev_.assign(W, 0.0);
+    dw_until_.assign(W, 0.0);
   }
 
   OpState &op(int kind, int layer) { return ops_[kind * (pb_.L + 2) + layer]; }
@@ -91,6 +89,21 @@ class Sim {
     }
     return t;
   }
+  // The part of ready(u, r) that comes from dW ops (F_i's P:84 gate and the
+  // WAR guard on dW_{i+1}; in_order dO_i on dW_{i+1}; the copy on dW_1).
+  double dw_gate(const Unit &u) {
+    const int i = u.layer;
+    double t = 0.0;
+    if (u.kind == FWD && pb_.fwd_gate) {
+      t = pb_.fwd_gate == 1 ? op_done(WGRAD, i) : bucket_done(i);
+      if (i < pb_.L) t = std::max(t, op_done(WGRAD, i + 1));
+    } else if (u.kind == DGRAD && pb_.in_order && i < pb_.L) {
+      t = op_done(WGRAD, i + 1);
+    } else if (u.kind == COPY && pb_.fwd_gate) {
+      t = op_done(WGRAD, 1);
+    }
+    return t;
+  }
   bool emittable(const Unit &u) {
     if (u.kind == WGRAD) return ready(u, 0) < kInf;
     for (int r = u.m_off; r < u.m_off + u.mt; ++r)
@@ -113,6 +126,12 @@ class Sim {
     need = std::max(1, std::min(need, (int)f.size()));
     std::nth_element(f.begin(), f.begin() + (need - 1), f.end());
     return f[need - 1];
+  }
+
+  int dw_busy(double t) const {
+    int n = 0;
+    for (double d : dw_until_) n += d > t;
+    return n;
   }
 
   double epi_time(const Unit &u) const {
@@ -147,6 +166,7 @@ class Sim {
             done = std::max(main_end, epi_[w]) + epi;
             disp_[w] = std::max(start, main_end - m_.stages * tkb);
             mma_[w] = main_end;
+            dw_until_[w] = u.kind == WGRAD ? main_end : 0.0;
             epi_prev_[w] = epi_[w];
             epi_[w] = done;
           }
@@ -164,7 +184,7 @@ class Sim {
   const Model &m_;
   bool timing_;
   std::vector<OpState> ops_;
-  std::vector<double> disp_, mma_, epi_, epi_prev_;
+  std::vector<double> disp_, mma_, epi_, epi_prev_, dw_until_;
 };
 
 std::vector<Unit> merge(const std::vector<Unit> &v) {
@@ -182,6 +202,15 @@ std::vector<Unit> merge(const std::vector<Unit> &v) {
   return out;
 }
 
+// List scheduling in dispatch order.  The critical chain is emitted row by
+// row (F_i / dO_i are row-local); at each step the next dispatch goes to the
+// earliest free worker at time t:
+//  * the next critical row if its inputs are (predicted) complete by t + lead;
+//  * else the next dW row group if it is ready and the workers busy with dW
+//    stay below P minus the critical op's width (so the chain keeps the
+//    workers it needs when its rows become ready);
+//  * else the critical row anyway (its worker waits), or the dW group if the
+//    chain cannot proceed.
 std::vector<Unit> plan_once(const Problem &pb, const Model &m, int group_rows) {
   Sim sim(pb, m, true);
   std::vector<Unit> def;   // dW ops split into row groups
@@ -192,32 +221,38 @@ std::vector<Unit> plan_once(const Problem &pb, const Model &m, int group_rows) {
       g.mt = std::min(group_rows, u.mt - r);
       def.push_back(g);
     }
+  std::vector<Unit> crit;  // row-local critical ops split into rows
+  std::vector<int> width;  // tiles of the whole op each critical unit belongs to
+  for (const Unit &u : pb.crit) {
+    const bool rowwise = u.kind != WGRAD;
+    for (int r = 0; r < u.mt; r += rowwise ? 1 : u.mt) {
+      Unit g = u;
+      g.m_off = u.m_off + r;
+      g.mt = rowwise ? 1 : u.mt;
+      crit.push_back(g);
+      width.push_back(u.mt * u.nt);
+    }
+  }
+  const int P = std::max(1, pb.workers);
   std::vector<Unit> out;
   size_t ci = 0, di = 0;
-  const double eps = 1.0;
-  while (ci < pb.crit.size() || di < def.size()) {
-    const bool c_ok = ci < pb.crit.size() && sim.emittable(pb.crit[ci]);
+  while (ci < crit.size() || di < def.size()) {
+    const bool c_ok = ci < crit.size() && sim.emittable(crit[ci]);
     const bool d_ok = di < def.size() && sim.emittable(def[di]);
     if (!c_ok && !d_ok) return {};   // dependency cycle: cannot happen for valid inputs
     bool take_c = c_ok;
     if (c_ok && d_ok) {
-      // The critical op goes next unless a ready dW row group can run first
-      // without delaying it: the workers the critical op needs must still be
-      // free by the time its first row is ready.
-      const Unit &c = pb.crit[ci];
-      const Unit &d = def[di];
-      const int need = c.mt * c.nt;
-      const double rc = sim.ready(c, c.m_off);
-      const double rd = sim.ready(d, 0);
-      if (rd <= sim.time_free(1, nullptr, 0.0) + eps && sim.time_free(need, &d, rd) <= rc + m.slack) take_c = false;
-#ifdef PLAN_DEBUG
-      fprintf(stderr, "c=%d/L%d rc=%.1f d=L%d rd=%.1f t1=%.1f tneed=%.1f -> %s\n", c.kind, c.layer, rc, d.layer, rd,
-              sim.time_free(1, nullptr, 0.0), sim.time_free(need, &d, rd), take_c ? "c" : "d");
-#endif
+      const double t = sim.time_free(1, nullptr, 0.0);
+      const double rc = sim.ready(crit[ci], crit[ci].m_off);
+      const double rd = sim.ready(def[di], 0);
+      // a chain waiting for dW ops (F_i's gate) makes those dW ops critical: no cap
+      const bool gated = sim.dw_gate(crit[ci]) >= rc - 1e-9;
+      const int cap = gated ? P : P - std::min(P, (int)(m.reserve * width[ci] + 0.5));
+      if (rc > t + m.lead && rd <= t + m.lead && sim.dw_busy(t) + def[di].mt * def[di].nt <= cap) take_c = false;
     }
     if (take_c) {
-      sim.emit(pb.crit[ci]);
-      out.push_back(pb.crit[ci++]);
+      sim.emit(crit[ci]);
+      out.push_back(crit[ci++]);
     } else {
       sim.emit(def[di]);
       out.push_back(def[di++]);

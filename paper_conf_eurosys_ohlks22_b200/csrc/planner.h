@@ -7,8 +7,8 @@
 // Algorithm 2.  The planner turns those two priority-ordered
 // chains into one FIFO order by list scheduling against a timing model of
 // the engine (P worker CTAs / CTA pairs, per-tile mainloop and epilogue
-// times): the next critical op is emitted as soon as it is (predicted) ready;
-// while it is not, deferred dW row groups fill the workers that would
+// times): the next critical row is emitted as soon as it is (predicted)
+// ready; while it is not, deferred dW row groups fill the workers that would
 // otherwise idle, as long as enough workers stay free for the critical op.
 // Every op is emitted after all ops it depends on, so FIFO dispensing with
 // blocking waits cannot deadlock (engine.cu).  A wrong prediction only costs
@@ -39,7 +39,8 @@ struct Model {
   double epi_dx = 6.6, epi_dx_act = 11.0;
   double epi_dw = 5.2, epi_copy = 1.5;
   double ar_latency = 25.0;                  // us: bucket all-reduce (N > 1)
-  double slack = 2.0;                        // us a dW row group may delay the next critical op
+  double lead = 2.0;                         // us: a critical row is dispatched this early
+  double reserve = 0.5;                      // fraction of the critical op's width kept free of dW
 };
 
 struct Problem {
