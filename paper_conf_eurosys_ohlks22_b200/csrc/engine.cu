@@ -568,36 +568,49 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (et == 0 && leader) etrace(t, 2);
       const bool tr2 = et == 0 && leader;
       if (tr2) etrace2(t, 0);
-      for (int c = h; c < ((dbg & 4) ? 0 : nch); c += kEpiPerQ) {
+      // TMEM loads run one chunk ahead of the epilogue math (tcgen05.ld is
+      // asynchronous until tcgen05.wait::ld)
+      const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * kMaxBN);
+      const int cend = min(nch, (T.N - T.n0 + 31) >> 5);   // chunks with col0 < N
+      uint32_t ra[32];
+      if (h < cend) tmem_ld32_issue(tbase + (uint32_t)(h * 32), ra);
+      for (int c = h; c < cend; c += kEpiPerQ) {
         const int col0 = T.n0 + c * 32;
-        if (col0 >= T.N) break;
+        tmem_ld_wait(ra);
         float v[32];
-        {
-          uint32_t r[32];
-          tmem_ld32(tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * kMaxBN + c * 32), r);
 #pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
-        }
+        for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(ra[i]);
+        if (c + kEpiPerQ < cend) tmem_ld32_issue(tbase + (uint32_t)((c + kEpiPerQ) * 32), ra);
         if (tr2 && c == h) etrace2(t, 1);
         if (T.kind == EPI_FWD) {
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] += bias_s[c * 32 + i];
-          round_bf16x32(v);
-          if (zout && !(dbg & 2)) store32_rows(zout, T.N, stg, lane, v, col0, row0, T.M);   // Z_i
-          if (!(dbg & 1)) act_chunk32(act, v);
-          if (!(dbg & 2)) store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);  // X_{i+1} (or Y)
+          uint32_t u[16];
+          pack32(v, u);                                         // Z_i in bf16 (RNE)
+          if (act == ACT_ID || (dbg & 1)) {
+            if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);   // X_{i+1} = Z_i (or Y)
+          } else {
+            if (zout && !(dbg & 2)) store32_rows_packed(zout, T.N, stg, lane, u, col0, row0, T.M);   // Z_i
+            unpack32(u, v);
+            act_chunk32(act, v);
+            if (!(dbg & 2)) store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);  // X_{i+1} (or Y)
+          }
         } else if (T.kind == EPI_DGRAD) {
           if (need_z && !(dbg & 1)) {
             float z[32];
             unpack_bf16x32(zr, z);
-            if (c + kEpiPerQ < nch && col0 + 32 * kEpiPerQ < T.N) ld_raw32(zrow + (c + kEpiPerQ) * 32, zr);
+            if (c + kEpiPerQ < cend) ld_raw32(zrow + (c + kEpiPerQ) * 32, zr);
             act_grad_mul_chunk32(act, v, z);
           }
-          round_bf16x32(v);
+          uint32_t u[16];
+          pack32(v, u);                                         // dZ_{i-1} in bf16 (RNE)
 #pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = row_ok ? v[i] : 0.f;
-          if (!(dbg & 2)) store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);  // dZ_{i-1} (or dX)
-          if (dbpart) red[q * kMaxBN + c * 32 + lane] = warp_colsum32(v, lane);
+          for (int j = 0; j < 16; ++j) u[j] = row_ok ? u[j] : 0u;
+          if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);  // dZ_{i-1} (or dX)
+          if (dbpart) {
+            unpack32(u, v);
+            red[q * kMaxBN + c * 32 + lane] = warp_colsum32(v, lane);
+          }
         } else {  // EPI_WGRAD: one split, scaled bf16 straight into the gradient bucket
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] *= alpha;

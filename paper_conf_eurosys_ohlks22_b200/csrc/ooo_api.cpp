@@ -162,6 +162,8 @@ GemmPlan plan_tc_mn(int M, int N, int K, bool weight_grad) {
 int engine_bn(int N) {
   const int forced = env_int("OOO_EBN", 0);
   if (forced && N % forced == 0) return forced;
+  const int narrow = env_int("OOO_EBN_NARROW", 0);   // experiment: 192-wide tiles for N <= this
+  if (narrow && N <= narrow && N % 192 == 0) return 192;
   // CTA pairs split B in halves of >= 64 columns: bn in {128, 256}
   return N % 256 == 0 ? 256 : 128;
 }
@@ -398,6 +400,7 @@ struct ooo_stack {
   const CUtensorMap *dmaps = nullptr;         // map table (workspace)
   const ooo::eng::LayerDev *dlayers = nullptr;
   int engine_ctas = 148;
+  bool test_comm_gate = false;                // OOO_TEST_COMM_GATE=1 (N = 1 only): see comm_active
   bool eng_pending = false;                   // ooo_backward enqueued, its kernel deferred
   std::vector<ooo::plan::Unit> eng_crit, eng_defer;   // the deferred backward's chains
   double eng_flops = 0;
@@ -637,7 +640,11 @@ StreamValueFn stream_value_fn(const char *name) {
 
 int map_index(int layer, int slot) { return (layer - 1) * MS_COUNT + slot; }
 
-bool comm_active(const ooo_stack *s) { return s->nccl != nullptr && s->d.comm_enabled; }
+// The comm stream takes part in the step (bucket all-reduces + ar_done flags
+// gating F_i).  test_comm_gate: world_size 1 with the same wait-value /
+// write-value chain but no all-reduce, so single-GPU tests exercise the N > 1
+// gating of the fused step.
+bool comm_active(const ooo_stack *s) { return (s->nccl != nullptr && s->d.comm_enabled) || s->test_comm_gate; }
 
 namespace pl = ooo::plan;
 static_assert(pl::FWD == EPI_FWD && pl::DGRAD == EPI_DGRAD && pl::WGRAD == EPI_WGRAD &&
@@ -1109,6 +1116,7 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
   s->d.acts = s->acts.data();
   s->p = make_plan(d);
   s->pdl = env_int("OOO_PDL", 1) != 0;
+  s->test_comm_gate = d->world_size == 1 && s->p.engine && env_int("OOO_TEST_COMM_GATE", 0) != 0;
   s->ws = static_cast<uint8_t *>(d->workspace);
   s->grads = static_cast<uint8_t *>(d->grads);
   const Plan &p = s->p;

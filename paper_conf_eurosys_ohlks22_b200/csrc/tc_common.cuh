@@ -89,6 +89,31 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
       : "r"(taddr));
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
+// Split form for software pipelining: issue the load, do other work, then
+// wait.  The wait names the destination registers as read-write operands so
+// that the compiler cannot move their uses above it.
+__device__ __forceinline__ void tmem_ld32_issue(uint32_t taddr, uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+      "{%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
+        "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]),
+        "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]), "=r"(r[25]),
+        "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+}
+__device__ __forceinline__ void tmem_ld_wait(uint32_t (&r)[32]) {
+  asm volatile("tcgen05.wait::ld.sync.aligned;"
+               : "+r"(r[0]), "+r"(r[1]), "+r"(r[2]), "+r"(r[3]), "+r"(r[4]), "+r"(r[5]), "+r"(r[6]),
+                 "+r"(r[7]), "+r"(r[8]), "+r"(r[9]), "+r"(r[10]), "+r"(r[11]), "+r"(r[12]), "+r"(r[13]),
+                 "+r"(r[14]), "+r"(r[15]), "+r"(r[16]), "+r"(r[17]), "+r"(r[18]), "+r"(r[19]),
+                 "+r"(r[20]), "+r"(r[21]), "+r"(r[22]), "+r"(r[23]), "+r"(r[24]), "+r"(r[25]),
+                 "+r"(r[26]), "+r"(r[27]), "+r"(r[28]), "+r"(r[29]), "+r"(r[30]), "+r"(r[31])
+               :
+               : "memory");
+}
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_launch_dependents() {
   asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
@@ -301,6 +326,43 @@ __device__ __forceinline__ void store32_rows(__nv_bfloat16 *g, int ldc, uint32_t
                  : "memory");
     const int grow = row0 + r;
     if (grow < M) *reinterpret_cast<uint4 *>(g + (size_t)grow * ldc + col0 + c * 8) = make_uint4(x, y, z, w);
+  }
+}
+// store32_rows for values already packed to bf16 pairs (u[j] = columns 2j, 2j+1).
+__device__ __forceinline__ void store32_rows_packed(__nv_bfloat16 *g, int ldc, uint32_t buf, int lane,
+                                                    const uint32_t (&u)[16], int col0, int row0, int M) {
+  __syncwarp();
+  const uint32_t rbase = buf + lane * 64;
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    const uint32_t a = rbase + ((c ^ ((lane >> 1) & 3)) << 4);
+    asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(u[4 * c]), "r"(u[4 * c + 1]),
+                 "r"(u[4 * c + 2]), "r"(u[4 * c + 3])
+                 : "memory");
+  }
+  __syncwarp();
+  const int c = lane & 3;
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int r = (lane >> 2) + 8 * k;
+    uint32_t x, y, z, w;
+    asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(x), "=r"(y), "=r"(z), "=r"(w)
+                 : "r"(buf + r * 64 + ((c ^ ((r >> 1) & 3)) << 4))
+                 : "memory");
+    const int grow = row0 + r;
+    if (grow < M) *reinterpret_cast<uint4 *>(g + (size_t)grow * ldc + col0 + c * 8) = make_uint4(x, y, z, w);
+  }
+}
+__device__ __forceinline__ void pack32(const float (&f)[32], uint32_t (&u)[16]) {
+#pragma unroll
+  for (int j = 0; j < 16; ++j) u[j] = pack_bf2(f[2 * j], f[2 * j + 1]);
+}
+__device__ __forceinline__ void unpack32(const uint32_t (&u)[16], float (&f)[32]) {
+#pragma unroll
+  for (int j = 0; j < 16; ++j) {
+    f[2 * j] = __uint_as_float(u[j] << 16);
+    f[2 * j + 1] = __uint_as_float(u[j] & 0xFFFF0000u);
   }
 }
 // Same for 32 rows x 32 columns into a 2 KiB 64B-swizzled buffer (16-B chunk

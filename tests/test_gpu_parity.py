@@ -183,3 +183,35 @@ def test_bf16_fused_step_across_iterations(kind, k, tokens, need_dx):
         _check(max_err(out, ref), BF16_TOL)
     fused.close()
     plain.close()
+
+
+def test_bf16_fused_step_comm_gated(monkeypatch):
+    """The N > 1 gating of the fused step (F_i waits for its bucket's
+    all-reduce flag, written by the comm stream after cuStreamWaitValue32 on
+    the bucket's dW counter) on one GPU: OOO_TEST_COMM_GATE runs that
+    wait/write chain without the all-reduce.  Results must be bit-identical
+    to the ungated stack (the all-reduce of one rank is the identity)."""
+    dims, acts = [256, 512, 256, 256, 512, 256], ["gelu", "id", "id", "gelu", "id"]
+    cases = [Case(dims, acts, 520, "bf16", step=t) for t in range(3)]
+    plain = cases[0].stack(bucket_layers=2)
+    monkeypatch.setenv("OOO_TEST_COMM_GATE", "1")
+    gated = cases[0].stack(bucket_layers=2)
+    monkeypatch.delenv("OOO_TEST_COMM_GATE")
+    Xs = [to_dev(c.X, "bf16") for c in cases]
+    dYs = [to_dev(c.dY, "bf16") for c in cases]
+    Ya, Yb = gated.forward(Xs[0]), plain.forward(Xs[0])
+    for t in range(3):
+        gated.backward(dYs[t], "first_k", 2)
+        plain.backward(dYs[t], "first_k", 2)
+        if t < 2:
+            Ya, Yb = gated.forward(Xs[t + 1]), plain.forward(Xs[t + 1])
+        else:
+            gated.join()
+            plain.join()
+        torch.cuda.synchronize()
+        assert torch.equal(Ya, Yb), t
+        assert torch.equal(gated.grads_buf, plain.grads_buf), t
+    _check(max_err({"Y": cases[2].oracle(2).Y[0], "dW": [to_np(w) for w in gated.dW],
+                    "db": [to_np(v) for v in gated.db], "dX": None}, cases[2].oracle(2)), BF16_TOL)
+    gated.close()
+    plain.close()
