@@ -50,6 +50,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample-tokens", type=int, default=0)
+    ap.add_argument("--runs", type=int, default=5, help="extra timed runs for mean +- s.e.")
     return ap.parse_args()
 
 
@@ -286,6 +287,13 @@ def main():
     ms_ooo = timed(g_ooo, args.steps, sampler)
     clocks = sampler.summary()
     ms_in = timed(g_in, args.steps)
+    # repeat runs (mean +- standard error) and the dual-stream
+    # control ooo_first_k(0) (no reordering)
+    reps = [timed(g_ooo, args.steps) for _ in range(args.runs)]
+    g_k0 = graph_for("first_k", 0)
+    for _ in range(3):
+        g_k0.launch(stream)
+    ms_k0 = timed(g_k0, args.steps)
 
     # ---- exposed communication: same graph with the all-reduce skipped (comm-off control)
     exposed = None
@@ -372,6 +380,8 @@ def main():
     grad_bytes = cfg.params() * (2 if dt == "bf16" else 4)
     t_ar = 2 * (world - 1) / world * grad_bytes / 770e9 * 1e3 if world > 1 else 0.0
     step_roof_ms = max(t_tensor or 0.0, t_ar)
+    hbm_bytes = cfg.hbm_min_bytes()
+    t_hbm = hbm_bytes / (peaks["hbm_gbs"] * 1e9) * 1e3
 
     # ---- e2e through the public API with host buffers
     e2e = None
@@ -428,8 +438,13 @@ def main():
         "exposed_allreduce_ms": exposed,
         "allreduce_standalone_ms": ar_ms,
         "hidden_fraction": (None if not exposed or not ar_ms else 1.0 - exposed["ooo_first_k"] / ar_ms),
+        "runs": {"n": len(reps), "mean_ms": statistics.mean(reps) if reps else None,
+                 "sem_ms": (statistics.stdev(reps) / math.sqrt(len(reps))) if len(reps) > 1 else None},
+        "ooo_first_k0": {"value": 1e3 / ms_k0, "ms_per_step": ms_k0},
         "step_roofline": {"ms": step_roof_ms, "frac": step_roof_ms / ms_ooo if step_roof_ms else None,
-                          "tensor_ms": t_tensor, "allreduce_ms_at_770GBps": t_ar, "gemm_flops": flops},
+                          "tensor_ms": t_tensor, "allreduce_ms_at_770GBps": t_ar, "gemm_flops": flops,
+                          "hbm_min_bytes": hbm_bytes, "hbm_ms": t_hbm,
+                          "hbm_inclusive_ms": max(step_roof_ms, t_hbm)},
         "roofline": roof,
         "kernels": {k: {"ms_per_step": v["ms"], "launches": v["n"]} for k, v in by_kind.items()},
         "instrumented_ms_per_step": ms_timed,

@@ -30,6 +30,22 @@ class StackConfig:
     def params(self) -> int:
         return sum(self.dims[i] * self.dims[i + 1] + self.dims[i + 1] for i in range(self.L))
 
+    def hbm_min_bytes(self, need_input_grad: bool = False) -> int:
+        """Compulsory HBM bytes of one step if every op streams its operands
+        once (no reuse across ops through L2): F_i reads X_i, W_i and writes
+        Z_i (+ X_{i+1} when act_i != id); dO_i reads dZ_i, W_i (+ Z_{i-1} for
+        act') and writes dZ_{i-1}; dW_i reads X_i, dZ_i and writes dW_i, db_i."""
+        e = 2 if self.dtype == "bf16" else 4
+        M, d, a = self.tokens, self.dims, self.acts
+        t = 0
+        for i in range(self.L):
+            din, dout = d[i], d[i + 1]
+            t += M * din + din * dout + M * dout * (2 if a[i] != "id" else 1)
+            if i > 0 or need_input_grad:
+                t += M * dout + din * dout + M * din * (2 if i > 0 and a[i - 1] != "id" else 1)
+            t += M * din + M * dout + din * dout + dout
+        return t * e
+
     def gemm_flops(self, need_input_grad: bool = False) -> int:
         """fwd + dX (layers 2..L, plus 1 if requested) + dW, 2*M*din*dout each."""
         M = self.tokens
