@@ -72,10 +72,15 @@ __device__ __forceinline__ void etrace_gt(int t, int slot) {
     g_etrace3[(size_t)t * 8 + slot] = v;
   }
 }
+// per-k-block clocks of CTA 0's first task: [150000 + kb][slot]
+__device__ __forceinline__ void ktrace(int j, int kb, int slot) {
+  if (g_etrace3 && blockIdx.x == 0 && j == 0 && kb < 1024) g_etrace3[(size_t)(150000 + kb) * 8 + slot] = clock64();
+}
 #else
 __device__ __forceinline__ void etrace(int, int) {}
 __device__ __forceinline__ void etrace2(int, int) {}
 __device__ __forceinline__ void etrace_gt(int, int) {}
+__device__ __forceinline__ void ktrace(int, int, int) {}
 #endif
 
 #ifndef OOO_EPI_WARPS
@@ -138,11 +143,32 @@ __device__ __forceinline__ void st_cluster_u32(uint32_t cluster_addr, int v) {
 // Bounded mbarrier wait with the default (CTA-scope) semantics.  Spinning
 // with .acquire.cluster would emit an L1 invalidation (CCTL.IVALL) on every
 // poll -- measured at 2/3 of all warp samples.
+// The timeout clock is read only every 1024 polls: a globaltimer read on
+// every poll delays the reaction to the phase flip (hot mainloop waits).
 __device__ __forceinline__ void mbar_wait_b(uint32_t bar, uint32_t parity) {
-  if (mbar_try_wait(bar, parity)) return;
-  const uint64_t t0 = gtimer();
-  while (!mbar_try_wait(bar, parity))
-    if (gtimer() - t0 > kTimeoutNs) __trap();
+  uint64_t t0 = 0;
+  for (uint32_t n = 1; !mbar_try_wait(bar, parity); ++n) {
+    if ((n & 1023u) == 0) {
+      if (t0 == 0) t0 = gtimer();
+      else if (gtimer() - t0 > kTimeoutNs) __trap();
+    }
+  }
+}
+// Idle-waiting variant for the epilogue warps: sleep between polls so that
+// eight waiting warps do not take issue slots from the producer / MMA
+// threads of the same SM sub-partitions.
+#ifndef OOO_EPI_SLEEP_NS
+#define OOO_EPI_SLEEP_NS 64
+#endif
+__device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
+  uint64_t t0 = 0;
+  for (uint32_t n = 1; !mbar_try_wait(bar, parity); ++n) {
+    if (OOO_EPI_SLEEP_NS > 0) __nanosleep(OOO_EPI_SLEEP_NS);
+    if ((n & 255u) == 0) {
+      if (t0 == 0) t0 = gtimer();
+      else if (gtimer() - t0 > kTimeoutNs) __trap();
+    }
+  }
 }
 // For barriers that receive arrivals from the peer CTA (release.cluster):
 // one cluster-scope acquire fence after the wait, not one per poll.
@@ -261,7 +287,7 @@ __device__ __forceinline__ bool deps(const Params &p, const TaskRt &T, int mblk)
     if (mblk < cl.MT) {
       if (T.layer > 1)
         ok = dep_ge<kWait>(ctr + cl.fwd_rows + (T.layer - 2) * cl.MT + mblk, p.layers[T.layer - 2].fwd_nt);
-      else
+      else if (!(p.dbg & 8))
         ok = dep_ge<kWait>(ctr + cl.xcopy + mblk, p.copy_nt);
     }
     if (ok && p.fwd_gate == 1) ok = dep_ge<kWait>(ctr + cl.dw_done + (T.layer - 1), Ld.dw_tiles);   // P:84, N = 1
@@ -280,6 +306,59 @@ __device__ __forceinline__ bool deps(const Params &p, const TaskRt &T, int mblk)
     if (p.fwd_gate) ok = dep_ge<kWait>(ctr + cl.dw_done, p.layers[0].dw_tiles);
   }
   return ok;
+}
+
+// Producer k-loop of one task, specialised per operand layout (no per-k-block
+// branches; stage / phase advanced incrementally): waits for a free ring
+// stage, then TMA-loads this CTA's A rows and its share of B, completing on
+// the leader's full barrier.
+template <int CG, bool A_MN, bool B_MN>
+__device__ __forceinline__ void produce(const TaskRt &T, const CUtensorMap *mA, const CUtensorMap *mB, uint32_t sbase,
+                                        uint32_t bar_empty, uint32_t bar_full, uint32_t L_full, bool leader,
+                                        uint32_t bytes, int am, int bn0, int bh, int &it, int j) {
+  using C = Cfg<CG>;
+  int s = it % C::STAGES;
+  uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;   // phase of the stage's next fill
+  for (int kb = 0; kb < T.nkb; ++kb) {
+    if (it + kb >= C::STAGES) mbar_wait_b(bar_empty + 8 * s, ph ^ 1u);
+    ktrace(j, kb, 0);
+    if (leader) mbar_expect_tx(bar_full + 8 * s, bytes);
+    const uint32_t lb = L_full + 8 * s;
+    const uint32_t sa = sbase + s * C::STAGE;
+    const uint32_t sb = sa + A_BYTES;
+    const int k0 = kb * BK;
+    if (CG == 2) {
+      if (!A_MN) {
+        tma_load_2d_pair(sa, mA, lb, k0, am);                       // box {64 K, 128 M}
+      } else {
+        tma_load_2d_pair(sa, mA, lb, am, k0);                       // box {64 M, 64 K}
+        tma_load_2d_pair(sa + 8192, mA, lb, am + 64, k0);
+      }
+      if (!B_MN) {
+        tma_load_2d_pair(sb, mB, lb, k0, bn0);                      // box {64 K, bn/2 N}
+      } else {
+        tma_load_2d_pair(sb, mB, lb, bn0, k0);                      // boxes {64 N, 64 K}
+        if (bh > 64) tma_load_2d_pair(sb + 8192, mB, lb, bn0 + 64, k0);
+      }
+    } else {
+      if (!A_MN) {
+        tma_load_2d(sa, mA, lb, k0, am);
+      } else {
+        tma_load_2d(sa, mA, lb, am, k0);
+        tma_load_2d(sa + 8192, mA, lb, am + 64, k0);
+      }
+      if (!B_MN) {
+        tma_load_2d(sb, mB, lb, k0, bn0);                           // box {64 K, bn N}
+      } else {
+        for (int c = 0; c < bh / 64; ++c) tma_load_2d(sb + 8192 * c, mB, lb, bn0 + 64 * c, k0);
+      }
+    }
+    if (++s == C::STAGES) {
+      s = 0;
+      ph ^= 1u;
+    }
+  }
+  it += T.nkb;
 }
 
 template <int CG>
@@ -397,40 +476,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint32_t bytes = CG * (A_BYTES + bh * BK * 2);      // all CTAs, on the leader's barrier
         const int am = T.m0 + BM * (int)rank;
         const int bn0 = T.n0 + bh * (int)rank;
-        for (int kb = 0; kb < T.nkb; ++kb, ++it) {
-          const int s = it % C::STAGES;
-          if (it >= C::STAGES) mbar_wait_b(bar_empty + 8 * s, ((it / C::STAGES) - 1) & 1);
-          if (leader && (kb == 0 || kb == T.nkb - 1)) etrace_gt(t, kb == 0 ? 6 : 7);
-          if (leader) mbar_expect_tx(bar_full + 8 * s, bytes);
-          const uint32_t lb = L_full + 8 * s;
-          const uint32_t sa = sbase + s * C::STAGE;
-          const uint32_t sb = sa + A_BYTES;
-          const int k0 = kb * BK;
-          if (CG == 2) {
-            if (!a_mn) {
-              tma_load_2d_pair(sa, mA, lb, k0, am);                // box {64 K, 128 M}
-            } else {
-              tma_load_2d_pair(sa, mA, lb, am, k0);                // box {64 M, 64 K}
-              tma_load_2d_pair(sa + 8192, mA, lb, am + 64, k0);
-            }
-            if (!b_mn) {
-              tma_load_2d_pair(sb, mB, lb, k0, bn0);               // box {64 K, bn/2 N}
-            } else {
-              for (int c = 0; c < bh / 64; ++c) tma_load_2d_pair(sb + 8192 * c, mB, lb, bn0 + 64 * c, k0);
-            }
-          } else {
-            if (!a_mn) {
-              tma_load_2d(sa, mA, lb, k0, am);
-            } else {
-              tma_load_2d(sa, mA, lb, am, k0);
-              tma_load_2d(sa + 8192, mA, lb, am + 64, k0);
-            }
-            if (!b_mn) {
-              tma_load_2d(sb, mB, lb, k0, bn0);                    // box {64 K, bn N}
-            } else {
-              for (int c = 0; c < bh / 64; ++c) tma_load_2d(sb + 8192 * c, mB, lb, bn0 + 64 * c, k0);
-            }
-          }
+        switch ((a_mn ? 2 : 0) + (b_mn ? 1 : 0)) {
+          case 1: produce<CG, false, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j); break;
+          case 0: produce<CG, false, false>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j); break;
+          default: produce<CG, true, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j); break;
         }
       }
     }
@@ -461,21 +510,43 @@ __global__ void __launch_bounds__(kThreads, 1)
         fence_after();
         etrace_gt(t, 4);                         // accumulator free: MMA may start
         const uint32_t dtm = tmem + (uint32_t)(acc * kMaxBN);
-        for (int kb = 0; kb < T.nkb; ++kb, ++it) {
-          const int s = it % C::STAGES;
-          mbar_wait_b(bar_full + 8 * s, (it / C::STAGES) & 1);
+        // Stage-0 / k-step-0 descriptors, advanced by plain adds in the loop
+        // (address field = bits 0-13, bytes >> 4): + STAGE >> 4 per stage,
+        // + 2 per 16-deep k-step K-major (32 B), + 128 MN-major (2 KiB).  No
+        // per-MMA branches or divisions: the issue loop must keep the tensor
+        // pipe fed (measured: the generic loop cost ~870 cycles per k-block
+        // against 512 of MMA work).
+        const uint64_t a0 = a_mn ? sdesc(sbase, 8192, 1024) : sdesc(sbase, 16, 1024);
+        const uint64_t b0 = b_mn ? sdesc(sbase + A_BYTES, 8192, 1024) : sdesc(sbase + A_BYTES, 16, 1024);
+        const uint64_t astep = a_mn ? 128u : 2u, bstep = b_mn ? 128u : 2u;
+        int s = it % C::STAGES;
+        uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;
+        for (int kb = 0; kb < T.nkb; ++kb) {
+          ktrace(j, kb, 2);
+          mbar_wait_b(bar_full + 8 * s, ph);
+          ktrace(j, kb, 3);
           fence_after();
-          const uint32_t sa = sbase + s * C::STAGE;
-          const uint32_t sb = sa + A_BYTES;
-#pragma unroll
-          for (int kk = 0; kk < BK / 16; ++kk) {
-            const uint64_t ad = a_mn ? sdesc(sa + kk * 2048, 8192, 1024) : sdesc(sa + kk * 32, 16, 1024);
-            const uint64_t bd = b_mn ? sdesc(sb + kk * 2048, 8192, 1024) : sdesc(sb + kk * 32, 16, 1024);
-            if (CG == 2) umma_bf16_pair(dtm, ad, bd, ID, (kb | kk) != 0 ? 1u : 0u);
-            else umma_bf16(dtm, ad, bd, ID, (kb | kk) != 0 ? 1u : 0u);
+          const uint64_t soff = (uint64_t)(s * (C::STAGE >> 4));
+          const uint64_t ad = a0 + soff, bd = b0 + soff;
+          if (CG == 2) {
+            umma_bf16_pair(dtm, ad, bd, ID, kb != 0 ? 1u : 0u);
+            umma_bf16_pair(dtm, ad + astep, bd + bstep, ID, 1u);
+            umma_bf16_pair(dtm, ad + 2 * astep, bd + 2 * bstep, ID, 1u);
+            umma_bf16_pair(dtm, ad + 3 * astep, bd + 3 * bstep, ID, 1u);
+            umma_commit_pair(bar_empty + 8 * s);
+          } else {
+            umma_bf16(dtm, ad, bd, ID, kb != 0 ? 1u : 0u);
+            umma_bf16(dtm, ad + astep, bd + bstep, ID, 1u);
+            umma_bf16(dtm, ad + 2 * astep, bd + 2 * bstep, ID, 1u);
+            umma_bf16(dtm, ad + 3 * astep, bd + 3 * bstep, ID, 1u);
+            umma_commit(bar_empty + 8 * s);
           }
-          if (CG == 2) umma_commit_pair(bar_empty + 8 * s); else umma_commit(bar_empty + 8 * s);
+          if (++s == C::STAGES) {
+            s = 0;
+            ph ^= 1u;
+          }
         }
+        it += T.nkb;
         if (CG == 2) umma_commit_pair(bar_tfull + 8 * acc); else umma_commit(bar_tfull + 8 * acc);
         etrace_gt(t, 5);                         // last MMA issued
       }
@@ -489,8 +560,8 @@ __global__ void __launch_bounds__(kThreads, 1)
     const uint32_t stg = sbase + C::STG_OFF + (warp - 2) * 2048;
     for (int j = 0, ja = 0;; ++j) {
       const int slot = j % Q;
-      if (leader) mbar_wait_b(bar_qfull + 8 * slot, (j / Q) & 1);
-      else mbar_wait_cl(bar_qfull + 8 * slot, (j / Q) & 1);
+      mbar_wait_sleep(bar_qfull + 8 * slot, (j / Q) & 1);
+      if (!leader) asm volatile("fence.acq_rel.cluster;" ::: "memory");
       const int t = task_slot[slot];
       ebar();                                   // everyone read the slot; previous task done with smem
       if (et == 0) {
@@ -563,7 +634,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       const __nv_bfloat16 *zrow = zin ? zin + (size_t)row * T.N + T.n0 : nullptr;
       uint4 zr[4];
       if (need_z && h < nch) ld_raw32(zrow + h * 32, zr);     // act' input, prefetched before the wait
-      mbar_wait_b(bar_tfull + 8 * acc, (jacc >> 1) & 1);
+      mbar_wait_sleep(bar_tfull + 8 * acc, (jacc >> 1) & 1);
       fence_after();
       if (et == 0 && leader) etrace(t, 2);
       const bool tr2 = et == 0 && leader;

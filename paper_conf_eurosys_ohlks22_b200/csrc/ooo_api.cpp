@@ -816,7 +816,7 @@ ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st)
   for (int i = 1; i <= L; ++i) flops += 2.0 * p.M * p.layer[i - 1].din * p.layer[i - 1].dout;
   // the next forward: copy X -> X_1, then F_1..F_L (critical chain)
   std::vector<pl::Unit> fwd;
-  fwd.push_back(unit_of(s, pl::COPY, 1));
+  if (!(env_int("OOO_DBG", 0) & 8)) fwd.push_back(unit_of(s, pl::COPY, 1));   // bit 3: timing experiments only
   for (int i = 1; i <= L; ++i) fwd.push_back(unit_of(s, pl::FWD, i));
   if (s->eng_pending && env_int("OOO_FUSE", 1) == 0) OOO_TRY(engine_flush(s));   // experiments: unfused
   if (s->eng_pending) {

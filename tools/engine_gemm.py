@@ -1,8 +1,13 @@
 """Throughput of the engine's forward pass on single-layer stacks (one GEMM
 per pass) vs torch.matmul (cuBLAS) -- isolates the engine mainloop/epilogue
-from the layer-chain dependencies.  python tools/engine_gemm.py [MxNxK ...]"""
+from the layer-chain dependencies.  python tools/engine_gemm.py [MxNxK ...]
+(runs with OOO_DBG=8: the forward skips its X -> X_1 copy, so X_1 is stale
+and Y is not checked; only the time of the GEMM tiles is meaningful)"""
 import json
+import os
 import sys
+
+os.environ["OOO_DBG"] = str(int(os.environ.get("OOO_DBG", "0")) | 8)
 
 import torch
 
