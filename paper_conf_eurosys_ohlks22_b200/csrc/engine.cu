@@ -643,6 +643,12 @@ __global__ void __launch_bounds__(kThreads, 1)
       // asynchronous until tcgen05.wait::ld)
       const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * kMaxBN);
       const int cend = min(nch, (T.N - T.n0 + 31) >> 5);   // chunks with col0 < N
+      // Work the row-local successor does not need is done after the early
+      // publish below, from the accumulator still in TMEM (pass 2): the Z_i
+      // store of an activated F_i, and the bias-gradient column sums of an
+      // identity-activation dO_i (round(acc) again; act' = 1).
+      const bool late_z = T.kind == EPI_FWD && zout != nullptr && act != ACT_ID && !(dbg & 1);
+      const bool late_db = T.kind == EPI_DGRAD && dbpart != nullptr && act == ACT_ID;
       uint32_t ra[32];
       if (h < cend) tmem_ld32_issue(tbase + (uint32_t)(h * 32), ra);
       for (int c = h; c < cend; c += kEpiPerQ) {
@@ -661,7 +667,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (act == ACT_ID || (dbg & 1)) {
             if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);   // X_{i+1} = Z_i (or Y)
           } else {
-            if (zout && !(dbg & 2)) store32_rows_packed(zout, T.N, stg, lane, u, col0, row0, T.M);   // Z_i
+            // Z_i (needed only by the next backward) is stored in pass 2
             unpack32(u, v);
             act_chunk32(act, v);
             if (!(dbg & 2)) store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);  // X_{i+1} (or Y)
@@ -678,7 +684,7 @@ __global__ void __launch_bounds__(kThreads, 1)
 #pragma unroll
           for (int j = 0; j < 16; ++j) u[j] = row_ok ? u[j] : 0u;
           if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);  // dZ_{i-1} (or dX)
-          if (dbpart) {
+          if (dbpart && !late_db) {
             unpack32(u, v);
             red[q * kMaxBN + c * 32 + lane] = warp_colsum32(v, lane);
           }
@@ -690,6 +696,41 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (tr2 && c == h) etrace2(t, 2);
       }
       if (tr2) etrace2(t, 3);
+      // ---- early publish of the row-local chain output (X_{i+1} / dZ_{i-1}):
+      // release reductions are cumulative, so every store of the pass above
+      // (all epilogue warps, ordered by the barrier) is visible before the count
+      if (T.kind != EPI_WGRAD) {
+        ebar();
+        if (et == 0 && mrow0 < T.M) {
+          if (T.kind == EPI_FWD) red_release_add(ctr + cl.fwd_rows + (T.layer - 1) * cl.MT + mblk, 1);
+          else if (T.layer >= 2) red_release_add(ctr + cl.dz_rows + (T.layer - 2) * cl.MT + mblk, 1);
+          if (leader) etrace(t, 3);
+        }
+      }
+      if (late_z || late_db) {   // ---- pass 2: off-critical-path work from TMEM
+        if (h < cend) tmem_ld32_issue(tbase + (uint32_t)(h * 32), ra);
+        for (int c = h; c < cend; c += kEpiPerQ) {
+          const int col0 = T.n0 + c * 32;
+          tmem_ld_wait(ra);
+          float v[32];
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(ra[i]);
+          if (c + kEpiPerQ < cend) tmem_ld32_issue(tbase + (uint32_t)((c + kEpiPerQ) * 32), ra);
+          uint32_t u[16];
+          if (late_z) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] += bias_s[c * 32 + i];
+            pack32(v, u);
+            if (!(dbg & 2)) store32_rows_packed(zout, T.N, stg, lane, u, col0, row0, T.M);   // Z_i
+          } else {
+            pack32(v, u);
+#pragma unroll
+            for (int j = 0; j < 16; ++j) u[j] = row_ok ? u[j] : 0u;
+            unpack32(u, v);
+            red[q * kMaxBN + c * 32 + lane] = warp_colsum32(v, lane);
+          }
+        }
+      }
       // accumulator buffer free for task j+2 (the leader's barrier counts all CTAs)
       fence_before();
       __syncwarp();
@@ -727,18 +768,15 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (et == 0 && mrow0 < T.M) {
         // release reductions are cumulative: every store of the tile (all
         // epilogue warps, ordered by the barrier above) is visible before the count
-        if (T.kind == EPI_FWD) {
-          red_release_add(ctr + cl.fwd_rows + (T.layer - 1) * cl.MT + mblk, 1);
-        } else if (T.kind == EPI_DGRAD) {
-          if (T.layer >= 2) {
-            red_release_add(ctr + cl.dz_rows + (T.layer - 2) * cl.MT + mblk, 1);
-            red_release_add(ctr + cl.dz_total + (T.layer - 2), 1);
-          }
-        } else {
+        // (F_i: nothing left to publish -- its Z_i store is ordered before the
+        // next backward by the launch boundary)
+        if (T.kind == EPI_DGRAD) {
+          if (T.layer >= 2) red_release_add(ctr + cl.dz_total + (T.layer - 2), 1);   // + the db partials
+        } else if (T.kind == EPI_WGRAD) {
           red_release_add(ctr + cl.dw_done + (T.layer - 1), 1);
           red_release_add(ctr + cl.bucket_done + Ld.bucket, 1);
+          if (leader) etrace(t, 3);
         }
-        if (leader) etrace(t, 3);
       }
     }
   }
