@@ -308,51 +308,103 @@ __device__ __forceinline__ bool deps(const Params &p, const TaskRt &T, int mblk)
   return ok;
 }
 
+// F_i's gate on the weights: S[dW_i] done (N = 1: dW_i's tiles, N > 1:
+// the bucket's all-reduce flag), blocking.
+__device__ __forceinline__ void wgate(const Params &p, const TaskRt &T) {
+  const LayerDev &Ld = p.layers[T.layer - 1];
+  if (p.fwd_gate == 1) wait_ge(p.ctr + p.cl.dw_done + (T.layer - 1), Ld.dw_tiles);
+  else if (p.fwd_gate == 2) wait_ge(p.ctr + p.cl.ar_done + Ld.bucket, 1);
+}
+
+// TMA loads of one k-block stage: this CTA's A rows / its share of B,
+// completing on the leader's full barrier.
+template <int CG, bool A_MN>
+__device__ __forceinline__ void load_a(const CUtensorMap *mA, uint32_t sa, uint32_t lb, int am, int k0) {
+  if (CG == 2) {
+    if (!A_MN) {
+      tma_load_2d_pair(sa, mA, lb, k0, am);                       // box {64 K, 128 M}
+    } else {
+      tma_load_2d_pair(sa, mA, lb, am, k0);                       // box {64 M, 64 K}
+      tma_load_2d_pair(sa + 8192, mA, lb, am + 64, k0);
+    }
+  } else {
+    if (!A_MN) {
+      tma_load_2d(sa, mA, lb, k0, am);
+    } else {
+      tma_load_2d(sa, mA, lb, am, k0);
+      tma_load_2d(sa + 8192, mA, lb, am + 64, k0);
+    }
+  }
+}
+template <int CG, bool B_MN>
+__device__ __forceinline__ void load_b(const CUtensorMap *mB, uint32_t sb, uint32_t lb, int bn0, int bh, int k0) {
+  if (CG == 2) {
+    if (!B_MN) {
+      tma_load_2d_pair(sb, mB, lb, k0, bn0);                      // box {64 K, bn/2 N}
+    } else {
+      tma_load_2d_pair(sb, mB, lb, bn0, k0);                      // boxes {64 N, 64 K}
+      if (bh > 64) tma_load_2d_pair(sb + 8192, mB, lb, bn0 + 64, k0);
+    }
+  } else {
+    if (!B_MN) {
+      tma_load_2d(sb, mB, lb, k0, bn0);                           // box {64 K, bn N}
+    } else {
+      for (int c = 0; c < bh / 64; ++c) tma_load_2d(sb + 8192 * c, mB, lb, bn0 + 64 * c, k0);
+    }
+  }
+}
+
+// Weight prefetch: the B operand of F_i / dO_i is W_i, which does not depend
+// on the row-local chain, so the first npre stages are claimed and their W
+// tiles requested before the producer waits for the activation rows (the
+// HBM latency of the weights overlaps the chain hand-off).  The full
+// barrier's expect_tx (leader) already counts the A bytes issued later.
+template <int CG, bool B_MN>
+__device__ __forceinline__ void prefetch_b(const CUtensorMap *mB, uint32_t sbase, uint32_t bar_empty,
+                                           uint32_t bar_full, uint32_t L_full, bool leader, uint32_t bytes, int bn0,
+                                           int bh, int it, int npre) {
+  using C = Cfg<CG>;
+  int s = it % C::STAGES;
+  uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;
+  for (int kb = 0; kb < npre; ++kb) {
+    if (it + kb >= C::STAGES) mbar_wait_b(bar_empty + 8 * s, ph ^ 1u);
+    if (leader) mbar_expect_tx(bar_full + 8 * s, bytes);
+    load_b<CG, B_MN>(mB, sbase + s * C::STAGE + A_BYTES, L_full + 8 * s, bn0, bh, kb * BK);
+    if (++s == C::STAGES) {
+      s = 0;
+      ph ^= 1u;
+    }
+  }
+}
+
 // Producer k-loop of one task, specialised per operand layout (no per-k-block
 // branches; stage / phase advanced incrementally): waits for a free ring
 // stage, then TMA-loads this CTA's A rows and its share of B, completing on
-// the leader's full barrier.
+// the leader's full barrier.  The first npre stages were claimed by
+// prefetch_b: only their A loads remain.
 template <int CG, bool A_MN, bool B_MN>
 __device__ __forceinline__ void produce(const TaskRt &T, const CUtensorMap *mA, const CUtensorMap *mB, uint32_t sbase,
                                         uint32_t bar_empty, uint32_t bar_full, uint32_t L_full, bool leader,
-                                        uint32_t bytes, int am, int bn0, int bh, int &it, int j) {
+                                        uint32_t bytes, int am, int bn0, int bh, int &it, int j, int npre) {
   using C = Cfg<CG>;
   int s = it % C::STAGES;
   uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;   // phase of the stage's next fill
-  for (int kb = 0; kb < T.nkb; ++kb) {
+  for (int kb = 0; kb < npre; ++kb) {
+    ktrace(j, kb, 0);
+    load_a<CG, A_MN>(mA, sbase + s * C::STAGE, L_full + 8 * s, am, kb * BK);
+    if (++s == C::STAGES) {
+      s = 0;
+      ph ^= 1u;
+    }
+  }
+  for (int kb = npre; kb < T.nkb; ++kb) {
     if (it + kb >= C::STAGES) mbar_wait_b(bar_empty + 8 * s, ph ^ 1u);
     ktrace(j, kb, 0);
     if (leader) mbar_expect_tx(bar_full + 8 * s, bytes);
     const uint32_t lb = L_full + 8 * s;
     const uint32_t sa = sbase + s * C::STAGE;
-    const uint32_t sb = sa + A_BYTES;
-    const int k0 = kb * BK;
-    if (CG == 2) {
-      if (!A_MN) {
-        tma_load_2d_pair(sa, mA, lb, k0, am);                       // box {64 K, 128 M}
-      } else {
-        tma_load_2d_pair(sa, mA, lb, am, k0);                       // box {64 M, 64 K}
-        tma_load_2d_pair(sa + 8192, mA, lb, am + 64, k0);
-      }
-      if (!B_MN) {
-        tma_load_2d_pair(sb, mB, lb, k0, bn0);                      // box {64 K, bn/2 N}
-      } else {
-        tma_load_2d_pair(sb, mB, lb, bn0, k0);                      // boxes {64 N, 64 K}
-        if (bh > 64) tma_load_2d_pair(sb + 8192, mB, lb, bn0 + 64, k0);
-      }
-    } else {
-      if (!A_MN) {
-        tma_load_2d(sa, mA, lb, k0, am);
-      } else {
-        tma_load_2d(sa, mA, lb, am, k0);
-        tma_load_2d(sa + 8192, mA, lb, am + 64, k0);
-      }
-      if (!B_MN) {
-        tma_load_2d(sb, mB, lb, k0, bn0);                           // box {64 K, bn N}
-      } else {
-        for (int c = 0; c < bh / 64; ++c) tma_load_2d(sb + 8192 * c, mB, lb, bn0 + 64 * c, k0);
-      }
-    }
+    load_a<CG, A_MN>(mA, sa, lb, am, kb * BK);
+    load_b<CG, B_MN>(mB, sa + A_BYTES, lb, bn0, bh, kb * BK);
     if (++s == C::STAGES) {
       s = 0;
       ph ^= 1u;
@@ -463,9 +515,6 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (T.kind == EPI_COPY) continue;        // epilogue warps only
         const Op &o = p.ops[T.op];
         const LayerDev &Ld = p.layers[T.layer - 1];
-        deps<true>(p, T, T.mblk0 + (int)rank);    // this CTA's row block (no-op after a ready claim)
-        asm volatile("fence.proxy.async.global;" ::: "memory");   // TMA reads see the producers' data
-        if (leader) etrace(t, 1);
         const CUtensorMap *mA = map_of(o.mapA, p.maps, &tmY, &tmDX);
         const CUtensorMap *mB = map_of(o.mapB, p.maps, &tmY, &tmDX);
         tma_prefetch(mA);      // descriptors live in global memory: warm the TMA descriptor cache
@@ -476,10 +525,24 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint32_t bytes = CG * (A_BYTES + bh * BK * 2);      // all CTAs, on the leader's barrier
         const int am = T.m0 + BM * (int)rank;
         const int bn0 = T.n0 + bh * (int)rank;
+        int npre = 0;
+        if (T.kind != EPI_WGRAD && !(p.dbg & 16)) {
+          // B = W_i: only F_i's gate on S[dW_i] guards the weights
+          if (T.kind == EPI_FWD && p.fwd_gate) {
+            wgate(p, T);
+            asm volatile("fence.proxy.async.global;" ::: "memory");
+          }
+          npre = min(T.nkb, C::STAGES);
+          if (b_mn) prefetch_b<CG, true>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre);
+          else prefetch_b<CG, false>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre);
+        }
+        deps<true>(p, T, T.mblk0 + (int)rank);    // this CTA's row block (no-op after a ready claim)
+        asm volatile("fence.proxy.async.global;" ::: "memory");   // TMA reads see the producers' data
+        if (leader) etrace(t, 1);
         switch ((a_mn ? 2 : 0) + (b_mn ? 1 : 0)) {
-          case 1: produce<CG, false, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j); break;
-          case 0: produce<CG, false, false>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j); break;
-          default: produce<CG, true, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j); break;
+          case 1: produce<CG, false, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j, npre); break;
+          case 0: produce<CG, false, false>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j, npre); break;
+          default: produce<CG, true, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j, npre); break;
         }
       }
     }

@@ -83,7 +83,7 @@ struct Params {
   int32_t in_order;        // dO_i also waits for dW_{i+1} (conventional backprop)
   int32_t fwd_gate;        // 0: none; 1: F_i waits dW_i (N = 1); 2: F_i waits ar_done[bucket(i)]
                            // (N > 1); both also wait dW_{i+1} (it reads X_{i+1}, which F_i overwrites)
-  int32_t dbg;             // tuning experiments only (OOO_DBG): bit0 skip act math, bit1 skip stores, bit3 no X copy (stale X_1)
+  int32_t dbg;             // tuning experiments only (OOO_DBG): bit0 skip act math, bit1 skip stores, bit3 no X copy (stale X_1), bit4 no weight prefetch
   int32_t copy_nt;         // column tiles per row block of the X -> X_1 copy
   const CUtensorMap *maps;
   int32_t *ctr;            // counter array base
