@@ -212,7 +212,8 @@ ooo_status ooo_destroy(ooo_stack *s);             /* joins, then frees host/NCCL
 /* ------------------------------------------------- introspection / timing */
 /* Device pointer of an internal store (teacher-forced parity tests):
  * kind 0 = X_i (i = 1..L), 1 = Z_i (NULL for identity layers: Z_i aliases
- * X_{i+1}), 2 = dZ_i, 3 = bias-grad partials of layer i ([rows][d_i] fp32). */
+ * X_{i+1}; for GELU layers of a bf16 engine stack it holds gelu'(Z_i), the
+ * factor the backward needs), 2 = dZ_i, 3 = bias-grad partials of layer i ([rows][d_i] fp32). */
 ooo_status ooo_tensor(ooo_stack *s, int32_t kind, int32_t layer, void **ptr, int64_t *rows);
 
 /* Per-launch timing.  ooo_set_timing(s, 1) makes subsequently enqueued or

@@ -690,7 +690,8 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
       const int nch = T.bn / 32;
       // param-space fields -> registers once per task (see act_chunk32)
-      const int act = o.act;
+      // dO_i after a GELU layer: the Z_{i-1} store holds gelu'(Z_{i-1}) (see F_i below)
+      const int act = (T.kind == EPI_DGRAD && o.act == ACT_GELU) ? (int)ACT_DSTORED : (int)o.act;
       const int dbg = p.dbg;
       const float alpha = p.alpha;
       const bool need_z = (T.kind == EPI_DGRAD) && act != ACT_ID && zin != nullptr && row_ok;
@@ -710,7 +711,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       // publish below, from the accumulator still in TMEM (pass 2): the Z_i
       // store of an activated F_i, and the bias-gradient column sums of an
       // identity-activation dO_i (round(acc) again; act' = 1).
-      const bool late_z = T.kind == EPI_FWD && zout != nullptr && act != ACT_ID && !(dbg & 1);
+      const bool late_z = T.kind == EPI_FWD && zout != nullptr && act == ACT_RELU && !(dbg & 1);
       const bool late_db = T.kind == EPI_DGRAD && dbpart != nullptr && act == ACT_ID;
       uint32_t ra[32];
       if (h < cend) tmem_ld32_issue(tbase + (uint32_t)(h * 32), ra);
@@ -729,8 +730,19 @@ __global__ void __launch_bounds__(kThreads, 1)
           pack32(v, u);                                         // Z_i in bf16 (RNE)
           if (act == ACT_ID || (dbg & 1)) {
             if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);   // X_{i+1} = Z_i (or Y)
+          } else if (act == ACT_GELU) {
+            // X_{i+1} = gelu(Z_i) and, for the next backward, gelu'(Z_i) in
+            // the Z_i store (one Phi / e^{-z^2/2} evaluation for both; the
+            // backward's dO_{i+1} epilogue then only multiplies)
+            unpack32(u, v);
+            float d[32];
+            gelu_and_grad_chunk32(v, d);
+            if (!(dbg & 2)) {
+              store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);    // X_{i+1} (or Y)
+              store32_rows(zout, T.N, stg, lane, d, col0, row0, T.M);   // gelu'(Z_i)
+            }
           } else {
-            // Z_i (needed only by the next backward) is stored in pass 2
+            // ReLU: Z_i (needed only by the next backward) is stored in pass 2
             unpack32(u, v);
             act_chunk32(act, v);
             if (!(dbg & 2)) store32_rows(out, T.N, stg, lane, v, col0, row0, T.M);  // X_{i+1} (or Y)

@@ -16,6 +16,7 @@ namespace ooo {
 namespace ew {
 
 __device__ __forceinline__ float act_grad_f(int act, float z) {
+  if (act == ACT_DSTORED) return z;   // the Z store holds act'(Z) (engine path)
   if (act == ACT_RELU) return z > 0.f ? 1.f : 0.f;
   if (act == ACT_GELU)
     return 0.5f * (1.f + erff(z * 0.70710678118654752f)) +

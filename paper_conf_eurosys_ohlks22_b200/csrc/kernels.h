@@ -7,7 +7,10 @@
 
 namespace ooo {
 
-enum Act : int { ACT_ID = 0, ACT_RELU = 1, ACT_GELU = 2 };
+enum Act : int { ACT_ID = 0, ACT_RELU = 1, ACT_GELU = 2,
+                 // backward only: the Z store holds act'(Z) (the engine's F_i
+                 // epilogue stores gelu'(Z_i) instead of Z_i), act' = stored value
+                 ACT_DSTORED = 3 };
 enum Epi : int { EPI_FWD = 0, EPI_DGRAD = 1, EPI_WGRAD = 2 };
 
 // Row-block height of the bias-gradient partials written by the dX epilogue

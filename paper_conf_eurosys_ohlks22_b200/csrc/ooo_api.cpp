@@ -159,8 +159,9 @@ GemmPlan plan_tc_mn(int M, int N, int K, bool weight_grad) {
 // Engine tile width for an output of width N: the widest of 256/192/128/64
 // that divides N (the dataflow pipeline hides wave quantisation, so wider
 // tiles -- better MMA efficiency, less L2 traffic per FLOP -- win).
-int engine_bn(int N) {
-  const int forced = env_int("OOO_EBN", 0);
+int engine_bn(int N, bool chain) {
+  int forced = env_int(chain ? "OOO_EBN_CHAIN" : "OOO_EBN_DW", 0);
+  if (!forced) forced = env_int("OOO_EBN", 0);
   if (forced && N % forced == 0) return forced;
   const int narrow = env_int("OOO_EBN_NARROW", 0);   // experiment: 192-wide tiles for N <= this
   if (narrow && N <= narrow && N % 192 == 0) return 192;
@@ -271,9 +272,9 @@ Plan make_plan(const ooo_stack_desc *d) {
     p.cg = env_int("OOO_CG", 2) == 1 ? 1 : 2;
     for (int i = 1; i <= p.L; ++i) {
       LayerPlan &lp = p.layer[i - 1];
-      lp.ebn_fwd = engine_bn(lp.dout);
-      lp.ebn_dx = engine_bn(lp.din);
-      lp.ebn_dw = engine_bn(lp.dout);
+      lp.ebn_fwd = engine_bn(lp.dout, true);
+      lp.ebn_dx = engine_bn(lp.din, true);
+      lp.ebn_dw = engine_bn(lp.dout, false);
     }
     p.off_maps = take((size_t)p.L * MS_COUNT * sizeof(CUtensorMap));
     p.off_layers = take((size_t)p.L * sizeof(ooo::eng::LayerDev));
@@ -570,7 +571,9 @@ ooo_status launch_seed_op(ooo_stack *s, const void *dY, cudaStream_t st, int pri
   int grid = 0;
   LaunchCtx ctx{st, prio};
   const int bm = s->p.dtype == OOO_BF16 ? kTcBM : kSimtBM;
-  CU_TRY(launch_seed(s->p.dtype == OOO_BF16, dY, r.Z, lp.act, r.dZ, r.db, s->p.M, lp.dout, bm, ctx, &grid));
+  // the engine's F_L stores gelu'(Z_L) in place of Z_L (engine.cu)
+  const int act = s->p.engine && lp.act == OOO_ACT_GELU_ERF ? (int)ACT_DSTORED : (int)lp.act;
+  CU_TRY(launch_seed(s->p.dtype == OOO_BF16, dY, r.Z, act, r.dZ, r.db, s->p.M, lp.dout, bm, ctx, &grid));
   const double bytes = (double)s->p.M * lp.dout * s->p.elt * (lp.act != OOO_ACT_IDENTITY ? 3.0 : 2.0) +
                        (double)s->p.R * lp.dout * 4.0;
   return end_rec(tr, st, grid, 0, bytes);

@@ -165,6 +165,7 @@ __device__ __forceinline__ float act_f(int act, float z) {
   return z;
 }
 __device__ __forceinline__ float act_grad_f(int act, float z) {
+  if (act == ACT_DSTORED) return z;                   // z already holds act'(Z)
   if (act == ACT_RELU) return z > 0.f ? 1.f : 0.f;
   if (act == ACT_GELU) {
     float Phi, ez;
@@ -189,8 +190,22 @@ __device__ __forceinline__ void act_chunk32(int act, float (&v)[32]) {
     for (int i = 0; i < 32; ++i) v[i] = fmaxf(v[i], 0.f);
   }
 }
+// GELU of a chunk, also returning gelu'(z) = Phi(z) + z phi(z) in d (the
+// derivative the backward multiplies by; shares Phi and e^{-z^2/2}).
+__device__ __forceinline__ void gelu_and_grad_chunk32(float (&v)[32], float (&d)[32]) {
+#pragma unroll
+  for (int i = 0; i < 32; ++i) {
+    float Phi, ez;
+    gauss_cdf_exp(v[i], Phi, ez);
+    d[i] = fmaf(v[i] * 0.39894228040143268f, ez, Phi);
+    v[i] *= Phi;
+  }
+}
 __device__ __forceinline__ void act_grad_mul_chunk32(int act, float (&v)[32], const float (&z)[32]) {
-  if (act == ACT_GELU) {
+  if (act == ACT_DSTORED) {
+#pragma unroll
+    for (int i = 0; i < 32; ++i) v[i] *= z[i];
+  } else if (act == ACT_GELU) {
 #pragma unroll
     for (int i = 0; i < 32; ++i) {
       float Phi, ez;
