@@ -159,12 +159,15 @@ GemmPlan plan_tc_mn(int M, int N, int K, bool weight_grad) {
 // Engine tile width for an output of width N: the widest of 256/192/128/64
 // that divides N (the dataflow pipeline hides wave quantisation, so wider
 // tiles -- better MMA efficiency, less L2 traffic per FLOP -- win).
-int engine_bn(int N, bool chain) {
+int engine_bn(int N, bool chain, int cg, int row_tiles, int workers) {
   int forced = env_int(chain ? "OOO_EBN_CHAIN" : "OOO_EBN_DW", 0);
   if (!forced) forced = env_int("OOO_EBN", 0);
-  if (forced && N % forced == 0) return forced;
+  if (forced && N % forced == 0 && (cg == 1 || forced % 128 == 0)) return forced;
+  // skinny token dimension (one CTA row): 64-wide chain tiles spread the
+  // weight stream of F_i / dO_i over 4x more SMs (1-CTA tiles only)
+  if (chain && cg == 1 && row_tiles * (N / 256) * 4 <= workers && N % 64 == 0) return 64;
   const int narrow = env_int("OOO_EBN_NARROW", 0);   // experiment: 192-wide tiles for N <= this
-  if (narrow && N <= narrow && N % 192 == 0) return 192;
+  if (narrow && cg == 1 && N <= narrow && N % 192 == 0) return 192;
   // CTA pairs split B in halves of >= 64 columns: bn in {128, 256}
   return N % 256 == 0 ? 256 : 128;
 }
@@ -269,12 +272,17 @@ Plan make_plan(const ooo_stack_desc *d) {
   // persistent dataflow engine (bf16): map table, layer table, counters
   p.engine = p.dtype == OOO_BF16 && 2 * p.L <= ooo::eng::kMaxOps && env_int("OOO_ENGINE", 1) != 0;
   if (p.engine) {
-    p.cg = env_int("OOO_CG", 2) == 1 ? 1 : 2;
+    // CTA pairs (256-row tiles) unless the token dimension fits one 128-row tile
+    const int cg_env = env_int("OOO_CG", 0);
+    p.cg = cg_env == 1 ? 1 : (cg_env == 2 ? 2 : (p.M <= 128 ? 1 : 2));
+    const int workers = kSMs / p.cg;
+    const int MT = (p.M + 127) / 128;
+    const int PT = (MT + p.cg - 1) / p.cg;                      // tile rows of F_i / dO_i
     for (int i = 1; i <= p.L; ++i) {
       LayerPlan &lp = p.layer[i - 1];
-      lp.ebn_fwd = engine_bn(lp.dout, true);
-      lp.ebn_dx = engine_bn(lp.din, true);
-      lp.ebn_dw = engine_bn(lp.dout, false);
+      lp.ebn_fwd = engine_bn(lp.dout, true, p.cg, PT, workers);
+      lp.ebn_dx = engine_bn(lp.din, true, p.cg, PT, workers);
+      lp.ebn_dw = engine_bn(lp.dout, false, p.cg, PT, workers);
     }
     p.off_maps = take((size_t)p.L * MS_COUNT * sizeof(CUtensorMap));
     p.off_layers = take((size_t)p.L * sizeof(ooo::eng::LayerDev));

@@ -13,7 +13,9 @@ from oracle import schedule as S
 from paper_conf_eurosys_ohlks22_b200 import configs
 from paper_conf_eurosys_ohlks22_b200.stack import engine_plan
 
-CG = 2   # engine default (CTA pairs): tile rows of 256
+def _cg(tokens):
+    """Engine CTAs per tile: pairs (256-row tiles) unless the tokens fit one 128-row tile."""
+    return 1 if tokens <= 128 else 2
 
 
 def _rows(n, per):
@@ -34,6 +36,7 @@ def _check_plan(dims, acts, tokens, kind, k, fused, workers, need_dx=False, buck
             assert key not in seen, key
             seen[key] = nt
     want = {}
+    CG = _cg(tokens)
     T = _rows(_rows(tokens, 128), CG)
     for op in D:
         i = abs(op)

@@ -14,23 +14,42 @@
 
 using namespace ooo::tc;
 
-template <int MODE>   // 0: TMEM load + bias + pack only; 1: + stores; 2: + stores, no TMEM; 3: TMA stores
-__global__ void __launch_bounds__(256, 1) epi(__nv_bfloat16 *out, int ldc, int tiles, long long *cyc,
+template <int MODE, bool MMA>   // 0: TMEM load + bias + pack only; 1: + stores; 2: + stores, no TMEM; 3: TMA stores
+// MMA: a 9th warp keeps issuing 128x128x16 MMAs into TMEM columns 256-511 meanwhile
+__global__ void __launch_bounds__(288, 1) epi(__nv_bfloat16 *out, int ldc, int tiles, long long *cyc,
                                               const __grid_constant__ CUtensorMap omap) {
   __shared__ __align__(1024) uint8_t stg_all[8 * 2048];
   __shared__ float bias_s[256];
   __shared__ uint32_t tslot;
+  __shared__ __align__(1024) uint8_t opnd[16384];
+  __shared__ __align__(8) uint64_t mbar;
+  __shared__ volatile int stop;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) { stop = 0; mbar_init(smem_u32(&mbar), 1); }
   if (warp == 0) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tslot)), "r"(256)
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(&tslot)), "r"(512)
                  : "memory");
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
   }
-  bias_s[threadIdx.x] = 0.25f * threadIdx.x;
+  if (threadIdx.x < 256) bias_s[threadIdx.x] = 0.25f * threadIdx.x;
   fence_before();
   __syncthreads();
   fence_after();
   const uint32_t tmem = tslot;
+  if (warp == 8) {
+    if (MMA && lane == 0) {
+      const uint32_t ID = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(128 >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+      const uint64_t ad = sdesc(smem_u32(opnd), 16, 1024), bd = sdesc(smem_u32(opnd), 16, 1024);
+      uint32_t ph = 0;
+      while (!stop) {
+        for (int k = 0; k < 4; ++k) umma_bf16(tmem + 256, ad + 2 * k, bd + 2 * k, ID, k ? 1u : 0u);
+        umma_commit(smem_u32(&mbar));
+        mbar_wait(smem_u32(&mbar), ph);
+        ph ^= 1;
+      }
+    }
+    __syncwarp();
+  } else {
   const int q = warp & 3, h = warp >> 2;
   const uint32_t stg = smem_u32(stg_all) + warp * 2048;
   const int row0 = blockIdx.x * 128 + q * 32;
@@ -53,6 +72,11 @@ __global__ void __launch_bounds__(256, 1) epi(__nv_bfloat16 *out, int ldc, int t
       if (MODE == 3) {
         unpack32(u, v);
         stage_store32(&omap, stg, lane, v, col0, row0);
+      } else if (MODE == 4) {
+        // direct: each lane stores its own row's 64 B (4 x st.global.v4), no smem
+        uint4 *gp = reinterpret_cast<uint4 *>(out + (size_t)(row0 + lane) * ldc + col0);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) gp[j] = make_uint4(u[4 * j], u[4 * j + 1], u[4 * j + 2], u[4 * j + 3]);
       } else if (MODE >= 1) {
         store32_rows_packed(out, ldc, stg, lane, u, col0, row0, 1 << 30);
       } else {
@@ -65,10 +89,11 @@ __global__ void __launch_bounds__(256, 1) epi(__nv_bfloat16 *out, int ldc, int t
     if (MODE == 3 && lane == 0) tma_store_wait_all();
     asm volatile("bar.sync 1, 256;" ::: "memory");
   }
-  if (threadIdx.x == 0) cyc[blockIdx.x] = clock64() - t0;
+  if (threadIdx.x == 0) { cyc[blockIdx.x] = clock64() - t0; stop = 1; }
+  }
   fence_before();
   __syncthreads();
-  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(256) : "memory");
+  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512) : "memory");
 }
 
 #include <cuda.h>
@@ -90,18 +115,20 @@ int main() {
   ((Enc)fn)(&om, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, out, dims, str, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
             CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   const int tiles = 200;
-  void (*ks[4])(__nv_bfloat16 *, int, int, long long *, CUtensorMap) = {epi<0>, epi<1>, epi<2>, epi<3>};
-  const char *names[4] = {"TMEM ld + bias + pack, no stores", "+ smem-transpose stores", "same with stores, no-TMEM math",
-                          "TMA (bulk tensor) stores"};
-  for (int m = 0; m < 4; ++m) {
-    ks[m]<<<148, 256>>>(out, ldc, tiles, d, om);
+  void (*ks[10])(__nv_bfloat16 *, int, int, long long *, CUtensorMap) = {epi<0, false>, epi<1, false>, epi<2, false>, epi<3, false>, epi<4, false>,
+                                                                       epi<0, true>, epi<1, true>, epi<2, true>, epi<3, true>, epi<4, true>};
+  const char *names[5] = {"TMEM ld + bias + pack, no stores", "+ smem-transpose stores", "same with stores, no-TMEM math",
+                          "TMA (bulk tensor) stores", "direct per-row st.global.v4 (no smem)"};
+  for (int m = 0; m < 10; ++m) {
+    if (m == 5) printf("-- with concurrent MMAs into the other TMEM half:\n");
+    ks[m]<<<148, 288>>>(out, ldc, tiles, d, om);
     cudaError_t e = cudaDeviceSynchronize();
     long long h[148];
     cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
     double mm = 0;
     for (int i = 0; i < 148; ++i) mm += h[i];
     mm /= 148;
-    printf("%-40s %8.0f cycles per 128x256 tile  (%s)\n", names[m], mm / tiles, cudaGetErrorString(e));
+    printf("%-40s %8.0f cycles per 128x256 tile  (%s)\n", names[m % 5], mm / tiles, cudaGetErrorString(e));
   }
   return 0;
 }
