@@ -14,6 +14,7 @@ import csv
 import io
 import json
 import os
+import re
 import subprocess
 import sys
 
@@ -46,7 +47,10 @@ def launches(path):
     hdr, data = rows[hi], rows[hi + 1:]
     ik, iv = hdr.index("Kernel Name"), hdr.index("Metric Value")
     per = collections.defaultdict(list)
+    ours = re.compile(r"\b(eng|ew|tc|simt)::")   # the library's kernels (not torch's input generation)
     for r in data:
+        if not ours.search(r[ik]):
+            continue
         per[r[ik].split("(")[0]].append(float(r[iv].replace(",", "")) / 1e3)   # ns -> us
     return per
 
