@@ -319,14 +319,14 @@ def main():
         torch.cuda.synchronize()
         barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        reps = 5
+        ar_reps = 5
         e0.record(stream)
-        for _ in range(reps):
+        for _ in range(ar_reps):
             for v in views:
                 dist.all_reduce(v)
         e1.record(stream)
         torch.cuda.synchronize()
-        ar_ms = max_over_ranks(e0.elapsed_time(e1) / reps)
+        ar_ms = max_over_ranks(e0.elapsed_time(e1) / ar_reps)
         g_off.close()
         g_off_in.close()
         stk_off.close()
