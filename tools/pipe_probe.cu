@@ -99,7 +99,7 @@ __device__ __forceinline__ uint32_t mapa(uint32_t a, uint32_t r) {
 template <bool kGlobalMaps>
 __global__ void __launch_bounds__(320, 1)
     probe2(const __grid_constant__ CUtensorMap mAp, const __grid_constant__ CUtensorMap mBp, const CUtensorMap *gmaps,
-           int nkb, int stages, int mt, int nt, long long *out, int poll_mode) {
+           int nkb, int stages, int mt, int nt, long long *out, int poll_mode, int kpass, int nmode) {
   const CUtensorMap &mA = kGlobalMaps ? gmaps[0] : mAp;
   const CUtensorMap &mB = kGlobalMaps ? gmaps[1] : mBp;
   if (kGlobalMaps && threadIdx.x == 0) {
@@ -133,7 +133,9 @@ __global__ void __launch_bounds__(320, 1)
   fence_after();
   const uint32_t tmem = tslot;
   const int pair = blockIdx.x >> 1;
-  const int m0 = (pair % mt) * 256 + 128 * rank, n0 = ((pair / mt) % nt) * 256 + 128 * rank;
+  const int m0 = (pair % mt) * 256 + 128 * rank;
+  const int n0 = (nmode ? pair % nt : (pair / mt) % nt) * 256 + 128 * rank;
+  const int kwrap = kpass > 0 ? kpass : nkb;   // k-blocks per pass over a K-range that fits L2
   const uint32_t Lfull = mapa(bars, 0);
   long long t0 = clock64();
   unsigned long long g0;
@@ -146,11 +148,11 @@ __global__ void __launch_bounds__(320, 1)
       if (blockIdx.x == 0 && kb < 16) out[200 + kb] = clock64() - t0;
       if (rank == 0) mbar_expect_tx(bars + 8 * s, 2 * STAGE);
       asm volatile("cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
-                   " [%0], [%1, {%3, %4}], [%2];" ::"r"(sa), "l"(&mA), "r"(fb), "r"(kb * 64), "r"(m0) : "memory");
+                   " [%0], [%1, {%3, %4}], [%2];" ::"r"(sa), "l"(&mA), "r"(fb), "r"((kb % kwrap) * 64), "r"(m0) : "memory");
       for (int c = 0; c < 2; ++c)
         asm volatile("cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes"
                      " [%0], [%1, {%3, %4}], [%2];" ::"r"(sb + 8192 * c), "l"(&mB), "r"(fb), "r"(n0 + 64 * c),
-                     "r"(kb * 64) : "memory");
+                     "r"((kb % kwrap) * 64) : "memory");
     }
   } else if (warp == 1 && lane == 0 && rank == 0) {
     const uint32_t ID = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(256 >> 3) << 17) |
@@ -264,8 +266,8 @@ int main() {
     at[0].val.clusterDim.z = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
-    if (variant != 1) cudaLaunchKernelEx(&cfg, probe2<false>, mA2, mBmn, (const CUtensorMap *)gm, nkb, stages, M / 256, N / 256, d, poll_mode);
-    else cudaLaunchKernelEx(&cfg, probe2<true>, mA2, mBmn, (const CUtensorMap *)gm, nkb, stages, M / 256, N / 256, d, poll_mode);
+    if (variant != 1) cudaLaunchKernelEx(&cfg, probe2<false>, mA2, mBmn, (const CUtensorMap *)gm, nkb, stages, M / 256, N / 256, d, poll_mode, 0, 0);
+    else cudaLaunchKernelEx(&cfg, probe2<true>, mA2, mBmn, (const CUtensorMap *)gm, nkb, stages, M / 256, N / 256, d, poll_mode, 0, 0);
     cudaError_t e = cudaDeviceSynchronize();
     long long h[148];
     cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
@@ -282,6 +284,53 @@ int main() {
     const char *vn[4] = {"params, no pollers", "global maps, no pollers", "params, 8 spinning waiters", "params, 8 sleeping waiters"};
     printf("pair  stages %d  %s : %7.1f cycles per k-block (ideal 512)  [%s]\n", stages, vn[variant], m / nkb,
            cudaGetErrorString(e));
+  }
+  // ---- L2 sharing experiment: 74 pairs, K = 1024 per pass (operands fit L2), 128 k-blocks
+  {
+    const int M2 = 74 * 256, N2 = 74 * 256, K2 = 1024;
+    void *A2, *B2;
+    cudaMalloc(&A2, (size_t)M2 * K2 * 2);
+    cudaMalloc(&B2, (size_t)K2 * N2 * 2);
+    cudaMemset(A2, 0, (size_t)M2 * K2 * 2);
+    cudaMemset(B2, 0, (size_t)K2 * N2 * 2);
+    CUtensorMap a2 = map2d(enc, A2, K2, M2, 64, 128);
+    CUtensorMap b2 = map2d(enc, B2, N2, K2, 64, 64);
+    struct Case { int mt, nt, nmode; const char *name; };
+    const Case cases[] = {{8, 8, 0, "A shared by ~9 pairs, B by ~9"},
+                          {25, 3, 0, "A shared by 3, B by 25 (engine hxh chain)"},
+                          {74, 1, 0, "A distinct, B shared by all"},
+                          {74, 74, 1, "A and B distinct per pair"},
+                          {1, 1, 0, "A and B shared by all 74"}};
+    const int stages = 6, nkb2 = 128;
+    const int smem = stages * 32768 + 16 * stages + 8 + 1024;
+    cudaFuncSetAttribute(probe2<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    for (const Case &c : cases) {
+      for (int rep = 0; rep < 2; ++rep) {
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(148, 1, 1);
+        cfg.blockDim = dim3(128, 1, 1);
+        cfg.dynamicSmemBytes = smem;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = 2;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        cudaLaunchKernelEx(&cfg, probe2<false>, a2, b2, (const CUtensorMap *)gm, nkb2, stages, c.mt, c.nt, d, 0, K2 / 64,
+                           c.nmode);
+        cudaError_t e = cudaDeviceSynchronize();
+        long long h[148];
+        cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
+        double m = 0, ns = 0;
+        for (int i = 0; i < 74; ++i) { m += h[i]; ns += h[74 + i]; }
+        m /= 74;
+        ns /= 74;
+        if (rep == 1)
+          printf("sharing: %-44s %7.1f cycles/kb  %.3f us/kb  -> %.1f TB/s into SMs  [%s]\n", c.name, m / nkb2,
+                 ns / 1e3 / nkb2, 74.0 * 65536 / (ns / nkb2) / 1e3, cudaGetErrorString(e));
+      }
+    }
   }
   return 0;
 }
