@@ -156,9 +156,9 @@ def time_cpu_oracle(cfg, sample_tokens: int):
 def cpu_sample_tokens(cfg, requested):
     if requested:
         return requested
-    # aim at ~10-30 s of fp64 work on a few host cores: ~2.5e11 FLOP
+    # aim at ~10-30 s of fp64 work on the host cores: ~8e11 FLOP (≈ 10 s measured on the B200 hosts)
     per_token = cfg.gemm_flops() / cfg.tokens
-    t = int(2.5e11 / per_token) // 8 * 8
+    t = int(8e11 / per_token) // 8 * 8
     return max(8, min(cfg.tokens, t))
 
 
