@@ -69,7 +69,7 @@ def build(force: bool = False, verbose: bool = True, trace: bool = False, varian
     """trace=True builds the debug variant lib/libooo_trace.so (-DOOO_TRACE:
     per-task timestamps in the engine, tools/engine_trace.py); `variant` +
     `defines` build tuning variants lib/libooo_<variant>.so."""
-    name = "libooo_trace.so" if trace else (f"libooo_{variant}.so" if variant else "libooo.so")
+    name = ("libooo_trace" if trace else "libooo") + (f"_{variant}" if variant else "") + ".so"
     lib = os.path.join(LIBDIR, name)
     objdir = OBJDIR + ("_trace" if trace else "") + (f"_{variant}" if variant else "")
     os.makedirs(LIBDIR, exist_ok=True)

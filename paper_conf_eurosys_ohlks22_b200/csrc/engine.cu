@@ -63,7 +63,7 @@ __device__ __forceinline__ void etrace2(int t, int slot) {
   if (g_etrace2 && t >= 0) g_etrace2[(size_t)t * 8 + slot] = clock64();
 }
 // pipeline globaltimer stamps [task][8] (third region): 4 accumulator free
-// (MMA may start), 5 last MMA issued, 6 first k-block load issued, 7 last
+// (MMA may start), 5 last MMA issued, 6 first k-block landed, 7 last landed
 __device__ unsigned long long *g_etrace3 = nullptr;
 __device__ __forceinline__ void etrace_gt(int t, int slot) {
   if (g_etrace3 && t >= 0) {
@@ -522,7 +522,10 @@ __global__ void __launch_bounds__(kThreads, 1)
         const bool a_mn = T.kind == EPI_WGRAD;
         const bool b_mn = T.kind != EPI_DGRAD;
         const int bh = T.bn / CG;                                 // this CTA's B columns
-        const uint32_t bytes = CG * (A_BYTES + bh * BK * 2);      // all CTAs, on the leader's barrier
+        // MN-major B arrives in whole 64-column boxes (a 96-column share of a
+        // 192-wide pair tile fetches 128 columns; the MMA reads the first 96)
+        const int bh_ld = b_mn ? (bh + 63) / 64 * 64 : bh;
+        const uint32_t bytes = CG * (A_BYTES + bh_ld * BK * 2);   // all CTAs, on the leader's barrier
         const int am = T.m0 + BM * (int)rank;
         const int bn0 = T.n0 + bh * (int)rank;
         int npre = 0;
@@ -588,6 +591,8 @@ __global__ void __launch_bounds__(kThreads, 1)
           ktrace(j, kb, 2);
           mbar_wait_b(bar_full + 8 * s, ph);
           ktrace(j, kb, 3);
+          if (kb == 0) etrace_gt(t, 6);           // first k-block landed
+          if (kb == T.nkb - 1) etrace_gt(t, 7);   // last k-block landed
           fence_after();
           const uint64_t soff = (uint64_t)(s * (C::STAGE >> 4));
           const uint64_t ad = a0 + soff, bd = b0 + soff;

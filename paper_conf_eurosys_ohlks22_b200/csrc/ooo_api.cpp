@@ -162,7 +162,7 @@ GemmPlan plan_tc_mn(int M, int N, int K, bool weight_grad) {
 int engine_bn(int N, bool chain, int cg, int row_tiles, int workers) {
   int forced = env_int(chain ? "OOO_EBN_CHAIN" : "OOO_EBN_DW", 0);
   if (!forced) forced = env_int("OOO_EBN", 0);
-  if (forced && N % forced == 0 && (cg == 1 || forced % 128 == 0)) return forced;
+  if (forced && N % forced == 0 && (cg == 1 || forced % 64 == 0) && (cg == 1 || forced >= 128)) return forced;
   // skinny token dimension (one CTA row): 64-wide chain tiles spread the
   // weight stream of F_i / dO_i over 4x more SMs (1-CTA tiles only)
   if (chain && cg == 1 && row_tiles * (N / 256) * 4 <= workers && N % 64 == 0) return 64;
