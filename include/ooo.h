@@ -101,7 +101,15 @@ typedef enum { OOO_ACT_IDENTITY = 0, OOO_ACT_RELU = 1, OOO_ACT_GELU_ERF = 2 } oo
  *   stream in D's order (critical ops high priority, sub-stream
  *   kernels serialise), all-reduces on the comm stream in D's dW order.
  *   k = 0 is dual-stream without reordering (the P:312 ablation). */
-typedef enum { OOO_SCHED_IN_ORDER = 0, OOO_SCHED_FIRST_K = 1 } ooo_sched_kind;
+/* OOO_SCHED_REGIONS: single-GPU multi-stream ooo computation (§4.1,
+ *   P:117-162): the critical ops (dO, then the next forward) form the
+ *   main-stream, split into regions; every dW_i (i >= 2) runs in the region
+ *   Algorithm 1 assigned it (multi-region joint scheduling, with
+ *   the memory-bounded pre-scheduling of P:162), dW_1 as soon as it is ready
+ *   (it gates F_1).  Needs a plan from ooo_plan_regions on the same stack
+ *   (OOO_ERR_STATE otherwise); k is ignored.  The backward order D is the
+ *   plan's (ooo_region_plan); the all-reduces follow D's dW order. */
+typedef enum { OOO_SCHED_IN_ORDER = 0, OOO_SCHED_FIRST_K = 1, OOO_SCHED_REGIONS = 2 } ooo_sched_kind;
 
 typedef struct {
   int32_t kind;   /* ooo_sched_kind */
@@ -159,6 +167,30 @@ ooo_status ooo_schedule_order(int32_t L, ooo_schedule sch, int32_t need_input_gr
  * mxm <= 0 -> L.  Byte counts are host arrays of length L. */
 int32_t ooo_max_k(int32_t L, int64_t m_fwd, const int64_t *m_dO, const int64_t *m_dW, int64_t mxm);
 
+/* Algorithm 1 "Multi-Region Joint Scheduling" (§4.1) and the
+ * memory-bounded pre-scheduling of P:162.  Pure host function.
+ *   n_regions N >= 1 main-stream regions R[0..N-1] in execution order,
+ *   t_main[N] = T_main(R[i]) (regions run back to back: start[i] = sum_{j<i}).
+ *   n_cands K >= 0 sub-stream kernels; row-major [K][N] tables t_sub =
+ *   T_sub(k, R[i]) and speedup = co-run speedup p of kernel k in R[i];
+ *   ready[K] = main-stream time at which kernel k's input is complete;
+ *   last_region[K] = last region k may run in (NULL: N-1);
+ *   nbytes[K] = bytes kernel k keeps alive while deferred (NULL: 0);
+ *   mxm = memory bound on the bytes held at region ends (<= 0: unlimited).
+ * Readings: runnable in R[i] = ready[k] <= start[i] + now[i] and
+ * i <= last_region[k]; ties -> first kernel / smallest region; when no open
+ * region has a runnable kernel the rest run as soon as ready (in the region
+ * in which they become ready); while the peak held bytes exceed mxm, one
+ * more leading region is pre-scheduled as soon as ready and Algorithm 1
+ * re-runs on the rest.
+ * Outputs (caller-owned host arrays): region_of[K]; order[K] = kernels in
+ * schedule order (region 0's list, then region 1's, ...); *k_pre = regions
+ * pre-scheduled.  OOO_ERR_INVALID_ARGUMENT on bad sizes / pointers / regions. */
+ooo_status ooo_region_schedule(int32_t n_regions, const double *t_main, int32_t n_cands, const double *t_sub,
+                               const double *speedup, const double *ready, const int32_t *last_region,
+                               const int64_t *nbytes, int64_t mxm, int32_t *region_of, int32_t *order,
+                               int32_t *k_pre);
+
 /* Extra bytes kept alive by deferring dW_1..dW_k (the memory cost of
  * deferral, §3; E8 at P:352-354): sum_{i=2..k} |dZ_i|. */
 int64_t ooo_deferral_bytes(const ooo_stack_desc *d, int32_t k);
@@ -197,6 +229,33 @@ ooo_status ooo_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void *dX
 
 /* `stream` waits for all outstanding backward work, all-reduces included. */
 ooo_status ooo_join(ooo_stack *s, void *stream);
+
+/* Plans OOO_SCHED_REGIONS (single-GPU multi-stream ooo, §4.1) for
+ * this stack, by the paper's steps 1-5:
+ *   1. profile on the GPU, for every region pair, the main-stream region
+ *      alone, each candidate dW_i alone and the two co-run (one engine
+ *      launch each, `reps` timed repetitions, the minimum kept); speedup =
+ *      (T_main + T_sub) / T_co-run;
+ *   2. main-stream = dO_L..dO_2 (dO_1 iff need_input_grad), then F_1..F_L of
+ *      the next iteration, in regions of `region_layers` consecutive layers;
+ *   3. candidates dW_2..dW_L (dW_1 gates F_1 and runs as soon as ready),
+ *      runnable once dO_{i+1} is done (interpolated by FLOPs inside its
+ *      region) and up to the region before F_{i-1} (which overwrites X_i);
+ *   4-5. Algorithm 1 with the memory bound desc.max_temp_bytes on the
+ *      deferred dZ_i bytes (ooo_region_schedule).
+ * Synchronous (host waits for the profiling launches; not capturable) and
+ * destructive: activations and gradients are overwritten, so an ooo_forward
+ * must run before the next ooo_backward (OOO_ERR_STATE otherwise).  bf16
+ * stacks only (OOO_ERR_UNSUPPORTED for fp32); region_layers >= 1, reps >= 1. */
+ooo_status ooo_plan_regions(ooo_stack *s, int32_t region_layers, int32_t reps, void *stream);
+
+/* The current region plan: *n_regions, *k_pre (pre-scheduled regions),
+ * region_of[L] (main-stream region of dW_i; that of dW_1 = the first
+ * forward region), ops[2L] / *n_ops = the backward order D it issues (+i dO_i,
+ * -i dW_i), t_main[n_regions] (profiled region times, ms; may be NULL).
+ * OOO_ERR_STATE without a plan. */
+ooo_status ooo_region_plan(const ooo_stack *s, int32_t *n_regions, int32_t *k_pre, int32_t *region_of,
+                           int32_t *ops, int32_t *n_ops, double *t_main, int32_t t_main_cap);
 
 /* Pre-compiled issue (§4.2): capture one training step
  * [ooo_backward(dY, sch, dX); ooo_forward(X, Y)] into an executable CUDA graph

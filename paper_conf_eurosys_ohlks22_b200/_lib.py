@@ -19,6 +19,7 @@ DTYPES = {"bf16": 0, "fp32": 1}
 ACTS = {"id": 0, "relu": 1, "gelu": 2}
 SCHED_IN_ORDER = 0
 SCHED_FIRST_K = 1
+SCHED_REGIONS = 2
 UNIQUE_ID_BYTES = 128
 
 
@@ -69,7 +70,7 @@ EXPORTS = [
     "ooo_schedule_order", "ooo_max_k", "ooo_deferral_bytes", "ooo_get_unique_id", "ooo_create_stack",
     "ooo_forward", "ooo_backward", "ooo_join", "ooo_graph_create", "ooo_graph_launch",
     "ooo_graph_destroy", "ooo_destroy", "ooo_tensor", "ooo_set_timing", "ooo_timing_read",
-    "ooo_engine_plan",
+    "ooo_engine_plan", "ooo_region_schedule", "ooo_plan_regions", "ooo_region_plan",
 ]
 
 _lib = None
@@ -108,6 +109,15 @@ def load() -> ctypes.CDLL:
     lib.ooo_engine_plan.restype = S
     lib.ooo_engine_plan.argtypes = [POINTER(StackDesc), Schedule, c_int32, c_int32, POINTER(c_int32), c_int32,
                                     POINTER(c_int32), POINTER(c_int32)]
+    lib.ooo_region_schedule.restype = S
+    lib.ooo_region_schedule.argtypes = [c_int32, POINTER(c_double), c_int32, POINTER(c_double), POINTER(c_double),
+                                        POINTER(c_double), POINTER(c_int32), POINTER(c_int64), c_int64,
+                                        POINTER(c_int32), POINTER(c_int32), POINTER(c_int32)]
+    lib.ooo_plan_regions.restype = S
+    lib.ooo_plan_regions.argtypes = [c_void_p, c_int32, c_int32, c_void_p]
+    lib.ooo_region_plan.restype = S
+    lib.ooo_region_plan.argtypes = [c_void_p, POINTER(c_int32), POINTER(c_int32), POINTER(c_int32),
+                                    POINTER(c_int32), POINTER(c_int32), POINTER(c_double), c_int32]
     lib.ooo_get_unique_id.restype = S
     lib.ooo_get_unique_id.argtypes = [c_void_p]
     lib.ooo_create_stack.restype = S
@@ -145,5 +155,6 @@ def check(status: int) -> None:
 
 def schedule(kind: str | int, k: int = 0) -> Schedule:
     if isinstance(kind, str):
-        kind = {"in_order": SCHED_IN_ORDER, "first_k": SCHED_FIRST_K, "ooo_first_k": SCHED_FIRST_K}[kind]
+        kind = {"in_order": SCHED_IN_ORDER, "first_k": SCHED_FIRST_K, "ooo_first_k": SCHED_FIRST_K,
+                "regions": SCHED_REGIONS}[kind]
     return Schedule(int(kind), int(k))

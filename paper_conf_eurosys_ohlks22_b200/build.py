@@ -24,7 +24,7 @@ LIB = os.path.join(LIBDIR, "libooo.so")
 OBJDIR = os.path.join(PKG, "build_obj")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-SOURCES = ["gemm_tc.cu", "engine.cu", "gemm_simt.cu", "ew.cu", "ooo_api.cpp", "nccl_dyn.cpp", "planner.cpp"]
+SOURCES = ["gemm_tc.cu", "engine.cu", "gemm_simt.cu", "ew.cu", "ooo_api.cpp", "nccl_dyn.cpp", "planner.cpp", "regions.cpp"]
 
 
 def _nvcc() -> str:

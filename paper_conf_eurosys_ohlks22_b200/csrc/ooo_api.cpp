@@ -419,6 +419,14 @@ struct ooo_stack {
   double eng_flops = 0;
   void *eng_dX = nullptr;
   bool eng_in_order = false;
+  // region plan (OOO_SCHED_REGIONS, §4.1; ooo_plan_regions)
+  bool has_regions = false;
+  std::vector<int> reg_D;          // backward order D of the plan
+  std::vector<int> reg_release;    // [L] release of dW_i: >= 0 index into the backward chain,
+                                   // <= -2: F_m of the next forward (m = -tag - 1)
+  std::vector<int> reg_region_of;  // [L] main-stream region of dW_i
+  std::vector<double> reg_tmain;   // profiled region times (ms)
+  int reg_kpre = 0;
 #ifdef OOO_TRACE
   std::vector<ooo::eng::Op> last_queue;       // debug: the most recent engine launch's ops
 #endif
@@ -751,12 +759,13 @@ ooo::eng::Op op_of_unit(const ooo_stack *s, const pl::Unit &u) {
 // reversed first-k dW_1..dW_k); the planner interleaves them (two priority
 // streams).  in_order (conventional backprop): one chain =
 // D, and the kernel adds the dW_{i+1} -> dO_i dependency.
-void engine_bwd_units(const ooo_stack *s, bool in_order, std::vector<pl::Unit> &crit,
+void engine_bwd_units(const ooo_stack *s, bool in_order, bool regions, std::vector<pl::Unit> &crit,
                       std::vector<pl::Unit> &defer, double &flops) {
   const Plan &p = s->p;
   for (int op : s->D) {
     const int i = op > 0 ? op : -op;
-    const pl::Unit u = unit_of(s, op > 0 ? pl::DGRAD : pl::WGRAD, i);
+    pl::Unit u = unit_of(s, op > 0 ? pl::DGRAD : pl::WGRAD, i);
+    if (regions && op < 0) u.release = s->reg_release[i - 1];   // Algorithm 1's region (§4.1)
     (op < 0 && !in_order ? defer : crit).push_back(u);
     flops += 2.0 * p.M * p.layer[i - 1].din * p.layer[i - 1].dout;
   }
@@ -819,7 +828,10 @@ ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const 
 ooo_status engine_flush(ooo_stack *s) {
   if (!s->eng_pending) return OOO_OK;
   s->eng_pending = false;
-  return engine_launch(s, s->eng_crit, s->eng_defer, nullptr, s->eng_dX, nullptr, s->eng_in_order, 0, 8,
+  std::vector<pl::Unit> defer = s->eng_defer;
+  for (pl::Unit &u : defer)
+    if (u.release <= -2) u.release = (int)s->eng_crit.size();   // its forward region: after the chain
+  return engine_launch(s, s->eng_crit, defer, nullptr, s->eng_dX, nullptr, s->eng_in_order, 0, 8,
                        s->eng_flops);
 }
 
@@ -842,7 +854,11 @@ ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st)
     const bool ar = comm_active(s);
     std::vector<pl::Unit> crit = s->eng_crit;
     crit.insert(crit.end(), fwd.begin(), fwd.end());
-    OOO_TRY(engine_launch(s, crit, s->eng_defer, Y, s->eng_dX, X, s->eng_in_order, ar ? 2 : 1, 9,
+    std::vector<pl::Unit> defer = s->eng_defer;
+    const int f1 = (int)(crit.size() - L);   // index of F_1 in the chain
+    for (pl::Unit &u : defer)
+      if (u.release <= -2) u.release = f1 + (-u.release - 1) - 1;   // region starting at F_m
+    OOO_TRY(engine_launch(s, crit, defer, Y, s->eng_dX, X, s->eng_in_order, ar ? 2 : 1, 9,
                           s->eng_flops + flops));
   } else {
     CU_TRY(cudaMemsetAsync(s->ctr, 0, (size_t)p.cl.fwd_end * 4, s->hi));
@@ -856,7 +872,8 @@ ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st)
 // Enqueues the counter reset, the seed and the comm stream's all-reduces; the
 // engine kernel itself is deferred to the next ooo_forward (fused step) or
 // ooo_join (backward alone).
-ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, void *dX, cudaStream_t st) {
+ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, bool regions, void *dX,
+                           cudaStream_t st) {
   const Plan &p = s->p;
   const int L = p.L;
   OOO_TRY(fork_from(s, st));
@@ -870,7 +887,7 @@ ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, void *dX
   s->eng_crit.clear();
   s->eng_defer.clear();
   s->eng_flops = 0;
-  engine_bwd_units(s, in_order, s->eng_crit, s->eng_defer, s->eng_flops);
+  engine_bwd_units(s, in_order, regions, s->eng_crit, s->eng_defer, s->eng_flops);
   s->eng_dX = dX;
   s->eng_in_order = in_order;
   s->eng_pending = true;
@@ -951,9 +968,15 @@ ooo_status enqueue_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void
     }
     k = std::min(k, mk);
   }
-  schedule_ops(L, sch.kind, k, s->d.need_input_grad != 0, s->D);
+  if (sch.kind == OOO_SCHED_REGIONS) {
+    if (!s->has_regions) return fail(OOO_ERR_STATE, "OOO_SCHED_REGIONS needs ooo_plan_regions first");
+    s->D = s->reg_D;
+  } else {
+    schedule_ops(L, sch.kind, k, s->d.need_input_grad != 0, s->D);
+  }
   if (s->timing) s->rec_cursor = 0;
-  if (s->p.engine) return engine_backward(s, dY, sch.kind == OOO_SCHED_IN_ORDER, dX, st);
+  if (s->p.engine)
+    return engine_backward(s, dY, sch.kind == OOO_SCHED_IN_ORDER, sch.kind == OOO_SCHED_REGIONS, dX, st);
   OOO_TRY(fork_from(s, st));
   const bool single = sch.kind == OOO_SCHED_IN_ORDER;
   cudaStream_t wst = single ? s->hi : s->lo;
@@ -985,6 +1008,185 @@ ooo_status enqueue_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void
   }
   s->have_fwd = false;
   s->bwd_pending = true;
+  return OOO_OK;
+}
+
+
+// ---- region planning (OOO_SCHED_REGIONS, §4.1) ---------------
+int fwd_nt_of(const Plan &p, int i) { return (p.layer[i - 1].dout + p.layer[i - 1].ebn_fwd - 1) / p.layer[i - 1].ebn_fwd; }
+int dx_nt_of(const Plan &p, int i) { return (p.layer[i - 1].din + p.layer[i - 1].ebn_dx - 1) / p.layer[i - 1].ebn_dx; }
+int dw_tiles_of(const Plan &p, int i) {
+  const LayerPlan &lp = p.layer[i - 1];
+  return ((lp.din + 127) / 128) * ((lp.dout + lp.ebn_dw - 1) / lp.ebn_dw);
+}
+
+// One profiling launch of the engine on the given ops alone: the completion
+// counters of every op NOT in the launch are preset to "complete", so the
+// launched ops wait only for each other (step 1 of §4.1).  Minimum
+// device time over `reps` timed launches after one warm-up (ms).
+ooo_status profile_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const std::vector<pl::Unit> &defer,
+                          int reps, double *ms) {
+  const Plan &p = s->p;
+  const ooo::eng::CounterLayout &cl = p.cl;
+  auto in = [&](int kind, int i) {
+    for (const pl::Unit &u : crit)
+      if (u.kind == kind && u.layer == i) return true;
+    for (const pl::Unit &u : defer)
+      if (u.kind == kind && u.layer == i) return true;
+    return false;
+  };
+  std::vector<int32_t> img(cl.total, 0);
+  for (int i = 1; i <= p.L; ++i) {
+    if (!in(pl::FWD, i))
+      for (int m = 0; m < cl.MT; ++m) img[cl.fwd_rows + (i - 1) * cl.MT + m] = fwd_nt_of(p, i);
+    if (i >= 2 && !in(pl::DGRAD, i)) {
+      for (int m = 0; m < cl.MT; ++m) img[cl.dz_rows + (i - 2) * cl.MT + m] = dx_nt_of(p, i);
+      img[cl.dz_total + i - 2] = cl.MT * dx_nt_of(p, i);
+    }
+    if (!in(pl::WGRAD, i)) img[cl.dw_done + i - 1] = dw_tiles_of(p, i);
+  }
+  const int copy_nt = (s->dims[0] + copy_bn(s->dims[0]) - 1) / copy_bn(s->dims[0]);
+  for (int m = 0; m < cl.MT; ++m) img[cl.xcopy + m] = copy_nt;
+  void *Y = s->lr[p.L - 1].dZ;                                  // scratch M x d_L target for F_L
+  void *dX = s->d.need_input_grad ? s->lr[0].X : nullptr;      // scratch M x d_0 target for dO_1
+  cudaEvent_t e0, e1;
+  CU_TRY(cudaEventCreate(&e0));
+  CU_TRY(cudaEventCreate(&e1));
+  double best = 1e30;
+  ooo_status st = OOO_OK;
+  for (int r = 0; r <= reps && st == OOO_OK; ++r) {
+    cudaError_t ce = cudaMemcpyAsync(s->ctr, img.data(), img.size() * 4, cudaMemcpyHostToDevice, s->hi);
+    if (ce == cudaSuccess) ce = cudaEventRecord(e0, s->hi);
+    if (ce != cudaSuccess) {
+      st = fail(OOO_ERR_CUDA, "profile launch: %s", cudaGetErrorString(ce));
+      break;
+    }
+    st = engine_launch(s, crit, defer, Y, dX, nullptr, false, 0, 10, 0.0);
+    if (st != OOO_OK) break;
+    ce = cudaEventRecord(e1, s->hi);
+    if (ce == cudaSuccess) ce = cudaEventSynchronize(e1);
+    float t = 0.f;
+    if (ce == cudaSuccess) ce = cudaEventElapsedTime(&t, e0, e1);
+    if (ce != cudaSuccess) st = fail(OOO_ERR_CUDA, "profile launch: %s", cudaGetErrorString(ce));
+    else if (r > 0) best = std::min(best, (double)t);
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  *ms = best;
+  return st;
+}
+
+ooo_status plan_regions(ooo_stack *s, int rl, int reps) {
+  const Plan &p = s->p;
+  const int L = p.L;
+  const bool need_dx = s->d.need_input_grad != 0;
+  // step 2: main-stream regions (backward dO blocks from the top, then forward F blocks)
+  struct Region { std::vector<pl::Unit> ops; std::vector<double> flops; std::vector<int> layers; bool fwd; };
+  std::vector<Region> R;
+  for (int hi = L; hi >= 1; hi -= rl) {
+    Region g;
+    g.fwd = false;
+    for (int i = hi; i > std::max(0, hi - rl); --i) {
+      if (i == 1 && !need_dx) continue;
+      g.ops.push_back(unit_of(s, pl::DGRAD, i));
+      g.flops.push_back(2.0 * p.M * p.layer[i - 1].din * p.layer[i - 1].dout);
+      g.layers.push_back(i);
+    }
+    if (!g.ops.empty()) R.push_back(g);
+  }
+  const int nb = (int)R.size();
+  std::vector<int> fwd_region(L + 1, 0);
+  for (int lo = 1; lo <= L; lo += rl) {
+    Region g;
+    g.fwd = true;
+    for (int i = lo; i <= std::min(L, lo + rl - 1); ++i) {
+      g.ops.push_back(unit_of(s, pl::FWD, i));
+      g.flops.push_back(2.0 * p.M * p.layer[i - 1].din * p.layer[i - 1].dout);
+      g.layers.push_back(i);
+      fwd_region[i] = (int)R.size();
+    }
+    R.push_back(g);
+  }
+  const int N = (int)R.size();
+  // step 1: profile -- regions alone, candidates alone, co-runs
+  std::vector<double> t_main(N), start(N);
+  for (int r = 0; r < N; ++r) OOO_TRY(profile_launch(s, R[r].ops, {}, reps, &t_main[r]));
+  double acc = 0;
+  for (int r = 0; r < N; ++r) {
+    start[r] = acc;
+    acc += t_main[r];
+  }
+  // candidates dW_2..dW_L (c = L - i: the paper's U in descending layer order)
+  const int K = L - 1;
+  std::vector<double> ready(K), t_alone(K), t_sub((size_t)K * N), sp((size_t)K * N, 0.0);
+  std::vector<int32_t> last(K);
+  std::vector<int64_t> nbytes(K);
+  for (int c = 0; c < K; ++c) {
+    const int i = L - c;
+    // runnable once dO_{i+1} is done: its completion inside its region, by FLOPs
+    ready[c] = 0.0;
+    if (i < L) {
+      for (int r = 0; r < nb; ++r) {
+        double f = 0, tot = 0;
+        bool here = false;
+        for (size_t j = 0; j < R[r].layers.size(); ++j) {
+          tot += R[r].flops[j];
+          if (!here) f += R[r].flops[j];
+          if (R[r].layers[j] == i + 1) here = true;
+        }
+        if (here) ready[c] = start[r] + t_main[r] * (tot > 0 ? f / tot : 1.0);
+      }
+    }
+    last[c] = std::max(0, fwd_region[i - 1] - 1);   // before F_{i-1} (WAR on X_i) and F_i
+    nbytes[c] = (int64_t)p.M * p.layer[i - 1].dout * p.elt;   // dZ_i kept alive (§3)
+    OOO_TRY(profile_launch(s, {}, {unit_of(s, pl::WGRAD, i)}, reps, &t_alone[c]));
+  }
+  for (int c = 0; c < K; ++c) {
+    const int i = L - c;
+    for (int r = 0; r < N; ++r) {
+      t_sub[(size_t)c * N + r] = t_alone[c];   // reading A6: T_sub(k, R) = k's profiled time
+      if (start[r] + t_main[r] <= ready[c] || r > last[c]) continue;   // never runnable there
+      double tc = 0;
+      OOO_TRY(profile_launch(s, R[r].ops, {unit_of(s, pl::WGRAD, i)}, reps, &tc));
+      sp[(size_t)c * N + r] = (t_main[r] + t_alone[c]) / tc;
+    }
+  }
+  // steps 3-5: Algorithm 1 (+ P:162 memory bound)
+  std::vector<int32_t> region_of(std::max(K, 1)), order(std::max(K, 1));
+  int32_t kpre = 0;
+  OOO_TRY(ooo_region_schedule(N, t_main.data(), K, t_sub.data(), sp.data(), ready.data(), last.data(),
+                              nbytes.data(), s->d.max_temp_bytes, region_of.data(), order.data(), &kpre));
+  // the plan: D = per backward region its dO ops then its dW ops, then dW_1
+  // and the forward regions' dW ops; release tags for the engine queue
+  std::vector<std::vector<int>> S(N);
+  for (int j = 0; j < K; ++j) S[region_of[order[j]]].push_back(L - order[j]);
+  s->reg_D.clear();
+  s->reg_release.assign(L, -1);
+  s->reg_region_of.assign(L, nb);
+  int ci = 0;   // backward chain index
+  for (int r = 0; r < nb; ++r) {
+    const int first = ci;
+    for (int i : R[r].layers) {
+      s->reg_D.push_back(+i);
+      ++ci;
+    }
+    for (int i : S[r]) {
+      s->reg_D.push_back(-i);
+      s->reg_release[i - 1] = first;
+      s->reg_region_of[i - 1] = r;
+    }
+  }
+  s->reg_D.push_back(-1);                    // dW_1 gates F_1: as soon as ready (reading A4)
+  s->reg_release[0] = ci;                    // after the last dO (the chain end if no forward follows)
+  for (int r = nb; r < N; ++r)
+    for (int i : S[r]) {
+      s->reg_D.push_back(-i);
+      s->reg_release[i - 1] = -(1 + R[r].layers[0]);   // region starting at F_m
+      s->reg_region_of[i - 1] = r;
+    }
+  s->reg_tmain = t_main;
+  s->reg_kpre = kpre;
+  s->has_regions = true;
   return OOO_OK;
 }
 
@@ -1080,7 +1282,7 @@ ooo_status ooo_engine_plan(const ooo_stack_desc *d, ooo_schedule sch, int32_t fu
   schedule_ops(tmp.p.L, sch.kind, sch.k, d->need_input_grad != 0, tmp.D);
   std::vector<pl::Unit> crit, defer;
   double flops = 0;
-  engine_bwd_units(&tmp, in_order, crit, defer, flops);
+  engine_bwd_units(&tmp, in_order, false, crit, defer, flops);
   if (fused) {
     crit.push_back(unit_of(&tmp, pl::COPY, 1));
     for (int i = 1; i <= tmp.p.L; ++i) crit.push_back(unit_of(&tmp, pl::FWD, i));
@@ -1293,7 +1495,7 @@ ooo_status ooo_forward(ooo_stack *s, const void *X, void *Y, void *stream) {
 
 ooo_status ooo_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void *dX, void *stream) {
   if (!s || !dY) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
-  if (sch.kind != OOO_SCHED_IN_ORDER && sch.kind != OOO_SCHED_FIRST_K)
+  if (sch.kind != OOO_SCHED_IN_ORDER && sch.kind != OOO_SCHED_FIRST_K && sch.kind != OOO_SCHED_REGIONS)
     return fail(OOO_ERR_INVALID_ARGUMENT, "schedule kind %d invalid", sch.kind);
   if (sch.k < 0) return fail(OOO_ERR_INVALID_ARGUMENT, "k must be >= 0");
   if (s->d.need_input_grad && !dX) return fail(OOO_ERR_INVALID_ARGUMENT, "need_input_grad set but dX NULL");
@@ -1315,7 +1517,7 @@ ooo_status ooo_graph_create(ooo_stack *s, const void *X, void *Y, const void *dY
   if (!s || !X || !Y || !dY || !out) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
   *out = nullptr;
   if (!s->have_fwd) return fail(OOO_ERR_STATE, "ooo_graph_create needs a preceding ooo_forward");
-  if (sch.kind != OOO_SCHED_IN_ORDER && sch.kind != OOO_SCHED_FIRST_K)
+  if (sch.kind != OOO_SCHED_IN_ORDER && sch.kind != OOO_SCHED_FIRST_K && sch.kind != OOO_SCHED_REGIONS)
     return fail(OOO_ERR_INVALID_ARGUMENT, "schedule kind %d invalid", sch.kind);
   if (sch.k < 0) return fail(OOO_ERR_INVALID_ARGUMENT, "k must be >= 0");
   if (s->d.need_input_grad && !dX) return fail(OOO_ERR_INVALID_ARGUMENT, "need_input_grad set but dX NULL");
@@ -1428,6 +1630,44 @@ ooo_status ooo_timing_read(ooo_stack *s, ooo_launch_record *out, int32_t cap, in
     ++cnt;
   }
   *n = cnt;
+  return OOO_OK;
+}
+
+
+ooo_status ooo_plan_regions(ooo_stack *s, int32_t region_layers, int32_t reps, void *stream) {
+  if (!s) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL stack");
+  if (region_layers < 1 || reps < 1) return fail(OOO_ERR_INVALID_ARGUMENT, "region_layers and reps must be >= 1");
+  if (!s->p.engine) return fail(OOO_ERR_UNSUPPORTED, "region planning profiles the bf16 engine (fp32 stack)");
+  if (s->p.L < 2) return fail(OOO_ERR_UNSUPPORTED, "region planning needs L >= 2");
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  OOO_TRY(engine_flush(s));
+  OOO_TRY(join_into(s, st));
+  CU_TRY(cudaStreamSynchronize(st));
+  CU_TRY(cudaStreamSynchronize(s->hi));
+  const bool timing = s->timing;
+  s->timing = false;
+  ooo_status r = plan_regions(s, region_layers, reps);
+  s->timing = timing;
+  s->have_fwd = false;       // activations / gradients were overwritten by the profiling launches
+  s->bwd_pending = false;
+  OOO_TRY(r);
+  CU_TRY(cudaStreamSynchronize(s->hi));
+  return check_async(s);
+}
+
+ooo_status ooo_region_plan(const ooo_stack *s, int32_t *n_regions, int32_t *k_pre, int32_t *region_of,
+                           int32_t *ops, int32_t *n_ops, double *t_main, int32_t t_main_cap) {
+  if (!s) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL stack");
+  if (!s->has_regions) return fail(OOO_ERR_STATE, "no region plan (ooo_plan_regions)");
+  if (n_regions) *n_regions = (int32_t)s->reg_tmain.size();
+  if (k_pre) *k_pre = s->reg_kpre;
+  if (region_of)
+    for (int i = 0; i < s->p.L; ++i) region_of[i] = s->reg_region_of[i];
+  if (ops)
+    for (size_t j = 0; j < s->reg_D.size(); ++j) ops[j] = s->reg_D[j];
+  if (n_ops) *n_ops = (int32_t)s->reg_D.size();
+  if (t_main)
+    for (int i = 0; i < std::min<int>(t_main_cap, (int)s->reg_tmain.size()); ++i) t_main[i] = s->reg_tmain[i];
   return OOO_OK;
 }
 

@@ -223,7 +223,9 @@ std::vector<Unit> plan_once(const Problem &pb, const Model &m, int group_rows) {
     }
   std::vector<Unit> crit;  // row-local critical ops split into rows
   std::vector<int> width;  // tiles of the whole op each critical unit belongs to
-  for (const Unit &u : pb.crit) {
+  std::vector<int> whole;  // index of that op in pb.crit
+  for (size_t o = 0; o < pb.crit.size(); ++o) {
+    const Unit &u = pb.crit[o];
     const bool rowwise = u.kind != WGRAD;
     for (int r = 0; r < u.mt; r += rowwise ? 1 : u.mt) {
       Unit g = u;
@@ -231,15 +233,24 @@ std::vector<Unit> plan_once(const Problem &pb, const Model &m, int group_rows) {
       g.mt = rowwise ? 1 : u.mt;
       crit.push_back(g);
       width.push_back(u.mt * u.nt);
+      whole.push_back((int)o);
     }
   }
+  // region release (§4.1): has critical op #rel started?
+  auto released = [&](const Unit &d, size_t ci) {
+    if (d.release < 0 || ci >= crit.size()) return true;
+    const int started = ci == 0 ? 0 : whole[ci - 1] + 1;   // ops whose first row was emitted
+    return started > d.release;
+  };
   const int P = std::max(1, pb.workers);
   std::vector<Unit> out;
   size_t ci = 0, di = 0;
   while (ci < crit.size() || di < def.size()) {
     const bool c_ok = ci < crit.size() && sim.emittable(crit[ci]);
-    const bool d_ok = di < def.size() && sim.emittable(def[di]);
-    if (!c_ok && !d_ok) return {};   // dependency cycle: cannot happen for valid inputs
+    const bool d_dep = di < def.size() && sim.emittable(def[di]);
+    if (!c_ok && !d_dep) return {};   // dependency cycle: cannot happen for valid inputs
+    // a release constraint never blocks the only unit that can proceed
+    const bool d_ok = d_dep && (released(def[di], ci) || !c_ok);
     bool take_c = c_ok;
     if (c_ok && d_ok) {
       const double t = sim.time_free(1, nullptr, 0.0);

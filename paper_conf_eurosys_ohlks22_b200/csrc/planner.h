@@ -29,6 +29,9 @@ struct Unit {
   int nkb;           // k-blocks per tile (0 for COPY)
   int bn;            // tile width
   int act;           // epilogue activation (0 = identity)
+  int release = -1;  // deferred units: emitted only once critical op #release (index into
+                     // Problem::crit) has started (region schedule, §4.1); -1 = no constraint,
+                     // >= crit.size() = after the whole chain
 };
 
 struct Model {

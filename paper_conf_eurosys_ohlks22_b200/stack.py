@@ -95,6 +95,27 @@ def engine_plan(dims, acts, tokens, kind="first_k", k=0, fused=True, workers=0, 
     return ops, bool(topo.value)
 
 
+def region_schedule(t_main, t_sub, speedup, ready, last_region=None, nbytes=None, mxm=0):
+    """Algorithm 1 (§4.1) + the P:162 memory bound, computed by the
+    library (``ooo_region_schedule``).  t_sub / speedup are [K][N] nested
+    lists.  Returns (S, k_pre): S[i] = candidate indices of region i in
+    schedule order."""
+    N, K = len(t_main), len(ready)
+    dbl = lambda v: (ctypes.c_double * max(1, len(v)))(*v)  # noqa: E731
+    flat = lambda m: [float(x) for row in m for x in row]  # noqa: E731
+    reg = (c_int32 * max(1, K))()
+    order = (c_int32 * max(1, K))()
+    kp = c_int32()
+    last = _i32arr(last_region) if last_region is not None else None
+    nb = (ctypes.c_int64 * max(1, K))(*nbytes) if nbytes is not None else None
+    check(load().ooo_region_schedule(int(N), dbl(t_main), int(K), dbl(flat(t_sub)), dbl(flat(speedup)),
+                                     dbl(ready), last, nb, int(mxm), reg, order, ctypes.byref(kp)))
+    S = [[] for _ in range(N)]
+    for j in range(K):
+        S[reg[order[j]]].append(order[j])
+    return S, kp.value
+
+
 def get_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(_lib.UNIQUE_ID_BYTES)
     check(load().ooo_get_unique_id(buf))
@@ -234,6 +255,25 @@ class OooStack:
                                       c_void_p(dY.data_ptr()), _lib.schedule(kind, k),
                                       c_void_p(dX.data_ptr() if dX is not None else None), ctypes.byref(h)))
         return StepGraph(self, h, (X, Y, dY, dX))
+
+    def plan_regions(self, region_layers: int = 6, reps: int = 1, stream=None) -> dict:
+        """Profile co-run speedups and plan OOO_SCHED_REGIONS (single-GPU
+        multi-stream ooo, §4.1, Algorithm 1).  Overwrites activations and
+        gradients: run forward() again before the next backward."""
+        check(load().ooo_plan_regions(self._h, int(region_layers), int(reps), _stream_handle(stream)))
+        return self.region_plan()
+
+    def region_plan(self) -> dict:
+        L = len(self.acts)
+        n, kp, nops = c_int32(), c_int32(), c_int32()
+        reg = (c_int32 * L)()
+        ops = (c_int32 * (2 * L))()
+        check(load().ooo_region_plan(self._h, ctypes.byref(n), ctypes.byref(kp), reg, ops, ctypes.byref(nops),
+                                     None, 0))
+        tm = (ctypes.c_double * max(1, n.value))()
+        check(load().ooo_region_plan(self._h, None, None, None, None, None, tm, n.value))
+        return {"n_regions": n.value, "k_pre": kp.value, "region_of": list(reg), "D": list(ops[: nops.value]),
+                "t_main_ms": list(tm[: n.value])}
 
     # ---- introspection -----------------------------------------------------
     def tensor(self, kind: str, layer: int):

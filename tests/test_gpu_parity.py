@@ -215,3 +215,88 @@ def test_bf16_fused_step_comm_gated(monkeypatch):
                     "db": [to_np(v) for v in gated.db], "dX": None}, cases[2].oracle(2)), BF16_TOL)
     gated.close()
     plain.close()
+
+
+# ------------------- single-GPU multi-stream ooo: Algorithm 1 regions (§4.1)
+def _region_plan_valid(stk, L, need_dx=False):
+    from oracle import schedule as S
+    plan = stk.region_plan()
+    D = plan["D"]
+    assert S.is_valid_order(D, L, need_dx), D          # a topological order of the backward
+    assert sorted(-op for op in D if op < 0) == list(range(1, L + 1))
+    return plan
+
+
+@pytest.mark.parametrize("tokens,rl,need_dx", [(384, 2, False), (264, 1, True), (136, 3, False)])
+def test_bf16_regions_schedule_bit_exact(tokens, rl, need_dx):
+    """OOO_SCHED_REGIONS (dW kernels placed by Algorithm 1 from profiled
+    co-run speedups) gives the gradients of in_order bit for bit and the
+    oracle's within the bf16 gate; eager and graph-captured alike."""
+    case = Case([256, 512, 256, 1024, 256, 256, 512], ["id", "gelu", "gelu", "id", "gelu", "id"], tokens, "bf16",
+                need_dx=need_dx)
+    stk = case.stack(bucket_layers=2)
+    stk.forward(to_dev(case.X, "bf16"))
+    plan = stk.plan_regions(region_layers=rl, reps=1)
+    _region_plan_valid(stk, case.L, need_dx)
+    assert plan["n_regions"] >= 2 and all(t > 0 for t in plan["t_main_ms"])
+    base = case.run(stk, "in_order", 0)
+    out = case.run(stk, "regions", 0)
+    assert torch.equal(out["raw"], base["raw"])
+    if need_dx:
+        assert np.array_equal(out["dX"], base["dX"])
+    g = case.run(stk, "regions", 0, graph=True, launches=2)
+    assert torch.equal(g["raw"], base["raw"])
+    _check(max_err(out, case.oracle()), BF16_TOL)
+    stk.close()
+
+
+def test_bf16_regions_fused_step_and_memory_bound():
+    """Regions across fused steps (backward(t) + forward(t+1) in one launch,
+    deferred dW in forward regions) and the P:162 memory bound (max_temp_bytes
+    below any deferral: the plan pre-schedules until nothing is held)."""
+    dims, acts = [256, 512, 256, 256, 512, 256, 256], ["gelu", "id", "id", "gelu", "id", "id"]
+    cases = [Case(dims, acts, 400, "bf16", step=t) for t in range(3)]
+    a = cases[0].stack()
+    b = cases[0].stack()
+    Xs = [to_dev(c.X, "bf16") for c in cases]
+    dYs = [to_dev(c.dY, "bf16") for c in cases]
+    a.forward(Xs[0])
+    a.plan_regions(region_layers=2)
+    Ya, Yb = a.forward(Xs[0]), b.forward(Xs[0])
+    for t in range(3):
+        a.backward(dYs[t], "regions")
+        b.backward(dYs[t], "in_order")
+        if t < 2:
+            Ya, Yb = a.forward(Xs[t + 1]), b.forward(Xs[t + 1])
+        else:
+            a.join()
+            b.join()
+        torch.cuda.synchronize()
+        assert torch.equal(Ya, Yb), t
+        assert torch.equal(a.grads_buf, b.grads_buf), t
+    a.close()
+    b.close()
+    tight = cases[0].stack(max_temp_bytes=1)
+    tight.forward(Xs[0])
+    plan = tight.plan_regions(region_layers=1)
+    assert 0 <= plan["k_pre"] <= plan["n_regions"]
+    _region_plan_valid(tight, len(acts))
+    out = cases[0].run(tight, "regions", 0)
+    _check(max_err(out, cases[0].oracle()), BF16_TOL)
+    tight.close()
+
+
+def test_bf16_regions_full_size_block_slice():
+    """Two BERT-base blocks at full width and 4096 tokens, one region per
+    block (the paper's per-block regions)."""
+    dims, acts, M = _block_slice(configs.C2, 2)
+    case = Case(dims, acts, M, "bf16")
+    stk = case.stack()
+    stk.forward(to_dev(case.X, "bf16"))
+    stk.plan_regions(region_layers=6)
+    _region_plan_valid(stk, case.L)
+    out = case.run(stk, "regions", 0, graph=True)
+    base = case.run(stk, "in_order", 0)
+    assert torch.equal(out["raw"], base["raw"])
+    _check(max_err(out, case.oracle()), BF16_TOL)
+    stk.close()
