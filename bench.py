@@ -45,6 +45,9 @@ def parse():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="C2", help="C1..C5 or a config name (default: configs[1] = BERT-base stack)")
     ap.add_argument("--k", default="auto", help="reverse first-k parameter, or 'auto' (paper's search, P:212-214)")
+    ap.add_argument("--regions", type=int, default=6,
+                    help="N = 1: also plan the single-GPU multi-stream schedule (Algorithm 1, §4.1) with regions of "
+                         "this many layers and time the better of it and reverse first-k; 0 = off")
     ap.add_argument("--bucket-layers", type=int, default=1)
     ap.add_argument("--nccl-max-ctas", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
@@ -256,10 +259,10 @@ def main():
     torch.cuda.synchronize()
     graphs = {}
 
-    def s_graph(Xb, Yb, dYb, k):
+    def s_graph(Xb, Yb, dYb, sch):
         stk.forward(Xb, Yb)          # the graph's backward needs a forward on these buffers
         torch.cuda.synchronize()
-        return stk.graph(Xb, Yb, dYb, "first_k", k)
+        return stk.graph(Xb, Yb, dYb, *sch)
 
     def graph_for(kind, k, s=stk):
         key = (id(s), kind, k)
@@ -281,7 +284,29 @@ def main():
         k_best, visited = search_k(L, tput)
     else:
         k_best, visited = int(args.k), []
-    g_ooo = graph_for("first_k", k_best)
+    g_fk = graph_for("first_k", k_best)
+    sched = ("first_k", k_best)
+    # ---- N = 1: the paper's single-GPU method -- multi-stream ooo with
+    # Algorithm 1 regions (§4.1), planned from profiled co-run
+    # speedups; the better of it and reverse first-k is the measured schedule
+    regions = None
+    if world == 1 and args.regions > 0:
+        t0 = time.time()
+        plan = stk.plan_regions(region_layers=args.regions, reps=1)
+        t_plan = time.time() - t0
+        stk.forward(X, Y)
+        torch.cuda.synchronize()
+        g_reg = graph_for("regions", 0)
+        probe = max(10, min(30, args.steps))
+        for _ in range(3):
+            g_reg.launch(stream)
+            g_fk.launch(stream)
+        ms_r, ms_f = timed(g_reg, probe), timed(g_fk, probe)
+        regions = {"region_layers": args.regions, "n_regions": plan["n_regions"], "k_pre": plan["k_pre"],
+                   "plan_seconds": t_plan, "probe_ms_per_step": ms_r, "first_k_probe_ms_per_step": ms_f}
+        if ms_r < ms_f:
+            sched = ("regions", 0)
+    g_ooo = graph_for(*sched)
     g_in = graph_for("in_order", 0)
     for _ in range(max(3, args.warmup)):
         g_ooo.launch(stream)
@@ -292,6 +317,9 @@ def main():
     ms_ooo = timed(g_ooo, args.steps, sampler)
     clocks = sampler.summary()
     ms_in = timed(g_in, args.steps)
+    ms_fk = ms_ooo if sched[0] == "first_k" else timed(g_fk, args.steps)
+    if regions is not None:
+        regions["ms_per_step"] = ms_ooo if sched[0] == "regions" else timed(graph_for("regions", 0), args.steps)
     # repeat runs (mean +- standard error) and the dual-stream
     # control ooo_first_k(0) (no reordering)
     reps = [timed(g_ooo, args.steps) for _ in range(args.runs)]
@@ -338,7 +366,7 @@ def main():
 
     # ---- per-kernel durations: instrumented replay of the same step (CUDA events per launch)
     stk.set_timing(True)
-    g_t = stk.graph(X, Y, dY, "first_k", k_best)
+    g_t = stk.graph(X, Y, dY, *sched)
     for _ in range(3):
         g_t.launch(stream)
     ms_timed = timed(g_t, max(3, args.steps // 2))
@@ -399,7 +427,7 @@ def main():
         sets = []
         for p in range(2):
             Xp, dYp, Yp = (X, dY, Y) if p == 0 else (torch.empty_like(X), torch.empty_like(dY), torch.empty_like(Y))
-            g = g_ooo if p == 0 else s_graph(Xp, Yp, dYp, k_best)
+            g = g_ooo if p == 0 else s_graph(Xp, Yp, dYp, sched)
             hX = torch.empty(X.shape, dtype=X.dtype, pin_memory=True)
             hdY = torch.empty(dY.shape, dtype=dY.dtype, pin_memory=True)
             hY = torch.empty(Y.shape, dtype=Y.dtype, pin_memory=True)
@@ -461,7 +489,9 @@ def main():
         "vs_baseline": None, "dtype": dt, "data": "synthetic",
         "config": {"workload": f"{cfg.name} ({cfg.note})", "layers": L, "tokens_per_gpu": M,
                    "global_batch_tokens": M * world, "dims": f"{cfg.dims[0]}/{max(cfg.dims)}",
-                   "schedule": "ooo_first_k", "k": k_best, "k_search_visited": visited,
+                   "schedule": (f"regions(Algorithm 1, {args.regions} layers per region)" if sched[0] == "regions"
+                                else "ooo_first_k"),
+                   "k": k_best, "k_search_visited": visited,
                    "bucket_layers": args.bucket_layers, "parallelism": f"dp{world}",
                    "l2": "working set (weights+activations+grads) >> 126 MB L2; no flush"},
         "tokens_per_s": value * M * world,
@@ -473,6 +503,8 @@ def main():
         "runs": {"n": len(reps), "mean_ms": statistics.mean(reps) if reps else None,
                  "sem_ms": (statistics.stdev(reps) / math.sqrt(len(reps))) if len(reps) > 1 else None},
         "ooo_first_k0": {"value": 1e3 / ms_k0, "ms_per_step": ms_k0},
+        "ooo_first_k": {"k": k_best, "value": 1e3 / ms_fk, "ms_per_step": ms_fk},
+        "regions": regions,
         "step_roofline": {"ms": step_roof_ms, "frac": step_roof_ms / ms_ooo if step_roof_ms else None,
                           "tensor_ms": t_tensor, "allreduce_ms_at_770GBps": t_ar, "gemm_flops": flops,
                           "hbm_min_bytes": hbm_bytes, "hbm_ms": t_hbm,
