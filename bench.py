@@ -290,7 +290,7 @@ def main():
     # Algorithm 1 regions (§4.1), planned from profiled co-run
     # speedups; the better of it and reverse first-k is the measured schedule
     regions = None
-    if world == 1 and args.regions > 0:
+    if world == 1 and args.regions > 0 and dt == "bf16":    # profiles the bf16 engine
         t0 = time.time()
         plan = stk.plan_regions(region_layers=args.regions, reps=1)
         t_plan = time.time() - t0

@@ -93,6 +93,14 @@ constexpr int kThreads = 64 + kEpiThreads;
 constexpr int kMaxBN = 256;
 constexpr int STG_BYTES = kEpiWarps * 2048;
 constexpr int Q = 4;                                 // task ring depth
+#ifndef OOO_TMA_STORE
+#define OOO_TMA_STORE 0
+#endif
+// 1: the row-local chain outputs of identity-activation F_i and of dO_i leave
+// through per-warp TMA bulk stores (64B-swizzled 32 x 32 boxes) instead of
+// the smem transpose + st.global path; the early publish waits for their
+// completion (cp.async.bulk.wait_group 0) before the release.
+constexpr bool kTmaStore = OOO_TMA_STORE != 0;
 constexpr uint32_t TMEM_COLS = 512;
 constexpr uint64_t kTimeoutNs = 4000000000ull;
 
@@ -662,6 +670,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         continue;
       }
       const Op &o = p.ops[T.op];
+      const CUtensorMap *mX = kTmaStore ? map_of(o.mapX, p.maps, &tmY, &tmDX) : nullptr;
       const LayerDev &Ld = p.layers[T.layer - 1];
       const int acc = ja & 1;
       const int jacc = ja++;
@@ -734,7 +743,8 @@ __global__ void __launch_bounds__(kThreads, 1)
           uint32_t u[16];
           pack32(v, u);                                         // Z_i in bf16 (RNE)
           if (act == ACT_ID || (dbg & 1)) {
-            if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);   // X_{i+1} = Z_i (or Y)
+            if (kTmaStore) stage_store32_packed(mX, stg, lane, u, col0, row0);
+            else if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);   // X_{i+1} = Z_i (or Y)
           } else if (act == ACT_GELU) {
             // X_{i+1} = gelu(Z_i) and, for the next backward, gelu'(Z_i) in
             // the Z_i store (one Phi / e^{-z^2/2} evaluation for both; the
@@ -763,7 +773,8 @@ __global__ void __launch_bounds__(kThreads, 1)
           pack32(v, u);                                         // dZ_{i-1} in bf16 (RNE)
 #pragma unroll
           for (int j = 0; j < 16; ++j) u[j] = row_ok ? u[j] : 0u;
-          if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);  // dZ_{i-1} (or dX)
+          if (kTmaStore) stage_store32_packed(mX, stg, lane, u, col0, row0);
+          else if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);  // dZ_{i-1} (or dX)
           if (dbpart && !late_db) {
             unpack32(u, v);
             red[q * kMaxBN + c * 32 + lane] = warp_colsum32(v, lane);
@@ -780,7 +791,12 @@ __global__ void __launch_bounds__(kThreads, 1)
       // release reductions are cumulative, so every store of the pass above
       // (all epilogue warps, ordered by the barrier) is visible before the count
       if (T.kind != EPI_WGRAD) {
+        if (kTmaStore) {
+          if (lane == 0) tma_store_wait_all();   // this warp's bulk stores are complete
+          __syncwarp();
+        }
         ebar();
+        if (kTmaStore && et == 0) asm volatile("fence.proxy.async.global;" ::: "memory");
         if (et == 0 && mrow0 < T.M) {
           if (T.kind == EPI_FWD) red_release_add(ctr + cl.fwd_rows + (T.layer - 1) * cl.MT + mblk, 1);
           else if (T.layer >= 2) red_release_add(ctr + cl.dz_rows + (T.layer - 2) * cl.MT + mblk, 1);

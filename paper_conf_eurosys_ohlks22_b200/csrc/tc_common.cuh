@@ -400,5 +400,23 @@ __device__ __forceinline__ void stage_store32(const CUtensorMap *map, uint32_t b
   if (lane == 0) tma_store_2d(map, buf, col0, row0);
 }
 
+// stage_store32 for values already packed to bf16 pairs.
+__device__ __forceinline__ void stage_store32_packed(const CUtensorMap *map, uint32_t buf, int lane,
+                                                     const uint32_t (&u)[16], int col0, int row0) {
+  if (lane == 0) tma_store_wait_read();
+  __syncwarp();
+  const uint32_t rbase = buf + lane * 64;
+#pragma unroll
+  for (int c = 0; c < 4; ++c) {
+    const uint32_t a = rbase + ((c ^ ((lane >> 1) & 3)) << 4);
+    asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(u[4 * c]), "r"(u[4 * c + 1]),
+                 "r"(u[4 * c + 2]), "r"(u[4 * c + 3])
+                 : "memory");
+  }
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  __syncwarp();
+  if (lane == 0) tma_store_2d(map, buf, col0, row0);
+}
+
 }  // namespace tc
 }  // namespace ooo

@@ -139,6 +139,11 @@ def test_bf16_bert_base_full_config_end_to_end():
     errs = max_err(out, ref)
     print("bert_base full-size errors", errs, "floor", bf16_floor(c.L))
     _check(errs, max(BF16_TOL, 2 * bf16_floor(c.L)))
+    # bench.py's N = 1 schedule: Algorithm 1 regions of one block (§4.1), graph-captured
+    stk.forward(to_dev(case.X, "bf16"))
+    stk.plan_regions(region_layers=6)
+    reg = case.run(stk, "regions", 0, graph=True, launches=2)
+    assert torch.equal(reg["raw"], out["raw"])
 
 
 # ------------------------------- fused step: backward(t) + forward(t+1)
@@ -299,4 +304,27 @@ def test_bf16_regions_full_size_block_slice():
     base = case.run(stk, "in_order", 0)
     assert torch.equal(out["raw"], base["raw"])
     _check(max_err(out, case.oracle()), BF16_TOL)
+    stk.close()
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("cfg", [configs.C3, configs.C4], ids=["bert_large", "gpt2_medium"])
+def test_bf16_144_layer_full_configs_end_to_end(cfg):
+    """Configs 2 and 3 end to end at full size (144 layers; 4096 / 512 tokens),
+    graph-captured reverse first-k and the Algorithm 1 region schedule (bench
+    launch configurations), gated at max(1e-2, 2 x the bf16 random-walk floor)
+    (SURVEY §8c G3), and bit-exact with in_order."""
+    case = Case(cfg.dims, cfg.acts, cfg.tokens, "bf16")
+    ref = case.oracle(cfg.L // 6)
+    stk = case.stack()
+    out = case.run(stk, "first_k", cfg.L // 6, graph=True)
+    errs = max_err(out, ref)
+    print(cfg.name, "full-size errors", errs, "floor", bf16_floor(cfg.L))
+    _check(errs, max(BF16_TOL, 2 * bf16_floor(cfg.L)))
+    stk.forward(to_dev(case.X, "bf16"))
+    stk.plan_regions(region_layers=6)
+    reg = case.run(stk, "regions", 0, graph=True)
+    assert torch.equal(reg["raw"], out["raw"])
+    base = case.run(stk, "in_order", 0)
+    assert torch.equal(base["raw"], out["raw"])
     stk.close()

@@ -20,23 +20,31 @@ def main():
            "`python bench.py --config Cn` (C2 = the bench line; the others are parity-test",
            "configs, measured for context).  ms/step = one CUDA-graph replay of",
            "[backward(t); forward(t+1)] (seed + one fused engine launch; the fp32 C1 uses",
-           "the per-layer multi-stream path).  `torch` = the same step as a plain",
+           "the per-layer multi-stream path).  The schedule is the better of reverse first-k",
+           "(k by the paper's search) and the Algorithm 1 region plan (6 layers per region,",
+           "bf16 only).  `torch` = the same step as a plain",
            "torch/cuBLAS op sequence in one CUDA graph (`tools/torch_baseline.py`, same box",
            "type, another call).  Step roofline = north-star definition (GEMM FLOP at the",
            "measured sustained bf16 peak; no all-reduce at N = 1).", "",
-           "| config | layers | tokens | ooo ms/step (k) | in-order ms | ooo speedup | step roofline ms | frac "
-           "| e2e it/s | torch ms | SM MHz (reasons) |",
-           "|---|---|---|---|---|---|---|---|---|---|---|"]
+           "| config | layers | tokens | ooo ms/step (schedule) | first-k ms (k) | regions ms | in-order ms "
+           "| ooo speedup | step roofline ms | frac | e2e it/s | torch ms | SM MHz (reasons) |",
+           "|---|---|---|---|---|---|---|---|---|---|---|---|---|"]
     for c in ["C2", "C3", "C4", "C5", "C1"]:
         p = os.path.join(d, f"bench_{c}.log")
         if not os.path.exists(p):
             continue
-        r = last_json(p)
+        try:
+            r = last_json(p)
+        except (IndexError, ValueError):
+            continue
         sr = r["step_roofline"]
         frac = "—" if sr["frac"] is None else f"{sr['frac']:.3f}"
         clk = r["clocks"]
         out.append(f"| {c} {r['config']['workload'].split(' ')[0]} | {r['config']['layers']} | "
-                   f"{r['config']['tokens_per_gpu']} | {r['ms_per_step']:.3f} (k={r['config']['k']}) | "
+                   f"{r['config']['tokens_per_gpu']} | {r['ms_per_step']:.3f} "
+                   f"({'regions' if r['config']['schedule'].startswith('regions') else 'first-k'}) | "
+                   f"{r['ooo_first_k']['ms_per_step']:.3f} (k={r['config']['k']}) | "
+                   f"{(r.get('regions') or {}).get('ms_per_step', float('nan')):.3f} | "
                    f"{r['in_order']['ms_per_step']:.3f} | {r['ooo_speedup_vs_in_order']:.2f} | {sr['ms']:.3f} | "
                    f"{frac} | {r['e2e']['value']:.0f} | {TORCH_MS.get(c, '—')} | "
                    f"{clk['sm_mhz']:.0f} ({','.join(clk['reasons']) or '-'}) |")

@@ -31,6 +31,10 @@ METRICS = [
     ("sm__throughput.avg.pct_of_peak_sustained_elapsed", "SM throughput"),
     ("gpu__compute_memory_throughput.avg.pct_of_peak_sustained_elapsed", "memory throughput"),
     ("sm__warps_active.avg.pct_of_peak_sustained_active", "achieved occupancy"),
+    ("lts__t_bytes.sum", "L2 traffic (all requests)"),
+    ("l1tex__m_xbar2l1tex_read_bytes.sum", "L2 -> SM read bytes"),
+    ("lts__t_sectors_srcunit_ltcfabric.sum", "L2 sectors from the other die (fabric)"),
+    ("lts__throughput.avg.pct_of_peak_sustained_elapsed", "L2 throughput"),
     ("launch__registers_per_thread", "registers/thread"),
     ("launch__grid_size", "grid"),
     ("launch__block_size", "block"),
