@@ -533,7 +533,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         // MN-major B arrives in whole 64-column boxes (a 96-column share of a
         // 192-wide pair tile fetches 128 columns; the MMA reads the first 96)
         const int bh_ld = b_mn ? (bh + 63) / 64 * 64 : bh;
-        const uint32_t bytes = CG * (A_BYTES + bh_ld * BK * 2);   // all CTAs, on the leader's barrier
+        const uint32_t a_bytes = T.kind == EPI_WGRAD ? (uint32_t)A_BYTES : (uint32_t)p.a_rows * (BK * 2);
+        const uint32_t bytes = CG * (a_bytes + bh_ld * BK * 2);   // all CTAs, on the leader's barrier
         const int am = T.m0 + BM * (int)rank;
         const int bn0 = T.n0 + bh * (int)rank;
         int npre = 0;

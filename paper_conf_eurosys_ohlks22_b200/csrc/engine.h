@@ -85,6 +85,9 @@ struct Params {
                            // (N > 1); both also wait dW_{i+1} (it reads X_{i+1}, which F_i overwrites)
   int32_t dbg;             // tuning experiments only (OOO_DBG): bit0 skip act math, bit1 skip stores, bit3 no X copy (stale X_1), bit4 no weight prefetch
   int32_t copy_nt;         // column tiles per row block of the X -> X_1 copy
+  int32_t a_rows;          // rows of the row-major A box of F_i / dO_i tiles: 128, or M rounded
+                           // up to 8 when all tokens fit one 128-row tile (1-CTA tiles): the
+                           // MMA's rows beyond it read stale smem and are never stored
   const CUtensorMap *maps;
   int32_t *ctr;            // counter array base
   const LayerDev *layers;  // index i-1

@@ -681,6 +681,13 @@ pl::Model plan_model() {
   return m;
 }
 
+// Rows of the A box of row-local (F_i / dO_i) tiles: all tokens fit one
+// 1-CTA tile -> only the M valid rows are fetched (no 128-row OOB fill).
+int a_box_rows(const Plan &p) {
+  if (p.cg == 1 && p.M < 128 && env_int("OOO_SMALL_ABOX", 1)) return (p.M + 7) / 8 * 8;
+  return 128;
+}
+
 int copy_bn(int d0) { return d0 % 256 == 0 ? 256 : (d0 % 128 == 0 ? 128 : 64); }
 
 // Whole-op planner units.  Row-local ops (F_i, dO_i, copy) span the PT =
@@ -795,6 +802,7 @@ ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const 
   P.fwd_gate = fwd_gate;
   P.dbg = env_int("OOO_DBG", 0);
   P.copy_nt = (s->dims[0] + copy_bn(s->dims[0]) - 1) / copy_bn(s->dims[0]);
+  P.a_rows = a_box_rows(p);
   P.maps = s->dmaps;
   P.ctr = s->ctr;
   P.layers = s->dlayers;
@@ -1390,11 +1398,11 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
       CUtensorMap *m = &maps[(size_t)(i - 1) * MS_COUNT];
       memset(m, 0, sizeof(CUtensorMap) * MS_COUNT);
       ooo_status st;
-      if ((st = make_map(&m[MS_FWD_A], r.X, lp.din, p.M, 64, 128)) != OOO_OK ||
+      if ((st = make_map(&m[MS_FWD_A], r.X, lp.din, p.M, 64, a_box_rows(p))) != OOO_OK ||
           (st = make_map(&m[MS_FWD_B], r.W, lp.dout, lp.din, 64, 64)) != OOO_OK ||
           (r.Xn && (st = make_map(&m[MS_FWD_X], r.Xn, lp.dout, p.M, 32, 32, 64)) != OOO_OK) ||
           (r.Z && (st = make_map(&m[MS_FWD_Z], r.Z, lp.dout, p.M, 32, 32, 64)) != OOO_OK) ||
-          (st = make_map(&m[MS_DX_A], r.dZ, lp.dout, p.M, 64, 128)) != OOO_OK ||
+          (st = make_map(&m[MS_DX_A], r.dZ, lp.dout, p.M, 64, a_box_rows(p))) != OOO_OK ||
           (st = make_map(&m[MS_DX_B], r.W, lp.dout, lp.din, 64, lp.ebn_dx / p.cg)) != OOO_OK ||
           (st = make_map(&m[MS_DZ_X], r.dZ, lp.dout, p.M, 32, 32, 64)) != OOO_OK ||
           (st = make_map(&m[MS_DW_A], r.X, lp.din, p.M, 64, 64)) != OOO_OK ||
