@@ -63,13 +63,15 @@ template <> struct V<float> {
   __device__ static void store_scalar(void *p, float f) { *reinterpret_cast<float *>(p) = f; }
 };
 
-// grid (ceil(M / bm), ceil(N / (32 * VEC))), block (32, 8)
+// grid (ceil(M / bm), ceil(N / (32 * VEC))), block (32, kSeedTY): kSeedTY
+// row lanes so that each thread has bm / kSeedTY rows, all loaded at once
+constexpr int kSeedTY = 32;
 template <typename T>
-__global__ void __launch_bounds__(256) seed_kernel(const T *__restrict__ dy, const T *__restrict__ z,
+__global__ void __launch_bounds__(32 * kSeedTY) seed_kernel(const T *__restrict__ dy, const T *__restrict__ z,
                                                    int act, T *__restrict__ dz,
                                                    float *__restrict__ dbpart, int M, int N, int bm) {
   constexpr int VEC = V<T>::N;
-  __shared__ float red[8][32 * VEC];
+  __shared__ float red[kSeedTY][32 * VEC];
   const int tx = threadIdx.x, ty = threadIdx.y;
   const int col = (blockIdx.y * 32 + tx) * VEC;
   const int r0 = blockIdx.x * bm;
@@ -77,32 +79,43 @@ __global__ void __launch_bounds__(256) seed_kernel(const T *__restrict__ dy, con
 #pragma unroll
   for (int j = 0; j < VEC; ++j) sum[j] = 0.f;
   if (col < N) {
-    for (int r = r0 + ty; r < r0 + bm && r < M; r += 8) {
-      const size_t o = (size_t)r * N + col;
-      float g[VEC];
-      V<T>::load(dy + o, g);
-      if (act != ACT_ID) {
-        float zz[VEC];
-        V<T>::load(z + o, zz);
+    // batches of U rows: all U loads in flight before the first use (the
+    // kernel is HBM-latency bound otherwise: one 16-B load per thread in flight)
+    constexpr int U = 4;
+    const int rend = min(r0 + bm, M);
+    for (int rb = r0 + ty; rb < rend; rb += kSeedTY * U) {
+      float g[U][VEC], zz[U][VEC];
 #pragma unroll
-        for (int j = 0; j < VEC; ++j) g[j] *= act_grad_f(act, zz[j]);
+      for (int u = 0; u < U; ++u) {
+        const int r = rb + kSeedTY * u;
+        if (r < rend) {
+          V<T>::load(dy + (size_t)r * N + col, g[u]);
+          if (act != ACT_ID) V<T>::load(z + (size_t)r * N + col, zz[u]);
+        }
       }
-      V<T>::store(dz + o, g);             // rounds g to the storage dtype
 #pragma unroll
-      for (int j = 0; j < VEC; ++j) sum[j] += g[j];
+      for (int u = 0; u < U; ++u) {
+        const int r = rb + kSeedTY * u;
+        if (r < rend) {
+          if (act != ACT_ID) {
+#pragma unroll
+            for (int j = 0; j < VEC; ++j) g[u][j] *= act_grad_f(act, zz[u][j]);
+          }
+          V<T>::store(dz + (size_t)r * N + col, g[u]);   // rounds g to the storage dtype
+#pragma unroll
+          for (int j = 0; j < VEC; ++j) sum[j] += g[u][j];   // rows in increasing order (fixed)
+        }
+      }
     }
   }
 #pragma unroll
   for (int j = 0; j < VEC; ++j) red[ty][tx * VEC + j] = sum[j];
   __syncthreads();
-  if (ty == 0 && col < N) {
+  if (ty < VEC && col < N) {   // row lane ty sums column col + ty over the kSeedTY lanes
+    float s = 0.f;
 #pragma unroll
-    for (int j = 0; j < VEC; ++j) {
-      float s = 0.f;
-#pragma unroll
-      for (int r = 0; r < 8; ++r) s += red[r][tx * VEC + j];     // fixed order
-      dbpart[(size_t)blockIdx.x * N + col + j] = s;
-    }
+    for (int r = 0; r < kSeedTY; ++r) s += red[r][tx * VEC + ty];     // fixed order
+    dbpart[(size_t)blockIdx.x * N + col + ty] = s;
   }
 }
 
@@ -160,7 +173,7 @@ cudaError_t launch_seed(bool bf16, const void *dy, const void *z, int act, void 
   dim3 grid((M + bm - 1) / bm, (N + 32 * vec - 1) / (32 * vec), 1);
   if (grid_ctas) *grid_ctas = grid.x * grid.y;
   cudaLaunchAttribute attr[1];
-  cudaLaunchConfig_t cfg = ew::cfg_for(grid, dim3(32, 8, 1), ctx, attr);
+  cudaLaunchConfig_t cfg = ew::cfg_for(grid, dim3(32, ew::kSeedTY, 1), ctx, attr);
   if (bf16)
     return cudaLaunchKernelEx(&cfg, ew::seed_kernel<__nv_bfloat16>,
                               static_cast<const __nv_bfloat16 *>(dy), static_cast<const __nv_bfloat16 *>(z),
