@@ -246,7 +246,9 @@ ooo_status ooo_join(ooo_stack *s, void *stream);
  * Synchronous (host waits for the profiling launches; not capturable) and
  * destructive: activations and gradients are overwritten, so an ooo_forward
  * must run before the next ooo_backward (OOO_ERR_STATE otherwise).  bf16
- * stacks only (OOO_ERR_UNSUPPORTED for fp32); region_layers >= 1, reps >= 1. */
+ * stacks with world_size 1 only (OOO_ERR_UNSUPPORTED otherwise: the paper's
+ * single-GPU method, and per-rank profiles could order the all-reduces
+ * differently on different ranks); region_layers >= 1, reps >= 1. */
 ooo_status ooo_plan_regions(ooo_stack *s, int32_t region_layers, int32_t reps, void *stream);
 
 /* The current region plan: *n_regions, *k_pre (pre-scheduled regions),

@@ -1647,6 +1647,9 @@ ooo_status ooo_plan_regions(ooo_stack *s, int32_t region_layers, int32_t reps, v
   if (region_layers < 1 || reps < 1) return fail(OOO_ERR_INVALID_ARGUMENT, "region_layers and reps must be >= 1");
   if (!s->p.engine) return fail(OOO_ERR_UNSUPPORTED, "region planning profiles the bf16 engine (fp32 stack)");
   if (s->p.L < 2) return fail(OOO_ERR_UNSUPPORTED, "region planning needs L >= 2");
+  // single-GPU method (§4): a plan profiled per rank could differ between
+  // ranks, and the all-reduce issue order (D's dW order) must be identical
+  if (s->d.world_size > 1) return fail(OOO_ERR_UNSUPPORTED, "region scheduling is single-GPU (world_size 1)");
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   OOO_TRY(engine_flush(s));
   OOO_TRY(join_into(s, st));
