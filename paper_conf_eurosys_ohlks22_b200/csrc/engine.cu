@@ -34,6 +34,7 @@
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "engine.h"
 #include "kernels.h"
@@ -45,6 +46,11 @@ namespace eng {
 using namespace ooo::tc;
 
 #ifdef OOO_TRACE
+__device__ __forceinline__ uint32_t cta_rank_raw() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
 // Debug builds only (libooo_trace.so): per-task stamps [task][8]:
 // globaltimer at dispensed / inputs ready / accumulator ready / published
 // (leader CTA; CTA index in the top 16 bits), then clock64 at the same points.
@@ -72,9 +78,13 @@ __device__ __forceinline__ void etrace_gt(int t, int slot) {
     g_etrace3[(size_t)t * 8 + slot] = v;
   }
 }
-// per-k-block clocks of CTA 0's first task: [150000 + kb][slot]
-__device__ __forceinline__ void ktrace(int j, int kb, int slot) {
-  if (g_etrace3 && blockIdx.x == 0 && j == 0 && kb < 1024) g_etrace3[(size_t)(150000 + kb) * 8 + slot] = clock64();
+// per-k-block clocks of task g_ktask (leader CTA; OOO_KTASK, default 0):
+// [150000 + kb][slot], slot 0 producer issue, 2 MMA wait start, 3 wait passed,
+// 4 MMAs + commit issued
+__device__ int g_ktask = 0;
+__device__ __forceinline__ void ktrace(int t, int kb, int slot) {
+  if (g_etrace3 && t == g_ktask && kb < 1024 && cta_rank_raw() == 0)
+    g_etrace3[(size_t)(150000 + kb) * 8 + slot] = clock64();
 }
 #else
 __device__ __forceinline__ void etrace(int, int) {}
@@ -393,12 +403,12 @@ __device__ __forceinline__ void prefetch_b(const CUtensorMap *mB, uint32_t sbase
 template <int CG, bool A_MN, bool B_MN>
 __device__ __forceinline__ void produce(const TaskRt &T, const CUtensorMap *mA, const CUtensorMap *mB, uint32_t sbase,
                                         uint32_t bar_empty, uint32_t bar_full, uint32_t L_full, bool leader,
-                                        uint32_t bytes, int am, int bn0, int bh, int &it, int j, int npre) {
+                                        uint32_t bytes, int am, int bn0, int bh, int &it, int t, int npre) {
   using C = Cfg<CG>;
   int s = it % C::STAGES;
   uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;   // phase of the stage's next fill
   for (int kb = 0; kb < npre; ++kb) {
-    ktrace(j, kb, 0);
+    ktrace(t, kb, 0);
     load_a<CG, A_MN>(mA, sbase + s * C::STAGE, L_full + 8 * s, am, kb * BK);
     if (++s == C::STAGES) {
       s = 0;
@@ -407,7 +417,7 @@ __device__ __forceinline__ void produce(const TaskRt &T, const CUtensorMap *mA, 
   }
   for (int kb = npre; kb < T.nkb; ++kb) {
     if (it + kb >= C::STAGES) mbar_wait_b(bar_empty + 8 * s, ph ^ 1u);
-    ktrace(j, kb, 0);
+    ktrace(t, kb, 0);
     if (leader) mbar_expect_tx(bar_full + 8 * s, bytes);
     const uint32_t lb = L_full + 8 * s;
     const uint32_t sa = sbase + s * C::STAGE;
@@ -552,9 +562,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         asm volatile("fence.proxy.async.global;" ::: "memory");   // TMA reads see the producers' data
         if (leader) etrace(t, 1);
         switch ((a_mn ? 2 : 0) + (b_mn ? 1 : 0)) {
-          case 1: produce<CG, false, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j, npre); break;
-          case 0: produce<CG, false, false>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j, npre); break;
-          default: produce<CG, true, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, j, npre); break;
+          case 1: produce<CG, false, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, t, npre); break;
+          case 0: produce<CG, false, false>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, t, npre); break;
+          default: produce<CG, true, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, t, npre); break;
         }
       }
     }
@@ -597,9 +607,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         int s = it % C::STAGES;
         uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;
         for (int kb = 0; kb < T.nkb; ++kb) {
-          ktrace(j, kb, 2);
+          ktrace(t, kb, 2);
           mbar_wait_b(bar_full + 8 * s, ph);
-          ktrace(j, kb, 3);
+          ktrace(t, kb, 3);
           if (kb == 0) etrace_gt(t, 6);           // first k-block landed
           if (kb == T.nkb - 1) etrace_gt(t, 7);   // last k-block landed
           fence_after();
@@ -611,6 +621,7 @@ __global__ void __launch_bounds__(kThreads, 1)
             umma_bf16_pair(dtm, ad + 2 * astep, bd + 2 * bstep, ID, 1u);
             umma_bf16_pair(dtm, ad + 3 * astep, bd + 3 * bstep, ID, 1u);
             umma_commit_pair(bar_empty + 8 * s);
+            ktrace(t, kb, 4);
           } else {
             umma_bf16(dtm, ad, bd, ID, kb != 0 ? 1u : 0u);
             umma_bf16(dtm, ad + astep, bd + bstep, ID, 1u);
@@ -894,6 +905,10 @@ int engine_smem_bytes(int cg) { return cg == 2 ? Cfg<2>::SMEM : Cfg<1>::SMEM; }
 
 #ifdef OOO_TRACE
 cudaError_t engine_set_trace(void *p) {
+  const char *kt = getenv("OOO_KTASK");
+  const int ktask = kt && *kt ? atoi(kt) : 0;
+  cudaError_t e0 = cudaMemcpyToSymbol(g_ktask, &ktask, sizeof(ktask));
+  if (e0 != cudaSuccess) return e0;
   // [task][8] phase stamps, [task][8] epilogue clocks, [task][8] pipeline stamps (same buffer)
   void *p2 = p ? static_cast<char *>(p) + (size_t)200000 * 8 * 8 : nullptr;
   void *p3 = p ? static_cast<char *>(p) + (size_t)2 * 200000 * 8 * 8 : nullptr;
