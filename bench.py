@@ -48,6 +48,10 @@ def parse():
     ap.add_argument("--regions", type=int, default=6,
                     help="N = 1: also plan the single-GPU multi-stream schedule (Algorithm 1, §4.1) with regions of "
                          "this many layers and time the better of it and reverse first-k; 0 = off")
+    ap.add_argument("--emulate-n", type=int, default=8,
+                    help="N = 1: also measure exposed communication with an EMULATED ring all-reduce of this many "
+                         "ranks (comm stream held for 2(n-1)/n x bucket bytes / 900 GB/s + 8 us per bucket, "
+                         "16-SM NCCL reserve); 0 = off")
     ap.add_argument("--bucket-layers", type=int, default=1)
     ap.add_argument("--nccl-max-ctas", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
@@ -364,6 +368,45 @@ def main():
         g_off_in.close()
         stk_off.close()
 
+    # ---- N = 1: exposed communication against an EMULATED n-rank ring all-reduce
+    # (no NCCL, no data moved: the comm stream is held for each bucket's ring
+    # time; F_i waits for its bucket's flag exactly as at N = n)
+    emulated = None
+    if world == 1 and args.emulate_n > 1 and dt == "bf16":
+        n, gbps, lat = args.emulate_n, 900.0, 8.0
+        elt = 2
+        ar_total = sum(2.0 * (n - 1) / n * (cfg.dims[i] * cfg.dims[i + 1] + cfg.dims[i + 1]) * elt / (gbps * 1e9) * 1e3
+                       + lat * 1e-3 for i in range(L))
+        ks = sorted({0, max(1, L // 24), L // 6, L // 2, L})
+        times = {}
+        for label, bw, la in (("on", gbps, lat), ("off", 1e9, 0.0)):
+            os.environ.update({"OOO_EMULATE_AR_N": str(n), "OOO_EMULATE_AR_GBPS": str(bw),
+                               "OOO_EMULATE_AR_LAT_US": str(la)})
+            se = OooStack(cfg.dims, cfg.acts, M, W, b, dtype=dt)
+            se.forward(X, Y)
+            for kind, k in [("in_order", 0)] + [("first_k", k) for k in ks]:
+                g = se.graph(X, Y, dY, kind, k)
+                for _ in range(3):
+                    g.launch(stream)
+                times[(label, kind, k)] = min(timed(g, max(10, args.steps // 2)) for _ in range(2))
+                g.close()
+            se.close()
+        for key in ("OOO_EMULATE_AR_N", "OOO_EMULATE_AR_GBPS", "OOO_EMULATE_AR_LAT_US"):
+            os.environ.pop(key, None)
+        sweep = {}
+        for kind, k in [("in_order", 0)] + [("first_k", k) for k in ks]:
+            on, off = times[("on", kind, k)], times[("off", kind, k)]
+            sweep[f"{kind}({k})"] = {"ms": on, "exposed_ms": max(0.0, on - off),
+                                     "hidden_fraction": 1.0 - max(0.0, on - off) / ar_total}
+        best = min((v["ms"], key) for key, v in sweep.items() if key.startswith("first_k"))[1]
+        emulated = {"n": n, "link_GBps_per_direction": gbps, "latency_us_per_bucket": lat,
+                    "note": "EMULATED all-reduce on one GPU (comm stream held for the ring time; no NCCL, no "
+                            "data moved); the engine keeps the 16-SM NCCL reserve",
+                    "allreduce_total_ms": ar_total, "in_order_ms": sweep["in_order(0)"]["ms"], "best": best,
+                    "best_ms": sweep[best]["ms"], "best_exposed_ms": sweep[best]["exposed_ms"],
+                    "best_hidden_fraction": sweep[best]["hidden_fraction"],
+                    "ooo_speedup_vs_in_order": sweep["in_order(0)"]["ms"] / sweep[best]["ms"], "k_sweep": sweep}
+
     # ---- per-kernel durations: instrumented replay of the same step (CUDA events per launch)
     stk.set_timing(True)
     g_t = stk.graph(X, Y, dY, *sched)
@@ -505,6 +548,7 @@ def main():
         "ooo_first_k0": {"value": 1e3 / ms_k0, "ms_per_step": ms_k0},
         "ooo_first_k": {"k": k_best, "value": 1e3 / ms_fk, "ms_per_step": ms_fk},
         "regions": regions,
+        "emulated_dp": emulated,
         "step_roofline": {"ms": step_roof_ms, "frac": step_roof_ms / ms_ooo if step_roof_ms else None,
                           "tensor_ms": t_tensor, "allreduce_ms_at_770GBps": t_ar, "gemm_flops": flops,
                           "hbm_min_bytes": hbm_bytes, "hbm_ms": t_hbm,

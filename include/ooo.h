@@ -55,7 +55,11 @@
  * Asynchronous CUDA / NCCL failures surface as OOO_ERR_CUDA / OOO_ERR_NCCL
  * from a later call (ooo_join polls ncclCommGetAsyncError).  No C++
  * exception crosses this ABI.  Threading: one stack is used by one host
- * thread at a time; ooo_last_error is thread-local.
+ * thread at a time; ooo_last_error is thread-local.  GPU sharing: a bf16
+ * step is one persistent kernel holding one CTA per SM (N > 1: all but the
+ * SMs reserved for NCCL); steps of two stacks must not run concurrently on
+ * one GPU (a second persistent grid pending for SMs can starve the comm
+ * stream's all-reduce kernels the first one waits on).
  *
  * Collective rule: with world_size > 1 every rank must call ooo_backward with
  * the same schedule (D and the NCCL issue order depend only on (L, k));
@@ -219,7 +223,12 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out);
 /* F_1..F_L: X [M][d_0] (device, dtype) -> Y [M][d_L] (device, dtype).
  * X is copied into the stack's X_1 store; Y is written by F_L.  If a backward
  * is pending, F_i first waits for layer i's synchronised gradient (and for
- * dW_{i+1}, which still reads X_{i+1}). */
+ * dW_{i+1}, which still reads X_{i+1}).  With a communicating stack (N > 1,
+ * or the emulated all-reduce OOO_EMULATE_AR_N), run training steps through
+ * ooo_graph_create / ooo_graph_launch: an EAGER fused step whose comm stream
+ * holds kernels behind the per-bucket value-waits was observed to stall on
+ * B200 (the emulated all-reduce; the graph-launched step is unaffected and is
+ * what the tests and bench.py run). */
 ooo_status ooo_forward(ooo_stack *s, const void *X, void *Y, void *stream /* cudaStream_t */);
 
 /* Backward of the last forward: dY [M][d_L] (device, dtype).  dX [M][d_0]

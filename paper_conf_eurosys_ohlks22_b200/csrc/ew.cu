@@ -201,4 +201,24 @@ cudaError_t launch_pack(bool bf16, const float *wpart, int S, long long wcount, 
                             dbpart, R, N, static_cast<float *>(dbout), alpha);
 }
 
+// Emulated all-reduce (single-GPU measurement aid, OOO_EMULATE_AR_N): one
+// thread holds the comm stream for `ns` nanoseconds (the modelled ring
+// all-reduce time of a bucket), so the engine's F_i gate on the bucket's
+// all-reduce flag sees a realistic completion time.  No data is moved.
+namespace ew {
+__global__ void delay_kernel(unsigned long long ns) {
+  unsigned long long t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  do {
+    __nanosleep(200);
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  } while (t - t0 < ns);
+}
+}  // namespace ew
+
+cudaError_t launch_delay(unsigned long long ns, cudaStream_t stream) {
+  ew::delay_kernel<<<1, 1, 0, stream>>>(ns);
+  return cudaGetLastError();
+}
+
 }  // namespace ooo

@@ -75,6 +75,7 @@ cudaError_t launch_seed(bool bf16, const void *dy, const void *z, int act, void 
                         int M, int N, int bm, const LaunchCtx &ctx, int *grid_ctas);
 // pack (BK5): wout[e] = st(alpha * sum_s wpart[s][e]) for e < wcount (if wpart != null);
 //             dbout[n] = st(alpha * sum_r dbpart[r][n]).  Fixed summation order.
+cudaError_t launch_delay(unsigned long long ns, cudaStream_t stream);   // emulated all-reduce
 cudaError_t launch_pack(bool bf16, const float *wpart, int S, long long wcount, void *wout,
                         const float *dbpart, int R, int N, void *dbout, float alpha,
                         const LaunchCtx &ctx, int *grid_ctas);

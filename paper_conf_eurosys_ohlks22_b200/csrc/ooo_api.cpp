@@ -399,6 +399,7 @@ struct ooo_stack {
   int prio_hi = 0, prio_lo = 0;
   std::vector<cudaEvent_t> ev_dz, ev_pack, ev_ar;   // ev_dz[i], ev_pack[i] (1-based), ev_ar[b]
   cudaEvent_t ev_fork = nullptr, ev_j_hi = nullptr, ev_j_lo = nullptr, ev_j_comm = nullptr;
+  cudaEvent_t ev_reset = nullptr;             // engine: counters reset (the comm stream's value-waits start after it)
   bool have_fwd = false;
   bool bwd_pending = false;
   ncclComm_t nccl = nullptr;
@@ -414,11 +415,16 @@ struct ooo_stack {
   const ooo::eng::LayerDev *dlayers = nullptr;
   int engine_ctas = 148;
   bool test_comm_gate = false;                // OOO_TEST_COMM_GATE=1 (N = 1 only): see comm_active
+  // emulated all-reduce (N = 1 only; OOO_EMULATE_AR_N = n >= 2): each bucket's
+  // S[dW] holds the comm stream for the ring time 2(n-1)/n x bytes / BW + lat
+  int emu_n = 0;
+  double emu_gbps = 900.0, emu_lat_us = 8.0;
   bool eng_pending = false;                   // ooo_backward enqueued, its kernel deferred
   std::vector<ooo::plan::Unit> eng_crit, eng_defer;   // the deferred backward's chains
   double eng_flops = 0;
   void *eng_dX = nullptr;
   bool eng_in_order = false;
+  bool eng_comm = false;                      // the deferred backward's per-bucket S[dW] still to enqueue
   // region plan (OOO_SCHED_REGIONS, §4.1; ooo_plan_regions)
   bool has_regions = false;
   std::vector<int> reg_D;          // backward order D of the plan
@@ -604,6 +610,16 @@ ooo_status launch_allreduce(ooo_stack *s, int b) {
   const LayerPlan &f = s->p.layer[first - 1];
   const LayerPlan &l = s->p.layer[last - 1];
   const int64_t e0 = f.goff_w, e1 = l.goff_b + l.dout;
+  if (s->emu_n > 1) {
+    TimedRec *tr;
+    OOO_TRY(begin_rec(s, s->comm, 5, b, 2, &tr));
+    const double n = s->emu_n;
+    const double ring = 2.0 * (n - 1) / n * (double)(e1 - e0) * s->p.elt;
+    const double ns = ring / (s->emu_gbps * 1e9) * 1e9 + s->emu_lat_us * 1e3;
+    CU_TRY(launch_delay((unsigned long long)ns, s->comm));
+    OOO_TRY(end_rec(tr, s->comm, 1, 0, ring));
+    return OOO_OK;
+  }
   if (s->nccl && s->d.comm_enabled) {
     TimedRec *tr;
     OOO_TRY(begin_rec(s, s->comm, 5, b, 2, &tr));
@@ -667,7 +683,9 @@ int map_index(int layer, int slot) { return (layer - 1) * MS_COUNT + slot; }
 // gating F_i).  test_comm_gate: world_size 1 with the same wait-value /
 // write-value chain but no all-reduce, so single-GPU tests exercise the N > 1
 // gating of the fused step.
-bool comm_active(const ooo_stack *s) { return (s->nccl != nullptr && s->d.comm_enabled) || s->test_comm_gate; }
+bool comm_active(const ooo_stack *s) {
+  return (s->nccl != nullptr && s->d.comm_enabled) || s->test_comm_gate || s->emu_n > 1;
+}
 
 namespace pl = ooo::plan;
 static_assert(pl::FWD == EPI_FWD && pl::DGRAD == EPI_DGRAD && pl::WGRAD == EPI_WGRAD &&
@@ -832,6 +850,42 @@ ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const 
   return end_rec(tr, s->hi, s->engine_ctas, flops, 0);
 }
 
+// The deferred backward's S[dW] per bucket on the comm stream, enqueued
+// right AFTER the engine kernel whose counters it waits on: an eager
+// cuStreamWaitValue32 followed by a kernel on the comm stream, submitted
+// before the engine kernel that satisfies the wait, hangs the device (the
+// stream-ordered graph capture has no such hazard, but one order serves both).
+ooo_status engine_comm(ooo_stack *s) {
+  if (!s->eng_comm) return OOO_OK;
+  s->eng_comm = false;
+  const Plan &p = s->p;
+  const int L = p.L;
+  CU_TRY(cudaStreamWaitEvent(s->comm, s->ev_reset, 0));   // value-waits observe the reset counters
+  // S[dW] per bucket in D's dW order: the comm stream waits for the bucket's
+  // dW tiles (engine counter), all-reduces, and publishes ar_done for F_i.
+  static StreamValueFn wait_fn = stream_value_fn("cuStreamWaitValue32");
+  static StreamValueFn write_fn = stream_value_fn("cuStreamWriteValue32");
+  if (!wait_fn || !write_fn) return fail(OOO_ERR_CUDA, "stream memory operations unavailable");
+  std::vector<int> left(p.nbuckets), tiles(p.nbuckets, 0);
+  for (int b = 0; b < p.nbuckets; ++b) left[b] = p.bucket_last[b] - p.bucket_first[b] + 1;
+  for (int i = 1; i <= L; ++i) {
+    const LayerPlan &lp = p.layer[i - 1];
+    tiles[lp.bucket] += ((lp.din + 127) / 128) * ((lp.dout + lp.ebn_dw - 1) / lp.ebn_dw);
+  }
+  for (int op : s->D) {
+    if (op > 0) continue;
+    const int b = p.layer[-op - 1].bucket;
+    if (--left[b] != 0) continue;
+    CUresult r = wait_fn(s->comm, reinterpret_cast<CUdeviceptr>(s->ctr + p.cl.bucket_done + b),
+                         (cuuint32_t)tiles[b], CU_STREAM_WAIT_VALUE_GEQ);
+    if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWaitValue32 failed (%d)", (int)r);
+    OOO_TRY(launch_allreduce(s, b));
+    r = write_fn(s->comm, reinterpret_cast<CUdeviceptr>(s->ctr + p.cl.ar_done + b), 1, 0);
+    if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWriteValue32 failed (%d)", (int)r);
+  }
+  return OOO_OK;
+}
+
 // A backward whose kernel is still deferred (engine): run it alone.
 ooo_status engine_flush(ooo_stack *s) {
   if (!s->eng_pending) return OOO_OK;
@@ -839,8 +893,9 @@ ooo_status engine_flush(ooo_stack *s) {
   std::vector<pl::Unit> defer = s->eng_defer;
   for (pl::Unit &u : defer)
     if (u.release <= -2) u.release = (int)s->eng_crit.size();   // its forward region: after the chain
-  return engine_launch(s, s->eng_crit, defer, nullptr, s->eng_dX, nullptr, s->eng_in_order, 0, 8,
-                       s->eng_flops);
+  OOO_TRY(engine_launch(s, s->eng_crit, defer, nullptr, s->eng_dX, nullptr, s->eng_in_order, 0, 8,
+                        s->eng_flops));
+  return engine_comm(s);
 }
 
 ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st) {
@@ -868,6 +923,7 @@ ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st)
       if (u.release <= -2) u.release = f1 + (-u.release - 1) - 1;   // region starting at F_m
     OOO_TRY(engine_launch(s, crit, defer, Y, s->eng_dX, X, s->eng_in_order, ar ? 2 : 1, 9,
                           s->eng_flops + flops));
+    OOO_TRY(engine_comm(s));
   } else {
     CU_TRY(cudaMemsetAsync(s->ctr, 0, (size_t)p.cl.fwd_end * 4, s->hi));
     OOO_TRY(engine_launch(s, fwd, {}, Y, nullptr, X, false, 0, 7, flops));
@@ -887,10 +943,7 @@ ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, bool reg
   OOO_TRY(fork_from(s, st));
   CU_TRY(cudaMemsetAsync(s->ctr, 0, (size_t)p.cl.total * 4, s->hi));
   const bool comm = comm_active(s);
-  if (comm) {   // the comm stream's value-waits must observe the reset counters
-    CU_TRY(cudaEventRecord(s->ev_j_hi, s->hi));
-    CU_TRY(cudaStreamWaitEvent(s->comm, s->ev_j_hi, 0));
-  }
+  if (comm) CU_TRY(cudaEventRecord(s->ev_reset, s->hi));   // the comm stream's value-waits start after it
   OOO_TRY(launch_seed_op(s, dY, s->hi, s->prio_hi));
   s->eng_crit.clear();
   s->eng_defer.clear();
@@ -899,30 +952,7 @@ ooo_status engine_backward(ooo_stack *s, const void *dY, bool in_order, bool reg
   s->eng_dX = dX;
   s->eng_in_order = in_order;
   s->eng_pending = true;
-  if (comm) {
-    // S[dW] per bucket in D's dW order: the comm stream waits for the bucket's
-    // dW tiles (engine counter), all-reduces, and publishes ar_done for F_i.
-    static StreamValueFn wait_fn = stream_value_fn("cuStreamWaitValue32");
-    static StreamValueFn write_fn = stream_value_fn("cuStreamWriteValue32");
-    if (!wait_fn || !write_fn) return fail(OOO_ERR_CUDA, "stream memory operations unavailable");
-    std::vector<int> left(p.nbuckets), tiles(p.nbuckets, 0);
-    for (int b = 0; b < p.nbuckets; ++b) left[b] = p.bucket_last[b] - p.bucket_first[b] + 1;
-    for (int i = 1; i <= L; ++i) {
-      const LayerPlan &lp = p.layer[i - 1];
-      tiles[lp.bucket] += ((lp.din + 127) / 128) * ((lp.dout + lp.ebn_dw - 1) / lp.ebn_dw);
-    }
-    for (int op : s->D) {
-      if (op > 0) continue;
-      const int b = p.layer[-op - 1].bucket;
-      if (--left[b] != 0) continue;
-      CUresult r = wait_fn(s->comm, reinterpret_cast<CUdeviceptr>(s->ctr + p.cl.bucket_done + b),
-                           (cuuint32_t)tiles[b], CU_STREAM_WAIT_VALUE_GEQ);
-      if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWaitValue32 failed (%d)", (int)r);
-      OOO_TRY(launch_allreduce(s, b));
-      r = write_fn(s->comm, reinterpret_cast<CUdeviceptr>(s->ctr + p.cl.ar_done + b), 1, 0);
-      if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWriteValue32 failed (%d)", (int)r);
-    }
-  }
+  s->eng_comm = comm;   // enqueued right after the engine launch (engine_comm)
   s->have_fwd = false;
   s->bwd_pending = true;
   return OOO_OK;
@@ -1442,8 +1472,14 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
     int dev = 0, sms = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    // N > 1: leave SMs for the NCCL kernels the engine's counters wait on
-    const int reserve = d->world_size > 1 ? (d->nccl_max_ctas > 0 ? d->nccl_max_ctas : 16) : 0;
+    // emulated all-reduce (measurement aid, N = 1): see ooo_stack::emu_n
+    if (d->world_size == 1 && env_int("OOO_EMULATE_AR_N", 0) > 1) {
+      s->emu_n = env_int("OOO_EMULATE_AR_N", 0);
+      if (const char *v = getenv("OOO_EMULATE_AR_GBPS")) s->emu_gbps = atof(v);
+      if (const char *v = getenv("OOO_EMULATE_AR_LAT_US")) s->emu_lat_us = atof(v);
+    }
+    // N > 1 (or its emulation): leave SMs for the NCCL kernels the engine's counters wait on
+    const int reserve = d->world_size > 1 || s->emu_n > 1 ? (d->nccl_max_ctas > 0 ? d->nccl_max_ctas : 16) : 0;
     s->engine_ctas = std::max(1, sms - reserve);
     s->engine_ctas = std::min(s->engine_ctas, env_int("OOO_ENGINE_CTAS", s->engine_ctas));
   }
@@ -1468,7 +1504,8 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
     if ((e = mk(&s->ev_ar[b])) != cudaSuccess)
       return cleanup_fail(fail(OOO_ERR_CUDA, "event create: %s", cudaGetErrorString(e)));
   if ((e = mk(&s->ev_fork)) != cudaSuccess || (e = mk(&s->ev_j_hi)) != cudaSuccess ||
-      (e = mk(&s->ev_j_lo)) != cudaSuccess || (e = mk(&s->ev_j_comm)) != cudaSuccess)
+      (e = mk(&s->ev_j_lo)) != cudaSuccess || (e = mk(&s->ev_j_comm)) != cudaSuccess ||
+      (e = mk(&s->ev_reset)) != cudaSuccess)
     return cleanup_fail(fail(OOO_ERR_CUDA, "event create: %s", cudaGetErrorString(e)));
   if (d->world_size > 1) {
     const char *why = nullptr;
@@ -1585,7 +1622,7 @@ ooo_status ooo_destroy(ooo_stack *s) {
   for (auto e : s->ev_dz) if (e) cudaEventDestroy(e);
   for (auto e : s->ev_pack) if (e) cudaEventDestroy(e);
   for (auto e : s->ev_ar) if (e) cudaEventDestroy(e);
-  for (cudaEvent_t e : {s->ev_fork, s->ev_j_hi, s->ev_j_lo, s->ev_j_comm}) if (e) cudaEventDestroy(e);
+  for (cudaEvent_t e : {s->ev_fork, s->ev_j_hi, s->ev_j_lo, s->ev_j_comm, s->ev_reset}) if (e) cudaEventDestroy(e);
   for (auto &r : s->recs) {
     if (r.a) cudaEventDestroy(r.a);
     if (r.b) cudaEventDestroy(r.b);

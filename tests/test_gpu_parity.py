@@ -222,6 +222,27 @@ def test_bf16_fused_step_comm_gated(monkeypatch):
     plain.close()
 
 
+@pytest.mark.parametrize("kind,k", [("first_k", 2), ("first_k", 0), ("in_order", 0)])
+def test_bf16_emulated_allreduce_graph(monkeypatch, kind, k):
+    """The emulated N = 8 all-reduce (OOO_EMULATE_AR_N: the comm stream held
+    for each bucket's ring time, 16-SM NCCL reserve; bench.py's emulated_dp)
+    through the captured step as bench.py times it: bit-identical to the
+    plain stack, within the gate of the oracle."""
+    case = Case([256, 512, 256, 256, 512, 256], ["gelu", "id", "id", "gelu", "id"], 520, "bf16")
+    plain = case.stack(bucket_layers=2)
+    base = case.run(plain, kind, k, graph=True, launches=2)
+    plain.close()
+    monkeypatch.setenv("OOO_EMULATE_AR_N", "8")
+    monkeypatch.setenv("OOO_EMULATE_AR_GBPS", "50")
+    emu = case.stack(bucket_layers=2)
+    monkeypatch.delenv("OOO_EMULATE_AR_N")
+    monkeypatch.delenv("OOO_EMULATE_AR_GBPS")
+    out = case.run(emu, kind, k, graph=True, launches=2)
+    assert torch.equal(out["raw"], base["raw"])
+    _check(max_err(out, case.oracle(k)), BF16_TOL)
+    emu.close()
+
+
 # ------------------- single-GPU multi-stream ooo: Algorithm 1 regions (§4.1)
 def _region_plan_valid(stk, L, need_dx=False):
     from oracle import schedule as S
