@@ -1,0 +1,88 @@
+"""Regenerate the derived profiles/rNN_* summaries from a profile_round.sh
+output directory: per-kernel table, emulated-DP sweep, chain-latency trace.
+(ncu_summary.py and configs_table.py cover the launch list, the --set full
+capture and the per-config table.)   python tools/write_profiles.py 01 gpurun_out/r01"""
+import json
+import os
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def kernels(rnd, d):
+    def table(csvp):
+        out = subprocess.run([sys.executable, os.path.join(ROOT, "tools", "ncu_kernels.py"), csvp, "/dev/null", "x"],
+                             capture_output=True, text=True, check=True).stdout.splitlines()
+        return out[2:]
+    met = ("gpu__time_duration.sum, dram__bytes_read.sum, dram__bytes_write.sum, "
+           "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active, dram__throughput.avg.pct_of_peak_sustained_elapsed")
+    lines = [f"# Round {rnd}: per-kernel ncu evidence (north star item 4), C2 = BERT-base stack, 4096 tokens", "",
+             f"`ncu --profile-from-start off -k regex:engine_kernel|gemm_tc_kernel|gemm_simt_kernel|pack_kernel|seed_kernel "
+             f"--metrics {met} --clock-control none` around `tools/engine_once.py` (serialised, cache-flushed replays: "
+             "per-launch times are not the live ones; read shares and per-kernel ratios).  DRAM % of peak is ncu's own peak.",
+             "", "## Product path: the fused engine step (Algorithm 1 regions) + the seed kernel (BK4)", ""]
+    lines += table(os.path.join(d, "engine_kernels.csv"))
+    lines += ["", "The engine runs the whole step (all F / dO / dW tiles with fused epilogues; the bucket pack/scale BK5 "
+              "is fused into the dW epilogue): tensor pipe active ≈ 47 % of its elapsed cycles -- the chain-latency bound "
+              f"of `r{rnd}_chain_latency.md`; it is not HBM-bound (≈ 21 % of DRAM peak).  The seed (dZ_L = dY ⊙ act'(Z_L) "
+              "+ db partials) is latency-bound at ≈ 1.2 TB/s (≈ 12 µs, 0.5 % of the step).", "",
+              "## Per-layer multi-stream path (`OOO_ENGINE=0`, reverse first-k(12)): one GEMM kernel per op, split-K dW "
+              "+ `pack_kernel` (BK5)", ""]
+    lines += table(os.path.join(d, "perlayer.csv"))
+    lines += ["", "`gemm_tc_kernel<BN, A_MN, B_MN, EPI>`: EPI 0 = F_i (bias + act), 1 = dO_i (act-grad + db partials), "
+              "2 = dW_i split-K partials.  Short per-layer kernels keep the tensor pipe at 13-31 % -- the reason the "
+              "product path is the persistent engine (DESIGN.md §5).  `pack_kernel` sums the fp32 split-K and db "
+              "partials in a fixed order with the 1/N scale: ≈ 6.5 MB per launch at ≈ 850 GB/s (launch/latency-bound "
+              "at this size)."]
+    open(os.path.join(ROOT, "profiles", f"r{rnd}_kernels.md"), "w").write("\n".join(lines) + "\n")
+
+
+def emulated(rnd, d):
+    rows = []
+    for c in ("C2", "C3", "C4"):
+        p = os.path.join(d, f"emu_{c}.log")
+        if os.path.exists(p):
+            rows += [json.loads(x) for x in open(p) if x.startswith("{")]
+    out = [f"# Round {rnd}: exposed communication with an EMULATED ring all-reduce (1 B200)", "",
+           "`python tools/emulated_dp.py Cn n` (DESIGN.md §5c): the comm stream runs the N = n sequence (value-wait on "
+           "the bucket's dW counter, \"all-reduce\", flag write that F_i waits on) with the all-reduce replaced by a "
+           "kernel that holds the stream for 2(n-1)/n x bucket bytes / 900 GB/s + 8 us; the engine keeps the 16-SM "
+           "NCCL reserve.  No data moves.  exposed = T(step) - T(step, zero-time comm); hidden = 1 - exposed / sum of "
+           "bucket times.  ms per captured step [backward(t); forward(t+1)], best of 3 x 20.", ""]
+    for r in rows:
+        out += [f"## {r['config']}, n = {r['emulated_n']} (sum of bucket all-reduce times "
+                f"{r['allreduce_total_ms']:.3f} ms)", "", "| schedule | ms/step | comm-off ms | exposed ms | hidden |",
+                "|---|---|---|---|---|"]
+        for s, v in r["schedules"].items():
+            out.append(f"| {s} | {v['ms']:.3f} | {v['ms_comm_off']:.3f} | {v['exposed_ms']:.3f} | "
+                       f"{v['hidden_fraction']:.3f} |")
+        out += ["", f"best ooo: {r['best_ooo']}, {r['ooo_speedup_vs_in_order']:.3f}x over in_order", ""]
+    open(os.path.join(ROOT, "profiles", f"r{rnd}_emulated_dp.md"), "w").write("\n".join(out) + "\n")
+
+
+def chain(rnd, d):
+    log = open(os.path.join(d, "trace_C2.log")).read().splitlines()
+    heads = [x for x in log if x.startswith("==")]
+    i0 = next(i for i, x in enumerate(log) if x.startswith("== forward alone"))
+    body = log[i0 + 1: i0 + 22]
+    out = [f"# Round {rnd}: chain-latency decomposition of the C2 step (1 B200)", "",
+           "`python tools/engine_trace.py C2 0` (debug build with per-task globaltimer stamps, ~5-10 % slower than the "
+           "product build).  The three launches: the backward alone (dO chain + every dW), the forward alone (F chain, "
+           "nothing to fill with), and the fused step.  Per op: dispense / input-ready / done ranges (µs from the "
+           "launch start), mean wait (dispense -> ready), mainloop (ready -> accumulator ready), epilogue (accumulator "
+           "ready -> published); \"loads\": first / last k-block landing after ready; epilogue phase clocks.", "",
+           "```"] + heads + [""] + body + ["```", "",
+           "Reading: an h×h F_i takes ≈ 10.7 µs per layer on the chain -- first k-block ≈ 1 µs after ready, the other "
+           "11 over ≈ 5 µs (0.45 µs per k-block), MMA tail 0.5 µs, epilogue loop ≈ 2.8 µs, release ≈ 1.2 µs; the fused "
+           "step ≈ backward-alone + forward-alone (F_1(t+1) waits for dW_1(t), i.e. the whole dO chain, P:84).  Same "
+           "breakdown for 128- and 192-wide tiles and an 8-stage ring (DESIGN.md §7)."]
+    open(os.path.join(ROOT, "profiles", f"r{rnd}_chain_latency.md"), "w").write("\n".join(out) + "\n")
+
+
+if __name__ == "__main__":
+    rnd, d = sys.argv[1], sys.argv[2]
+    kernels(rnd, d)
+    emulated(rnd, d)
+    chain(rnd, d)
+    print("ok")
