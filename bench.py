@@ -52,7 +52,9 @@ def parse():
                     help="N = 1: also measure exposed communication with an EMULATED ring all-reduce of this many "
                          "ranks (comm stream held for 2(n-1)/n x bucket bytes / 900 GB/s + 8 us per bucket, "
                          "16-SM NCCL reserve); 0 = off")
-    ap.add_argument("--bucket-layers", type=int, default=1)
+    ap.add_argument("--bucket-layers", type=int, default=6,
+                    help="consecutive layers per all-reduce bucket (6 = one transformer block: per-call latency; "
+                         "measured with the emulated all-reduce, DESIGN.md §5c)")
     ap.add_argument("--nccl-max-ctas", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -375,14 +377,15 @@ def main():
     if world == 1 and args.emulate_n > 1 and dt == "bf16":
         n, gbps, lat = args.emulate_n, 900.0, 8.0
         elt = 2
+        nbk = (L + args.bucket_layers - 1) // args.bucket_layers
         ar_total = sum(2.0 * (n - 1) / n * (cfg.dims[i] * cfg.dims[i + 1] + cfg.dims[i + 1]) * elt / (gbps * 1e9) * 1e3
-                       + lat * 1e-3 for i in range(L))
+                       for i in range(L)) + nbk * lat * 1e-3
         ks = sorted({0, max(1, L // 24), L // 6, L // 2, L})
         times = {}
         for label, bw, la in (("on", gbps, lat), ("off", 1e9, 0.0)):
             os.environ.update({"OOO_EMULATE_AR_N": str(n), "OOO_EMULATE_AR_GBPS": str(bw),
                                "OOO_EMULATE_AR_LAT_US": str(la)})
-            se = OooStack(cfg.dims, cfg.acts, M, W, b, dtype=dt)
+            se = OooStack(cfg.dims, cfg.acts, M, W, b, dtype=dt, bucket_layers=args.bucket_layers)
             se.forward(X, Y)
             for kind, k in [("in_order", 0)] + [("first_k", k) for k in ks]:
                 g = se.graph(X, Y, dY, kind, k)
@@ -400,6 +403,7 @@ def main():
                                      "hidden_fraction": 1.0 - max(0.0, on - off) / ar_total}
         best = min((v["ms"], key) for key, v in sweep.items() if key.startswith("first_k"))[1]
         emulated = {"n": n, "link_GBps_per_direction": gbps, "latency_us_per_bucket": lat,
+                    "bucket_layers": args.bucket_layers,
                     "note": "EMULATED all-reduce on one GPU (comm stream held for the ring time; no NCCL, no "
                             "data moved); the engine keeps the 16-SM NCCL reserve",
                     "allreduce_total_ms": ar_total, "in_order_ms": sweep["in_order(0)"]["ms"], "best": best,

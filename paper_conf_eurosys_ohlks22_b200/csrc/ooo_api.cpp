@@ -910,6 +910,13 @@ ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st)
   for (int i = 1; i <= L; ++i) fwd.push_back(unit_of(s, pl::FWD, i));
   if (s->eng_pending && env_int("OOO_FUSE", 1) == 0) OOO_TRY(engine_flush(s));   // experiments: unfused
   if (s->eng_pending) {
+    if (s->emu_n > 1) {
+      cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+      CU_TRY(cudaStreamIsCapturing(st, &cs));
+      if (cs != cudaStreamCaptureStatusActive)
+        return fail(OOO_ERR_UNSUPPORTED, "emulated all-reduce: run the fused step through ooo_graph_create "
+                                         "(an eager step with kernels on the comm stream stalls, see ooo.h)");
+    }
     // backward(t) + forward(t+1) in one launch (Fig. 4(c)); counters were
     // reset by ooo_backward.  F_i is gated on dW_i (N = 1) or on its bucket's
     // all-reduce (N > 1) and on dW_{i+1} (it reads X_{i+1}).
