@@ -195,6 +195,17 @@ ooo_status ooo_region_schedule(int32_t n_regions, const double *t_main, int32_t 
                                const int64_t *nbytes, int64_t mxm, int32_t *region_of, int32_t *order,
                                int32_t *k_pre);
 
+/* Heuristic search for reverse first-k's k (§5.1; readings in
+ * DESIGN.md Q4, parity unpinned beyond the prose): dk0 = max(1, round(L/10)),
+ * scan k = 0, dk, ... < L, then the open range (best - dk, best + dk) with dk
+ * halved, until a pass with dk == 1; ties -> smaller k; each k measured once
+ * through `throughput(k, ctx)` (higher is better; the caller times the step).
+ * visited (room for L + 1 entries, may be NULL) receives the measured ks in
+ * order, *n_visited their count.  Returns the best k, or -1 if L < 1 or
+ * throughput is NULL.  Pure host function. */
+int32_t ooo_k_search(int32_t L, double (*throughput)(int32_t k, void *ctx), void *ctx, int32_t *visited,
+                     int32_t *n_visited);
+
 /* Extra bytes kept alive by deferring dW_1..dW_k (the memory cost of
  * deferral, §3; E8 at P:352-354): sum_{i=2..k} |dZ_i|. */
 int64_t ooo_deferral_bytes(const ooo_stack_desc *d, int32_t k);

@@ -70,7 +70,7 @@ EXPORTS = [
     "ooo_schedule_order", "ooo_max_k", "ooo_deferral_bytes", "ooo_get_unique_id", "ooo_create_stack",
     "ooo_forward", "ooo_backward", "ooo_join", "ooo_graph_create", "ooo_graph_launch",
     "ooo_graph_destroy", "ooo_destroy", "ooo_tensor", "ooo_set_timing", "ooo_timing_read",
-    "ooo_engine_plan", "ooo_region_schedule", "ooo_plan_regions", "ooo_region_plan",
+    "ooo_engine_plan", "ooo_region_schedule", "ooo_plan_regions", "ooo_region_plan", "ooo_k_search",
 ]
 
 _lib = None
