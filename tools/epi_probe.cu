@@ -57,6 +57,74 @@ __global__ void __launch_bounds__(288, 1) epi(__nv_bfloat16 *out, int ldc, int t
   for (int tile = 0; tile < tiles; ++tile) {
     const uint32_t tbase = tmem + ((uint32_t)(q * 32) << 16);
     uint32_t ra[32];
+    if (MODE == 5) {
+      // 64-column chunks: warp h takes columns [128 h, 128 h + 128) as two
+      // 64-col halves; 4 KiB per-warp transpose, full 128-B row stores
+      uint8_t *sw = stg_all + warp * 2048;   // 2 KiB per warp: 32 rows x 64 B halves, two passes
+      for (int c2 = 0; c2 < 2; ++c2) {
+        const int cbase = h * 4 + c2 * 2;            // 32-col chunk index of the first half
+        uint32_t ra2[32];
+        tmem_ld32_issue(tbase + (uint32_t)(cbase * 32), ra);
+        tmem_ld32_issue(tbase + (uint32_t)((cbase + 1) * 32), ra2);
+        tmem_ld_wait(ra);
+        tmem_ld_wait(ra2);
+        uint32_t u[32];
+#pragma unroll
+        for (int i = 0; i < 16; ++i)
+          u[i] = pack_bf2(__uint_as_float(ra[2 * i]) + bias_s[cbase * 32 + 2 * i],
+                          __uint_as_float(ra[2 * i + 1]) + bias_s[cbase * 32 + 2 * i + 1]);
+#pragma unroll
+        for (int i = 0; i < 16; ++i)
+          u[16 + i] = pack_bf2(__uint_as_float(ra2[2 * i]) + bias_s[cbase * 32 + 32 + 2 * i],
+                               __uint_as_float(ra2[2 * i + 1]) + bias_s[cbase * 32 + 32 + 2 * i + 1]);
+        // two 16-row passes through a 2 KiB buffer: rows of 128 B, chunk c at c ^ (r & 7)
+        for (int pass = 0; pass < 2; ++pass) {
+          __syncwarp();
+          if ((lane >> 4) == pass) {
+            const int r = lane & 15;
+            const uint32_t rb = smem_u32(sw) + r * 128;
+#pragma unroll
+            for (int c = 0; c < 8; ++c)
+              asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(rb + ((c ^ (r & 7)) << 4)),
+                           "r"(u[4 * c]), "r"(u[4 * c + 1]), "r"(u[4 * c + 2]), "r"(u[4 * c + 3]) : "memory");
+          }
+          __syncwarp();
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const int r = (lane >> 3) + 4 * k, c = lane & 7;
+            uint32_t x, y, z, w;
+            asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(x), "=r"(y), "=r"(z), "=r"(w)
+                         : "r"(smem_u32(sw) + r * 128 + ((c ^ (r & 7)) << 4)) : "memory");
+            const int col0 = (tile % 3) * 256 + cbase * 32;
+            *reinterpret_cast<uint4 *>(out + (size_t)(row0 + pass * 16 + r) * ldc + col0 + c * 8) = make_uint4(x, y, z, w);
+          }
+        }
+      }
+      asm volatile("bar.sync 1, 256;" ::: "memory");
+      continue;
+    }
+    if (MODE == 6) {
+      // two TMEM loads in flight: chunk c+2 and c+4 issued while c is processed
+      uint32_t rb[32];
+      tmem_ld32_issue(tbase + (uint32_t)(h * 32), ra);
+      tmem_ld32_issue(tbase + (uint32_t)((h + 2) * 32), rb);
+#pragma unroll
+      for (int cc = 0; cc < 4; ++cc) {
+        const int c = h + 2 * cc;
+        const int col0 = (tile % 3) * 256 + c * 32;
+        uint32_t (&cur)[32] = (cc & 1) ? rb : ra;
+        tmem_ld_wait(cur);
+        float v[32];
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(cur[i]) + bias_s[c * 32 + i];
+        if (cc + 2 < 4) tmem_ld32_issue(tbase + (uint32_t)((c + 4) * 32), cur);
+        uint32_t u[16];
+        pack32(v, u);
+        store32_rows_packed(out, ldc, stg, lane, u, col0, row0, 1 << 30);
+      }
+      asm volatile("bar.sync 1, 256;" ::: "memory");
+      continue;
+    }
     tmem_ld32_issue(tbase + (uint32_t)(h * 32), ra);
     for (int c = h; c < 8; c += 2) {
       const int col0 = (tile % 3) * 256 + c * 32;
@@ -115,12 +183,13 @@ int main() {
   ((Enc)fn)(&om, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, out, dims, str, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
             CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   const int tiles = 200;
-  void (*ks[10])(__nv_bfloat16 *, int, int, long long *, CUtensorMap) = {epi<0, false>, epi<1, false>, epi<2, false>, epi<3, false>, epi<4, false>,
-                                                                       epi<0, true>, epi<1, true>, epi<2, true>, epi<3, true>, epi<4, true>};
-  const char *names[5] = {"TMEM ld + bias + pack, no stores", "+ smem-transpose stores", "same with stores, no-TMEM math",
-                          "TMA (bulk tensor) stores", "direct per-row st.global.v4 (no smem)"};
-  for (int m = 0; m < 10; ++m) {
-    if (m == 5) printf("-- with concurrent MMAs into the other TMEM half:\n");
+  void (*ks[14])(__nv_bfloat16 *, int, int, long long *, CUtensorMap) = {epi<0, false>, epi<1, false>, epi<2, false>, epi<3, false>, epi<4, false>, epi<5, false>, epi<6, false>,
+                                                                       epi<0, true>, epi<1, true>, epi<2, true>, epi<3, true>, epi<4, true>, epi<5, true>, epi<6, true>};
+  const char *names[7] = {"TMEM ld + bias + pack, no stores", "+ smem-transpose stores", "same with stores, no-TMEM math",
+                          "TMA (bulk tensor) stores", "direct per-row st.global.v4 (no smem)",
+                          "64-col chunks, full 128-B row stores", "smem-transpose stores, 2 TMEM loads in flight"};
+  for (int m = 0; m < 14; ++m) {
+    if (m == 7) printf("-- with concurrent MMAs into the other TMEM half:\n");
     ks[m]<<<148, 288>>>(out, ldc, tiles, d, om);
     cudaError_t e = cudaDeviceSynchronize();
     long long h[148];
@@ -128,7 +197,7 @@ int main() {
     double mm = 0;
     for (int i = 0; i < 148; ++i) mm += h[i];
     mm /= 148;
-    printf("%-40s %8.0f cycles per 128x256 tile  (%s)\n", names[m % 5], mm / tiles, cudaGetErrorString(e));
+    printf("%-40s %8.0f cycles per 128x256 tile  (%s)\n", names[m % 7], mm / tiles, cudaGetErrorString(e));
   }
   return 0;
 }
