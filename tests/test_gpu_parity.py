@@ -349,3 +349,30 @@ def test_bf16_144_layer_full_configs_end_to_end(cfg):
     base = case.run(stk, "in_order", 0)
     assert torch.equal(base["raw"], out["raw"])
     stk.close()
+
+
+def test_regions_error_paths():
+    """OOO_SCHED_REGIONS without a plan -> OOO_ERR_STATE; planning an fp32
+    stack -> OOO_ERR_UNSUPPORTED; a plan is discarded by nothing but a new
+    plan, and planning leaves the stack needing a forward (OOO_ERR_STATE)."""
+    from paper_conf_eurosys_ohlks22_b200._lib import OooError
+    case = Case([256, 256, 256, 256], ["gelu", "id", "id"], 256, "bf16")
+    stk = case.stack()
+    X, dY = to_dev(case.X, "bf16"), to_dev(case.dY, "bf16")
+    stk.forward(X)
+    with pytest.raises(OooError, match="STATE"):
+        stk.backward(dY, "regions")
+    stk.forward(X)
+    stk.plan_regions(region_layers=1)
+    with pytest.raises(OooError, match="STATE"):
+        stk.backward(dY, "regions")          # the profiling launches overwrote the activations
+    stk.forward(X)
+    stk.backward(dY, "regions")
+    stk.join()
+    stk.close()
+    c32 = Case([256, 256, 256], ["relu", "id"], 32, "fp32")
+    s32 = c32.stack()
+    s32.forward(to_dev(c32.X, "fp32"))
+    with pytest.raises(OooError, match="UNSUPPORTED"):
+        s32.plan_regions()
+    s32.close()
