@@ -1,7 +1,7 @@
 """Single-GPU multi-stream ooo with Algorithm 1 regions (§4.1) vs reverse
 first-k and in-order, one captured step each (tuning / evidence tool).
 
-    python tools/regions_bench.py C2 [region_layers ...]
+    python tools/regions_bench.py C2 [region_layers ...] [--reps=N]
 Prints one JSON line per config: profiling (planning) time, plan summary and
 ms/step of regions / first_k(k) / in_order.
 """
@@ -33,7 +33,8 @@ def timed(g, stream, steps=30, reps=3):
 
 
 cfg = configs.get(sys.argv[1] if len(sys.argv) > 1 else "C2")
-rls = [int(a) for a in sys.argv[2:]] or [6]
+rls = [int(a) for a in sys.argv[2:] if not a.startswith("--")] or [6]
+REPS = next((int(a[7:]) for a in sys.argv[2:] if a.startswith("--reps=")), 1)
 dev = torch.device("cuda")
 stream = torch.cuda.current_stream()
 W, b = synth.weights_torch(cfg.dims, cfg.acts, cfg.dtype, dev)
@@ -48,7 +49,7 @@ for kind, k in (("in_order", 0), ("first_k", 0), ("first_k", cfg.L // 6)):
     g.close()
 for rl in rls:
     t0 = time.time()
-    plan = stk.plan_regions(region_layers=rl, reps=1)
+    plan = stk.plan_regions(region_layers=rl, reps=REPS)
     t_plan = time.time() - t0
     stk.forward(X, Y)
     g = stk.graph(X, Y, dY, "regions", 0)
