@@ -93,6 +93,9 @@ __device__ __forceinline__ void etrace_gt(int, int) {}
 __device__ __forceinline__ void ktrace(int, int, int) {}
 #endif
 
+#ifndef OOO_ENGINE_PDL
+#define OOO_ENGINE_PDL 1
+#endif
 #ifndef OOO_EPI_WARPS
 #define OOO_EPI_WARPS 8
 #endif
@@ -931,24 +934,29 @@ cudaError_t launch_engine(int cg, const Params &p, const CUtensorMap *tmY, const
   cudaLaunchConfig_t cfg = {};
   cfg.blockDim = dim3(kThreads, 1, 1);
   cfg.stream = stream;
-  cudaLaunchAttribute attr[2];
+  cudaLaunchAttribute attr[3];
   attr[0].id = cudaLaunchAttributePriority;
   attr[0].val.priority = priority;
+  // programmatic dependent launch: the prologue (TMEM allocation, barrier
+  // setup, cluster sync) overlaps the preceding kernel (the seed); every
+  // read of its data follows griddepcontrol.wait (pdl_wait)
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = OOO_ENGINE_PDL;
   if (cg == 2) {
     cfg.gridDim = dim3((ctas / 2) * 2, 1, 1);   // whole CTA pairs
     cfg.dynamicSmemBytes = Cfg<2>::SMEM;
-    attr[1].id = cudaLaunchAttributeClusterDimension;
-    attr[1].val.clusterDim.x = 2;
-    attr[1].val.clusterDim.y = 1;
-    attr[1].val.clusterDim.z = 1;
+    attr[2].id = cudaLaunchAttributeClusterDimension;
+    attr[2].val.clusterDim.x = 2;
+    attr[2].val.clusterDim.y = 1;
+    attr[2].val.clusterDim.z = 1;
     cfg.attrs = attr;
-    cfg.numAttrs = 2;
+    cfg.numAttrs = 3;
     return cudaLaunchKernelEx(&cfg, engine_kernel<2>, *tmY, *tmDX, p);
   }
   cfg.gridDim = dim3(ctas, 1, 1);
   cfg.dynamicSmemBytes = Cfg<1>::SMEM;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = 2;
   return cudaLaunchKernelEx(&cfg, engine_kernel<1>, *tmY, *tmDX, p);
 }
 

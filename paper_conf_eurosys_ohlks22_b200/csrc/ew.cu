@@ -71,6 +71,9 @@ __global__ void __launch_bounds__(32 * kSeedTY) seed_kernel(const T *__restrict_
                                                    int act, T *__restrict__ dz,
                                                    float *__restrict__ dbpart, int M, int N, int bm) {
   constexpr int VEC = V<T>::N;
+  // the engine launched after the seed may start its prologue now (it reads
+  // dZ_L only after griddepcontrol.wait, i.e. after this grid completes)
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   __shared__ float red[kSeedTY][32 * VEC];
   const int tx = threadIdx.x, ty = threadIdx.y;
   const int col = (blockIdx.y * 32 + tx) * VEC;
