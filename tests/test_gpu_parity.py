@@ -376,3 +376,34 @@ def test_regions_error_paths():
     with pytest.raises(OooError, match="UNSUPPORTED"):
         s32.plan_regions()
     s32.close()
+
+
+# ------------------------------------------------------------------ degenerate shapes
+@pytest.mark.parametrize("dtype,need_dx", [("bf16", False), ("bf16", True), ("fp32", False), ("fp32", True)])
+def test_single_layer_stack_all_schedules(dtype, need_dx):
+    """L = 1: the step is the seed, dW_1 (and dO_1 with input grad) and F_1;
+    every schedule degenerates to the same op list and must be bit-exact."""
+    case = Case([320, 192], ["gelu"], 136, dtype, need_dx=need_dx)
+    ref = case.oracle(1)
+    stk = case.stack()
+    base = None
+    for kind, k in [("in_order", 0), ("first_k", 0), ("first_k", 1)]:
+        out = case.run(stk, kind, k, graph=(dtype == "bf16" and kind == "first_k" and k == 1))
+        _check(max_err(out, ref), BF16_TOL if dtype == "bf16" else FP32_TOL)
+        if base is None:
+            base = out["raw"]
+        assert torch.equal(out["raw"], base), (kind, k)
+    stk.close()
+
+
+def test_bf16_narrowest_and_widest_widths():
+    """The 64-wide minimum next to a 4096-wide FFN layer (widths at both ends
+    of the tile plans), ragged token tail, with input grad."""
+    case = Case([64, 4096, 64, 128], ["gelu", "relu", "id"], 200, "bf16", need_dx=True)
+    ref = case.oracle(2)
+    stk = case.stack()
+    out = case.run(stk, "first_k", 2)
+    _check(max_err(out, ref), BF16_TOL)
+    inorder = case.run(stk, "in_order", 0)
+    assert torch.equal(inorder["raw"], out["raw"])
+    stk.close()

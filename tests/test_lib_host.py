@@ -121,3 +121,15 @@ def test_product_k_search_matches_oracle_reading():
         if L > 1:
             peak = rng.randint(0, L - 1)
             assert search_k(L, lambda k: -abs(k - peak))[0] == peak
+
+
+def test_degenerate_sizes_without_gpu(lib):
+    """Empty token batch -> UNSUPPORTED (nothing to compute, header: tokens >= 1);
+    a one-layer stack's schedule is the lone dW_1 (dO_1 only with input grad)."""
+    for t in (0, -8):
+        with pytest.raises(_lib.OooError) as e:
+            stack.query_sizes([64, 64], ["id"], t)
+        assert e.value.status == 2
+    for kind, k in [("in_order", 0), ("first_k", 0), ("first_k", 1), ("first_k", 5)]:
+        assert stack.schedule_order(1, kind, k) == [-1]
+        assert sorted(stack.schedule_order(1, kind, k, need_input_grad=True)) == [-1, 1]
