@@ -106,6 +106,9 @@ constexpr int kThreads = 64 + kEpiThreads;
 constexpr int kMaxBN = 256;
 constexpr int STG_BYTES = kEpiWarps * 2048;
 constexpr int Q = 4;                                 // task ring depth
+#ifndef OOO_EARLY_WAIT
+#define OOO_EARLY_WAIT 0   // experiment: wait for k-block kb + 1 between kb's 2nd and 3rd MMA
+#endif
 #ifndef OOO_TMA_STORE
 #define OOO_TMA_STORE 0
 #endif
@@ -609,6 +612,37 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint64_t astep = a_mn ? 128u : 2u, bstep = b_mn ? 128u : 2u;
         int s = it % C::STAGES;
         uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;
+#if OOO_EARLY_WAIT
+        if (CG == 2) {
+          // the barrier wait (+ fence) of k-block kb + 1 runs while kb's last
+          // two MMAs execute, so the issuer's per-k-block overhead is covered
+          // by queued tensor work; kb's stage is released right after
+          mbar_wait_b(bar_full + 8 * s, ph);
+          fence_after();
+          for (int kb = 0; kb < T.nkb; ++kb) {
+            const uint64_t soff = (uint64_t)(s * (C::STAGE >> 4));
+            const uint64_t ad = a0 + soff, bd = b0 + soff;
+            umma_bf16_pair(dtm, ad, bd, ID, kb != 0 ? 1u : 0u);
+            umma_bf16_pair(dtm, ad + astep, bd + bstep, ID, 1u);
+            const int s_cur = s;
+            if (++s == C::STAGES) {
+              s = 0;
+              ph ^= 1u;
+            }
+            if (kb + 1 < T.nkb) {
+              mbar_wait_b(bar_full + 8 * s, ph);
+              fence_after();
+            }
+            umma_bf16_pair(dtm, ad + 2 * astep, bd + 2 * bstep, ID, 1u);
+            umma_bf16_pair(dtm, ad + 3 * astep, bd + 3 * bstep, ID, 1u);
+            umma_commit_pair(bar_empty + 8 * s_cur);
+          }
+          it += T.nkb;
+          umma_commit_pair(bar_tfull + 8 * acc);
+          etrace_gt(t, 5);
+          continue;
+        }
+#endif
         for (int kb = 0; kb < T.nkb; ++kb) {
           ktrace(t, kb, 2);
           mbar_wait_b(bar_full + 8 * s, ph);
