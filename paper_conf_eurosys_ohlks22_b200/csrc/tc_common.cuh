@@ -311,6 +311,49 @@ __device__ __forceinline__ void stage_store(const CUtensorMap *map, uint32_t buf
   __syncwarp();
   if (lane == 0) tma_store_2d(map, buf, col0, row0);
 }
+#ifndef OOO_STG256
+#define OOO_STG256 1   // 32-B global stores (STG.256), 2 lanes per 64-B row segment (0: 16-B stores)
+#endif
+// Read back a warp's 32 x 32 bf16 transpose buffer (row r at buf + 64 r,
+// 16-B chunk c at (c ^ ((r >> 1) & 3)) << 4) and store it row-major.
+__device__ __forceinline__ void readback_store32(__nv_bfloat16 *g, int ldc, uint32_t buf, int lane, int col0,
+                                                 int row0, int M) {
+#if OOO_STG256
+  const int c = (lane & 1) * 2;
+#pragma unroll
+  for (int k = 0; k < 2; ++k) {
+    const int r = (lane >> 1) + 16 * k;
+    uint32_t x0, y0, z0, w0, x1, y1, z1, w1;
+    asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(x0), "=r"(y0), "=r"(z0), "=r"(w0)
+                 : "r"(buf + r * 64 + ((c ^ ((r >> 1) & 3)) << 4))
+                 : "memory");
+    asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(x1), "=r"(y1), "=r"(z1), "=r"(w1)
+                 : "r"(buf + r * 64 + (((c + 1) ^ ((r >> 1) & 3)) << 4))
+                 : "memory");
+    const int grow = row0 + r;
+    if (grow < M)
+      asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(
+                       g + (size_t)grow * ldc + col0 + c * 8),
+                   "r"(x0), "r"(y0), "r"(z0), "r"(w0), "r"(x1), "r"(y1), "r"(z1), "r"(w1)
+                   : "memory");
+  }
+#else
+  const int c = lane & 3;
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const int r = (lane >> 2) + 8 * k;
+    uint32_t x, y, z, w;
+    asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(x), "=r"(y), "=r"(z), "=r"(w)
+                 : "r"(buf + r * 64 + ((c ^ ((r >> 1) & 3)) << 4))
+                 : "memory");
+    const int grow = row0 + r;
+    if (grow < M) *reinterpret_cast<uint4 *>(g + (size_t)grow * ldc + col0 + c * 8) = make_uint4(x, y, z, w);
+  }
+#endif
+}
 // Store one warp's 32 rows x 32 columns (bf16, lane = row) to a row-major
 // global tensor through a 2 KiB per-warp smem transpose: lanes write their
 // row (4 x 16 B, 64B-swizzled -> conflict-free), then read back so that
@@ -330,18 +373,7 @@ __device__ __forceinline__ void store32_rows(__nv_bfloat16 *g, int ldc, uint32_t
                  : "memory");
   }
   __syncwarp();
-  const int c = lane & 3;
-#pragma unroll
-  for (int k = 0; k < 4; ++k) {
-    const int r = (lane >> 2) + 8 * k;
-    uint32_t x, y, z, w;
-    asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
-                 : "=r"(x), "=r"(y), "=r"(z), "=r"(w)
-                 : "r"(buf + r * 64 + ((c ^ ((r >> 1) & 3)) << 4))
-                 : "memory");
-    const int grow = row0 + r;
-    if (grow < M) *reinterpret_cast<uint4 *>(g + (size_t)grow * ldc + col0 + c * 8) = make_uint4(x, y, z, w);
-  }
+  readback_store32(g, ldc, buf, lane, col0, row0, M);
 }
 // store32_rows for values already packed to bf16 pairs (u[j] = columns 2j, 2j+1).
 __device__ __forceinline__ void store32_rows_packed(__nv_bfloat16 *g, int ldc, uint32_t buf, int lane,
@@ -356,18 +388,7 @@ __device__ __forceinline__ void store32_rows_packed(__nv_bfloat16 *g, int ldc, u
                  : "memory");
   }
   __syncwarp();
-  const int c = lane & 3;
-#pragma unroll
-  for (int k = 0; k < 4; ++k) {
-    const int r = (lane >> 2) + 8 * k;
-    uint32_t x, y, z, w;
-    asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];"
-                 : "=r"(x), "=r"(y), "=r"(z), "=r"(w)
-                 : "r"(buf + r * 64 + ((c ^ ((r >> 1) & 3)) << 4))
-                 : "memory");
-    const int grow = row0 + r;
-    if (grow < M) *reinterpret_cast<uint4 *>(g + (size_t)grow * ldc + col0 + c * 8) = make_uint4(x, y, z, w);
-  }
+  readback_store32(g, ldc, buf, lane, col0, row0, M);
 }
 __device__ __forceinline__ void pack32(const float (&f)[32], uint32_t (&u)[16]) {
 #pragma unroll
