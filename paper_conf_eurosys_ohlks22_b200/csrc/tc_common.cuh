@@ -357,8 +357,8 @@ __device__ __forceinline__ void readback_store32(__nv_bfloat16 *g, int ldc, uint
 // Store one warp's 32 rows x 32 columns (bf16, lane = row) to a row-major
 // global tensor through a 2 KiB per-warp smem transpose: lanes write their
 // row (4 x 16 B, 64B-swizzled -> conflict-free), then read back so that
-// each group of 4 lanes owns one 64-B row segment -> fully coalesced
-// st.global.v4.  No async engine involved (TMA bulk stores would queue
+// each pair of lanes (4 lanes with OOO_STG256=0) owns one 64-B row segment
+// -> fully coalesced st.global.v8 (v4).  No async engine involved (TMA bulk stores would queue
 // behind the producer's TMA loads), so nothing to wait for.
 __device__ __forceinline__ void store32_rows(__nv_bfloat16 *g, int ldc, uint32_t buf, int lane,
                                              const float (&v)[32], int col0, int row0, int M) {
