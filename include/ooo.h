@@ -75,7 +75,7 @@
 extern "C" {
 #endif
 
-#define OOO_ABI_VERSION 1
+#define OOO_ABI_VERSION 2
 #define OOO_UNIQUE_ID_BYTES 128
 
 typedef struct ooo_stack ooo_stack;   /* opaque */
@@ -140,11 +140,21 @@ typedef struct {
   int32_t world_size;          /* N >= 1 */
   int32_t rank;                /* 0 <= rank < N */
   const void *nccl_unique_id;  /* OOO_UNIQUE_ID_BYTES from ooo_get_unique_id on rank 0, shared by
-                                  the caller (e.g. torch.distributed broadcast); NULL iff N == 1 */
+                                  the caller (e.g. torch.distributed broadcast).  Required for N > 1.
+                                  N == 1: NULL = no communicator; non-NULL = a ONE-rank NCCL
+                                  communicator, so a single GPU runs the whole N > 1 data plane
+                                  (per-bucket ncclAllReduce on the comm stream, F_i gated on the
+                                  all-reduce flags, the SM reserve) -- the all-reduce of one rank is
+                                  the identity, so results equal the non-communicating stack's. */
   int32_t comm_enabled;        /* 1: all-reduce each bucket.  0: comm-off control -- same streams,
                                   events and kernels, the all-reduce is skipped (exposed-comm
                                   measurement); gradients are then the local shard's. */
   int32_t nccl_max_ctas;       /* > 0: ncclConfig_t.maxCTAs (bounds SMs taken from the GEMMs); 0 = NCCL default */
+  int32_t wait_timeout_ms;     /* bound of every wait inside the bf16 engine kernel (dependency
+                                  counters; F_i's wait for its bucket's all-reduce, which peer ranks
+                                  drive): beyond it the kernel traps and the CUDA context reports an
+                                  error instead of hanging.  <= 0 = default: 4000 ms for a stack
+                                  without a communicator, 120000 ms with one. */
 } ooo_stack_desc;
 
 /* ---------------------------------------------------------------- info */
@@ -227,19 +237,27 @@ ooo_status ooo_get_unique_id(void *out /* OOO_UNIQUE_ID_BYTES */);
 
 /* ------------------------------------------------------------- the path */
 /* Validates, plans the workspace, encodes TMA descriptors, creates the
- * priority streams / events and (N > 1) the NCCL communicator -- collective
- * over ranks.  Uses the current CUDA device. */
+ * priority streams / events and (nccl_unique_id given) the NCCL communicator
+ * -- collective over ranks.  With a communicator it then warms NCCL up: it
+ * zeroes `grads` and all-reduces every bucket once (NCCL connects its
+ * channels lazily on first use; a cold first call inside a training step
+ * could take longer than the engine's wait bound) and waits for it.  Uses
+ * the current CUDA device. */
 ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out);
 
 /* F_1..F_L: X [M][d_0] (device, dtype) -> Y [M][d_L] (device, dtype).
+ * X and Y (and dY, dX of ooo_backward / ooo_graph_create) must be 32-byte
+ * aligned for bf16 stacks (the engine stores 32-byte row vectors), 16-byte for
+ * fp32; OOO_ERR_INVALID_ARGUMENT otherwise.
  * X is copied into the stack's X_1 store; Y is written by F_L.  If a backward
  * is pending, F_i first waits for layer i's synchronised gradient (and for
- * dW_{i+1}, which still reads X_{i+1}).  With a communicating stack (N > 1,
- * or the emulated all-reduce OOO_EMULATE_AR_N), run training steps through
- * ooo_graph_create / ooo_graph_launch: an EAGER fused step whose comm stream
- * holds kernels behind the per-bucket value-waits was observed to stall on
- * B200 (the emulated all-reduce; the graph-launched step is unaffected and is
- * what the tests and bench.py run). */
+ * dW_{i+1}, which still reads X_{i+1}).  A communicating bf16 stack (a NCCL
+ * communicator, or the emulated all-reduce OOO_EMULATE_AR_N) runs its fused
+ * training steps only through ooo_graph_create / ooo_graph_launch: an eager
+ * ooo_forward after ooo_backward returns OOO_ERR_UNSUPPORTED (an EAGER fused
+ * step whose comm stream holds kernels behind the per-bucket value-waits was
+ * observed to stall on B200; the graph-launched step is unaffected).  Eager
+ * ooo_backward + ooo_join (no forward in the same launch) is allowed. */
 ooo_status ooo_forward(ooo_stack *s, const void *X, void *Y, void *stream /* cudaStream_t */);
 
 /* Backward of the last forward: dY [M][d_L] (device, dtype).  dX [M][d_0]
@@ -249,6 +267,16 @@ ooo_status ooo_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void *dX
 
 /* `stream` waits for all outstanding backward work, all-reduces included. */
 ooo_status ooo_join(ooo_stack *s, void *stream);
+
+/* S[dW] of every bucket back to back on the stack's comm stream and
+ * communicator, no compute (collective: every rank calls it): the
+ * stand-alone all-reduce time the hidden fraction is measured against
+ * (SURVEY §8d AR_ms), with exactly the buckets, sizes, dtype and
+ * communicator a training step uses.  `grads` is summed in place again
+ * (its values change; run a backward afterwards for valid gradients).
+ * Buckets are issued from the last (layer L) to the first.  `stream` waits
+ * for the all-reduces.  OOO_ERR_STATE for a stack without communicator. */
+ooo_status ooo_allreduce_buckets(ooo_stack *s, void *stream);
 
 /* Plans OOO_SCHED_REGIONS (single-GPU multi-stream ooo, §4.1) for
  * this stack, by the paper's steps 1-5:
@@ -315,6 +343,20 @@ typedef struct {
 } ooo_launch_record;
 ooo_status ooo_set_timing(ooo_stack *s, int32_t enable);
 ooo_status ooo_timing_read(ooo_stack *s, ooo_launch_record *out, int32_t cap, int32_t *n);
+
+/* Per-launch timing of a captured step over a whole timed region.  For a
+ * graph captured while the stack's timing was on: the next `slots` calls of
+ * ooo_graph_launch each record into their own set of CUDA events (the graph's
+ * event-record nodes are re-pointed before each launch, host side; the
+ * launches stay back to back on the caller's stream), later launches use the
+ * stack's events again.  OOO_ERR_STATE if the graph has no timing brackets. */
+ooo_status ooo_graph_set_timing_slots(ooo_graph *g, int32_t slots);
+/* After those launches completed: the records of every timed launch, launch
+ * after launch (*per_launch records each, in capture order), `ms` measured in
+ * that launch; start_ms relative to the first launch's first record.
+ * *n = total records (only the first `cap` are written). */
+ooo_status ooo_graph_timing_read(ooo_graph *g, ooo_launch_record *out, int32_t cap, int32_t *n,
+                                 int32_t *per_launch);
 
 #ifdef __cplusplus
 }

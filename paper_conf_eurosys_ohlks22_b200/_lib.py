@@ -42,6 +42,7 @@ class StackDesc(ctypes.Structure):
         ("nccl_unique_id", c_void_p),
         ("comm_enabled", c_int32),
         ("nccl_max_ctas", c_int32),
+        ("wait_timeout_ms", c_int32),
     ]
 
 
@@ -71,6 +72,7 @@ EXPORTS = [
     "ooo_forward", "ooo_backward", "ooo_join", "ooo_graph_create", "ooo_graph_launch",
     "ooo_graph_destroy", "ooo_destroy", "ooo_tensor", "ooo_set_timing", "ooo_timing_read",
     "ooo_engine_plan", "ooo_region_schedule", "ooo_plan_regions", "ooo_region_plan", "ooo_k_search",
+    "ooo_allreduce_buckets", "ooo_graph_set_timing_slots", "ooo_graph_timing_read",
 ]
 
 _lib = None
@@ -128,6 +130,8 @@ def load() -> ctypes.CDLL:
     lib.ooo_backward.argtypes = [c_void_p, c_void_p, Schedule, c_void_p, c_void_p]
     lib.ooo_join.restype = S
     lib.ooo_join.argtypes = [c_void_p, c_void_p]
+    lib.ooo_allreduce_buckets.restype = S
+    lib.ooo_allreduce_buckets.argtypes = [c_void_p, c_void_p]
     lib.ooo_graph_create.restype = S
     lib.ooo_graph_create.argtypes = [c_void_p, c_void_p, c_void_p, c_void_p, Schedule, c_void_p,
                                      POINTER(c_void_p)]
@@ -141,6 +145,11 @@ def load() -> ctypes.CDLL:
     lib.ooo_tensor.argtypes = [c_void_p, c_int32, c_int32, POINTER(c_void_p), POINTER(c_int64)]
     lib.ooo_set_timing.restype = S
     lib.ooo_set_timing.argtypes = [c_void_p, c_int32]
+    lib.ooo_graph_set_timing_slots.restype = S
+    lib.ooo_graph_set_timing_slots.argtypes = [c_void_p, c_int32]
+    lib.ooo_graph_timing_read.restype = S
+    lib.ooo_graph_timing_read.argtypes = [c_void_p, POINTER(LaunchRecord), c_int32, POINTER(c_int32),
+                                          POINTER(c_int32)]
     lib.ooo_timing_read.restype = S
     lib.ooo_timing_read.argtypes = [c_void_p, POINTER(LaunchRecord), c_int32, POINTER(c_int32)]
     _lib = lib

@@ -24,7 +24,7 @@ LIB = os.path.join(LIBDIR, "libooo.so")
 OBJDIR = os.path.join(PKG, "build_obj")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-SOURCES = ["gemm_tc.cu", "engine.cu", "gemm_simt.cu", "ew.cu", "ooo_api.cpp", "nccl_dyn.cpp", "planner.cpp", "regions.cpp"]
+SOURCES = ["engine.cu", "gemm_simt.cu", "ew.cu", "ooo_api.cpp", "nccl_dyn.cpp", "planner.cpp", "regions.cpp"]
 
 
 def _nvcc() -> str:
@@ -83,7 +83,7 @@ def build(force: bool = False, verbose: bool = True, trace: bool = False, varian
 
     def compile_one(src):
         obj = os.path.join(objdir, src + ".o")
-        cmd = [nvcc] + flags + ["-Xptxas", "-v"] * (src == "gemm_tc.cu" and verbose is None) + \
+        cmd = [nvcc] + flags + ["-Xptxas", "-v"] * (src == "engine.cu" and verbose is None) + \
               ["-c", os.path.join(CSRC, src), "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:

@@ -118,7 +118,11 @@ constexpr int Q = 4;                                 // task ring depth
 // completion (cp.async.bulk.wait_group 0) before the release.
 constexpr bool kTmaStore = OOO_TMA_STORE != 0;
 constexpr uint32_t TMEM_COLS = 512;
-constexpr uint64_t kTimeoutNs = 4000000000ull;
+// Bound of every wait (ns), from Params::timeout_ns (the stack's
+// wait_timeout_ms): a wait that exceeds it traps (the launch fails with an
+// error) instead of hanging.  Written by thread 0 before the prologue's
+// barrier; every wait follows that barrier.
+__shared__ uint64_t s_timeout_ns;
 
 template <int CG> struct Cfg {
   static constexpr int B_BYTES = (kMaxBN / CG) * BK * 2;   // this CTA's share of B
@@ -174,7 +178,7 @@ __device__ __forceinline__ void mbar_wait_b(uint32_t bar, uint32_t parity) {
   for (uint32_t n = 1; !mbar_try_wait(bar, parity); ++n) {
     if ((n & 1023u) == 0) {
       if (t0 == 0) t0 = gtimer();
-      else if (gtimer() - t0 > kTimeoutNs) __trap();
+      else if (gtimer() - t0 > s_timeout_ns) __trap();
     }
   }
 }
@@ -190,7 +194,7 @@ __device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
     if (OOO_EPI_SLEEP_NS > 0) __nanosleep(OOO_EPI_SLEEP_NS);
     if ((n & 255u) == 0) {
       if (t0 == 0) t0 = gtimer();
-      else if (gtimer() - t0 > kTimeoutNs) __trap();
+      else if (gtimer() - t0 > s_timeout_ns) __trap();
     }
   }
 }
@@ -240,14 +244,15 @@ __device__ __forceinline__ int ld_relaxed(const int32_t *p) {
 __device__ __forceinline__ void red_release_add(int32_t *p, int v) {
   asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
-// Wait until *p >= target.  A dependency that is not met within 4 s means a
-// broken schedule: trap (the launch fails with an error) instead of hanging.
+// Wait until *p >= target.  A dependency that is not met within the bound
+// means a broken schedule or a stalled peer rank: trap (the launch fails with
+// an error) instead of hanging.
 __device__ __forceinline__ void wait_ge(const int32_t *p, int target) {
   if (ld_relaxed(p) < target) {
     const uint64_t t0 = gtimer();
     while (ld_relaxed(p) < target) {
       __nanosleep(32);
-      if (gtimer() - t0 > kTimeoutNs) __trap();
+      if (gtimer() - t0 > s_timeout_ns) __trap();
     }
   }
   (void)ld_acquire(p);   // one acquire orders the producer tiles' stores before our reads
@@ -466,6 +471,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   const bool leader = rank == 0;
 
   if (warp == 0 && lane == 0) {
+    s_timeout_ns = p.timeout_ns;
     for (int s = 0; s < C::STAGES; ++s) {
       mbar_init(bar_full + 8 * s, 1);           // leader's expect_tx arrival (+ the CTAs' bytes)
       mbar_init(bar_empty + 8 * s, 1);          // leader's MMA commit

@@ -88,6 +88,7 @@ struct Params {
   int32_t a_rows;          // rows of the row-major A box of F_i / dO_i tiles: 128, or M rounded
                            // up to 8 when all tokens fit one 128-row tile (1-CTA tiles): the
                            // MMA's rows beyond it read stale smem and are never stored
+  uint64_t timeout_ns;     // bound of every in-kernel wait (trap beyond it)
   const CUtensorMap *maps;
   int32_t *ctr;            // counter array base
   const LayerDev *layers;  // index i-1

@@ -1,4 +1,4 @@
-// fp32 SIMT GEMMs with the same fused epilogues as gemm_tc.cu, for the fp32
+// fp32 SIMT GEMMs with the fused epilogues of kernels.h (EpiArgs), for the fp32
 // mode (BASELINE config 0: 4-layer MLP width 256, batch 32).  Exact fp32 FFMA:
 // TF32 tensor cores would round operands to 10 mantissa bits and miss the
 // 1e-4 fp32 parity bar (reading Q10).  The fp32 config is launch-bound (each

@@ -18,7 +18,8 @@ enum Epi : int { EPI_FWD = 0, EPI_DGRAD = 1, EPI_WGRAD = 2 };
 constexpr int kTcBM = 128;     // tcgen05 path (bf16)
 constexpr int kSimtBM = 64;    // SIMT path (fp32)
 
-// Epilogue arguments shared by the tensor-core and SIMT GEMMs.
+// Epilogue arguments of the per-layer fp32 SIMT GEMMs (the bf16 engine has its
+// own task descriptors, engine.h).
 //   FWD  : v = acc + bias[n];  z_out[m][n] = st(v) (optional);
 //          x_out[m][n] = st(act(ld(st(v))))                       (layer forward F_i)
 //   DGRAD: v = acc * act'(zin[m][n]) (act' = 1 for ACT_ID, zin unused);
@@ -47,18 +48,6 @@ struct LaunchCtx {
   int priority;
   bool pdl = false;   // programmatic dependent launch (the kernel must griddepcontrol.wait)
 };
-
-// ---- tcgen05 bf16 GEMM (gemm_tc.cu).  A is M x K, B is K x N (logical).
-// a_mn / b_mn: operand stored MN-major (true) or K-major (false) -- see the
-// tensor-map builders below.  Returns a CUDA error code.
-// Persistent: `ctas` CTAs walk the ceil(M/128) x ceil(N/bn) x splits work units.
-// tmZ / tmX: bf16 output maps (box {64 cols, 32 rows}, 128B swizzle) for the
-// Z / X outputs of F_i, the dZ (or dX) output of dO_i and the bucket of dW_i.
-cudaError_t launch_gemm_tc(int epi, int bn, const CUtensorMap *tmA, const CUtensorMap *tmB,
-                           const CUtensorMap *tmZ, const CUtensorMap *tmX, const EpiArgs &args, int ctas,
-                           const LaunchCtx &ctx);
-int gemm_tc_smem_bytes(int bn);
-cudaError_t gemm_tc_init();   // sets max dynamic smem on every instantiation
 
 // ---- fp32 SIMT GEMM (gemm_simt.cu): generic strides.
 //   A(m, k) = A[m * sam + k * sak];  B(k, n) = B[k * sbk + n * sbn]

@@ -104,56 +104,9 @@ struct Plan {
 
 constexpr int kSMs = 148;
 
-// Tile plan of one tcgen05 GEMM (persistent kernel, 128 x BN tiles).  Cost
-// model: waves x (BN + c0), c0 ~ fixed per-tile overhead in column units,
-// so narrow outputs pick a BN that fills the 148 SMs evenly (e.g. N = 768 ->
-// BN = 192: 32 x 4 = 128 tiles in one wave).  Weight-gradient GEMMs with few
-// output tiles split K (tokens) into S fixed ranges summed by the pack kernel
-// in a fixed order (deterministic).
 int env_int(const char *name, int dflt) {
   const char *v = getenv(name);
   return v && *v ? atoi(v) : dflt;
-}
-
-GemmPlan plan_tc_mn(int M, int N, int K, bool weight_grad) {
-  GemmPlan p;
-  const int mt = (M + 127) / 128;
-  const int nkb = (K + 63) / 64;
-  const int forced = env_int(weight_grad ? "OOO_BN_DW" : "OOO_BN", 0);
-  const int cands[4] = {256, 192, 128, 64};
-  double best = 1e30;
-  int best_bn = 128, best_S = 1;
-  for (int bn : cands) {
-    if (N % 64 != 0) continue;
-    if (forced && bn != forced) continue;
-    const int nt = (N + bn - 1) / bn;
-    const double waste = (double)(nt * bn - N) / (nt * bn);
-    if (waste > 0.25) continue;
-    const int tiles = mt * nt;
-    int S = 1;
-    if (weight_grad && tiles < kSMs) {
-      S = std::max(1, std::min(kSMs / tiles, nkb / 4));
-    }
-    const int kps = (nkb + S - 1) / S;
-    const int units = tiles * ((nkb + kps - 1) / kps);
-    const int waves = (units + kSMs - 1) / kSMs;
-    // per-unit cost ~ k-blocks x MMA time (N < 96 is shared-memory bound) +
-    // epilogue, + fp32 partial write / pack re-read when split
-    const int Sx = (nkb + kps - 1) / kps;
-    double cost = (double)waves * ((double)kps * (std::max(bn, 96) + 16) + 2.0 * bn + (Sx > 1 ? 6.0 * bn : 0.0));
-    if (cost < best * 0.999) {
-      best = cost;
-      best_bn = bn;
-      best_S = S;
-    }
-  }
-  p.bn = best_bn;
-  const int S = best_S;
-  p.kb_per_split = (nkb + S - 1) / S;
-  p.splits = (nkb + p.kb_per_split - 1) / p.kb_per_split;   // every split >= 1 k-block
-  const int units = mt * ((N + p.bn - 1) / p.bn) * p.splits;
-  p.grid = dim3(std::min(units, kSMs), 1, 1);
-  return p;
 }
 
 // Engine tile width for an output of width N: the widest of 256/192/128/64
@@ -206,6 +159,9 @@ ooo_status validate_desc(const ooo_stack_desc *d, bool need_pointers) {
   if (d->dtype != OOO_BF16 && d->dtype != OOO_FP32)
     return fail(OOO_ERR_INVALID_ARGUMENT, "dtype %d invalid", d->dtype);
   if (d->bucket_layers < 1) return fail(OOO_ERR_INVALID_ARGUMENT, "bucket_layers must be >= 1");
+  if (d->dtype == OOO_BF16 && 2 * d->num_layers > ooo::eng::kMaxOps)
+    return fail(OOO_ERR_UNSUPPORTED, "bf16 stacks: num_layers = %d > %d (engine op table)", d->num_layers,
+                ooo::eng::kMaxOps / 2);
   if (d->world_size < 1 || d->rank < 0 || d->rank >= d->world_size)
     return fail(OOO_ERR_INVALID_ARGUMENT, "world_size %d / rank %d invalid", d->world_size, d->rank);
   if (need_pointers) {
@@ -257,11 +213,7 @@ Plan make_plan(const ooo_stack_desc *d) {
     lp.goff_b = goff + (int64_t)lp.din * lp.dout;
     goff = lp.goff_b + lp.dout;
     lp.bucket = (i - 1) / d->bucket_layers;
-    if (p.dtype == OOO_BF16) {
-      lp.fwd = plan_tc_mn(p.M, lp.dout, lp.din, false);
-      lp.dx = plan_tc_mn(p.M, lp.din, lp.dout, false);
-      lp.dw = plan_tc_mn(lp.din, lp.dout, p.M, true);
-    } else {
+    if (p.dtype == OOO_FP32) {   // per-layer SIMT GEMMs on the hi / lo streams
       lp.fwd = plan_simt(p.M, lp.dout, lp.din, false);
       lp.dx = plan_simt(p.M, lp.din, lp.dout, false);
       lp.dw = plan_simt(lp.din, lp.dout, p.M, true);
@@ -274,7 +226,7 @@ Plan make_plan(const ooo_stack_desc *d) {
   p.off_wpart = wpart ? take(wpart) : 0;
   p.nbuckets = (p.L + d->bucket_layers - 1) / d->bucket_layers;
   // persistent dataflow engine (bf16): map table, layer table, counters
-  p.engine = p.dtype == OOO_BF16 && 2 * p.L <= ooo::eng::kMaxOps && env_int("OOO_ENGINE", 1) != 0;
+  p.engine = p.dtype == OOO_BF16;   // bf16: the persistent dataflow engine (validate_desc bounds L)
   if (p.engine) {
     // CTA pairs (256-row tiles) unless the token dimension fits one 128-row tile
     const int cg_env = env_int("OOO_CG", 0);
@@ -379,8 +331,6 @@ struct LayerRt {
   void *X = nullptr, *Z = nullptr, *Xn = nullptr, *dZ = nullptr;
   float *db = nullptr;
   void *gw = nullptr, *gb = nullptr;
-  CUtensorMap fwdA, fwdB, dxA, dxB, dwA, dwB;   // operand loads
-  CUtensorMap fwdZ, fwdX, dzX, gwX;              // output stores: Z_i, X_{i+1}, dZ_i, dW_i bucket
 };
 
 struct TimedRec {
@@ -414,6 +364,8 @@ struct ooo_stack {
   const CUtensorMap *dmaps = nullptr;         // map table (workspace)
   const ooo::eng::LayerDev *dlayers = nullptr;
   int engine_ctas = 148;
+  bool comm_stack = false;                    // a NCCL communicator (N > 1, or the one-rank mode)
+  int timeout_ms = 4000;                      // engine wait bound (desc.wait_timeout_ms)
   bool test_comm_gate = false;                // OOO_TEST_COMM_GATE=1 (N = 1 only): see comm_active
   // emulated all-reduce (N = 1 only; OOO_EMULATE_AR_N = n >= 2): each bucket's
   // S[dW] holds the comm stream for the ring time 2(n-1)/n x bytes / BW + lat
@@ -442,6 +394,16 @@ struct ooo_graph {
   ooo_stack *s = nullptr;
   cudaGraph_t graph = nullptr;
   cudaGraphExec_t exec = nullptr;
+  // per-launch timing (ooo_graph_set_timing_slots): the timing brackets
+  // captured into the graph (record info in capture order), their event-record
+  // nodes, and `slots` sets of events the nodes are re-pointed to, one set per
+  // launch, so every launch of a timed region keeps its own measurement
+  struct TNode { cudaGraphNode_t node; int rec, which; };
+  std::vector<ooo_launch_record> tinfo;
+  std::vector<TNode> tnodes;
+  std::vector<cudaEvent_t> sev;    // [slot][rec][2]
+  int slots = 0;
+  long launches = 0;
 };
 
 namespace {
@@ -495,20 +457,9 @@ ooo_status launch_fwd(ooo_stack *s, int i, void *Y, cudaStream_t st, int prio) {
   TimedRec *tr;
   OOO_TRY(begin_rec(s, st, 0, i, 0, &tr));
   LaunchCtx ctx{st, prio, s->pdl};
-  int grid = lp.fwd.grid.x * lp.fwd.grid.y * lp.fwd.grid.z;
-  if (s->p.dtype == OOO_BF16) {
-    CUtensorMap ymap;
-    const CUtensorMap *xm = &r.fwdX;
-    if (i == s->p.L) {   // the caller's Y: encoded per call (baked into a captured graph)
-      OOO_TRY(make_map(&ymap, Y, lp.dout, s->p.M, 64, 32));
-      xm = &ymap;
-    }
-    const CUtensorMap *zm = r.Z ? &r.fwdZ : xm;
-    CU_TRY(launch_gemm_tc(EPI_FWD, lp.fwd.bn, &r.fwdA, &r.fwdB, zm, xm, a, grid, ctx));
-  } else {
-    SimtOperands o{static_cast<const float *>(r.X), lp.din, 1, static_cast<const float *>(r.W), lp.dout, 1};
-    CU_TRY(launch_gemm_simt(EPI_FWD, o, a, ctx, &grid));
-  }
+  int grid = 0;
+  SimtOperands o{static_cast<const float *>(r.X), lp.din, 1, static_cast<const float *>(r.W), lp.dout, 1};
+  CU_TRY(launch_gemm_simt(EPI_FWD, o, a, ctx, &grid));
   return end_rec(tr, st, grid, 2.0 * s->p.M * lp.din * lp.dout, 0);
 }
 
@@ -535,21 +486,9 @@ ooo_status launch_dx(ooo_stack *s, int i, void *dX, cudaStream_t st, int prio) {
   TimedRec *tr;
   OOO_TRY(begin_rec(s, st, 1, i, st == s->hi ? 0 : 1, &tr));
   LaunchCtx ctx{st, prio, s->pdl};
-  int grid = lp.dx.grid.x * lp.dx.grid.y * lp.dx.grid.z;
-  if (s->p.dtype == OOO_BF16) {
-    CUtensorMap dxmap;
-    const CUtensorMap *xm = nullptr;
-    if (i >= 2) {
-      xm = &s->lr[i - 2].dzX;
-    } else {             // the caller's dX: encoded per call
-      OOO_TRY(make_map(&dxmap, dX, lp.din, s->p.M, 64, 32));
-      xm = &dxmap;
-    }
-    CU_TRY(launch_gemm_tc(EPI_DGRAD, lp.dx.bn, &r.dxA, &r.dxB, xm, xm, a, grid, ctx));
-  } else {
-    SimtOperands o{static_cast<const float *>(r.dZ), lp.dout, 1, static_cast<const float *>(r.W), 1, lp.dout};
-    CU_TRY(launch_gemm_simt(EPI_DGRAD, o, a, ctx, &grid));
-  }
+  int grid = 0;
+  SimtOperands o{static_cast<const float *>(r.dZ), lp.dout, 1, static_cast<const float *>(r.W), 1, lp.dout};
+  CU_TRY(launch_gemm_simt(EPI_DGRAD, o, a, ctx, &grid));
   return end_rec(tr, st, grid, 2.0 * s->p.M * lp.din * lp.dout, 0);
 }
 
@@ -567,13 +506,9 @@ ooo_status launch_dw_pack(ooo_stack *s, int i, cudaStream_t st, int prio, int si
   TimedRec *tr;
   OOO_TRY(begin_rec(s, st, 2, i, sid, &tr));
   LaunchCtx ctx{st, prio, s->pdl};
-  int grid = lp.dw.grid.x * lp.dw.grid.y * lp.dw.grid.z;
-  if (s->p.dtype == OOO_BF16) {
-    CU_TRY(launch_gemm_tc(EPI_WGRAD, lp.dw.bn, &r.dwA, &r.dwB, &r.gwX, &r.gwX, a, grid, ctx));
-  } else {
-    SimtOperands o{static_cast<const float *>(r.X), 1, lp.din, static_cast<const float *>(r.dZ), lp.dout, 1};
-    CU_TRY(launch_gemm_simt(EPI_WGRAD, o, a, ctx, &grid));
-  }
+  int grid = 0;
+  SimtOperands o{static_cast<const float *>(r.X), 1, lp.din, static_cast<const float *>(r.dZ), lp.dout, 1};
+  CU_TRY(launch_gemm_simt(EPI_WGRAD, o, a, ctx, &grid));
   OOO_TRY(end_rec(tr, st, grid, 2.0 * s->p.M * lp.din * lp.dout, 0));
   // pack (plain launch: it does not use griddepcontrol)
   ctx.pdl = false;
@@ -650,6 +585,17 @@ ooo_status join_into(ooo_stack *s, cudaStream_t st) {
   CU_TRY(cudaStreamWaitEvent(st, s->ev_j_hi, 0));
   CU_TRY(cudaStreamWaitEvent(st, s->ev_j_lo, 0));
   CU_TRY(cudaStreamWaitEvent(st, s->ev_j_comm, 0));
+  return OOO_OK;
+}
+
+// Caller activation buffers: the bf16 engine's epilogue stores rows with
+// 32-byte vector stores (st.global.v8.b32) and its X -> X_1 copy reads 16-byte
+// vectors, so X / Y / dY / dX must be 32-byte aligned (TMA descriptors alone
+// would accept 16); fp32 stacks need 16 bytes.
+ooo_status check_align(const ooo_stack *s, const void *p, const char *name) {
+  const uintptr_t a = s->p.dtype == OOO_BF16 ? 32 : 16;
+  if (reinterpret_cast<uintptr_t>(p) % a != 0)
+    return fail(OOO_ERR_INVALID_ARGUMENT, "%s must be %d-byte aligned", name, (int)a);
   return OOO_OK;
 }
 
@@ -821,6 +767,7 @@ ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const 
   P.dbg = env_int("OOO_DBG", 0);
   P.copy_nt = (s->dims[0] + copy_bn(s->dims[0]) - 1) / copy_bn(s->dims[0]);
   P.a_rows = a_box_rows(p);
+  P.timeout_ns = (uint64_t)s->timeout_ms * 1000000ull;
   P.maps = s->dmaps;
   P.ctr = s->ctr;
   P.layers = s->dlayers;
@@ -841,9 +788,9 @@ ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const 
 #endif
   CUtensorMap tmY, tmDX;
   if (Y) OOO_TRY(make_map(&tmY, Y, p.layer[p.L - 1].dout, p.M, 32, 32, 64));
-  else tmY = s->lr[0].dxA;    // unused placeholder
+  else memset(&tmY, 0, sizeof(tmY));    // unused placeholder
   if (dX) OOO_TRY(make_map(&tmDX, dX, s->dims[0], p.M, 32, 32, 64));
-  else tmDX = s->lr[0].dxA;
+  else memset(&tmDX, 0, sizeof(tmDX));
   TimedRec *tr;
   OOO_TRY(begin_rec(s, s->hi, rec_kind, 0, 0, &tr));
   CU_TRY(ooo::eng::launch_engine(p.cg, P, &tmY, &tmDX, s->engine_ctas, s->hi, s->prio_hi));
@@ -910,12 +857,13 @@ ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st)
   for (int i = 1; i <= L; ++i) fwd.push_back(unit_of(s, pl::FWD, i));
   if (s->eng_pending && env_int("OOO_FUSE", 1) == 0) OOO_TRY(engine_flush(s));   // experiments: unfused
   if (s->eng_pending) {
-    if (s->emu_n > 1) {
+    if (s->emu_n > 1 || (s->nccl && s->d.comm_enabled)) {
       cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
       CU_TRY(cudaStreamIsCapturing(st, &cs));
       if (cs != cudaStreamCaptureStatusActive)
-        return fail(OOO_ERR_UNSUPPORTED, "emulated all-reduce: run the fused step through ooo_graph_create "
-                                         "(an eager step with kernels on the comm stream stalls, see ooo.h)");
+        return fail(OOO_ERR_UNSUPPORTED, "communicating stack: run the fused step (ooo_backward; ooo_forward) "
+                                         "through ooo_graph_create, or ooo_join before ooo_forward (an eager "
+                                         "fused step with kernels on the comm stream stalls, see ooo.h)");
     }
     // backward(t) + forward(t+1) in one launch (Fig. 4(c)); counters were
     // reset by ooo_backward.  F_i is gated on dW_i (N = 1) or on its bucket's
@@ -1337,7 +1285,7 @@ ooo_status ooo_engine_plan(const ooo_stack_desc *d, ooo_schedule sch, int32_t fu
   pb.rows = (tmp.p.cl.MT + tmp.p.cg - 1) / tmp.p.cg;
   pb.workers = workers > 0 ? workers : std::max(1, kSMs / tmp.p.cg);
   pb.in_order = in_order;
-  pb.fwd_gate = fused ? (d->world_size > 1 && d->comm_enabled ? 2 : 1) : 0;
+  pb.fwd_gate = fused ? ((d->world_size > 1 || d->nccl_unique_id) && d->comm_enabled ? 2 : 1) : 0;
   pb.bucket.resize(pb.L);
   for (int i = 1; i <= pb.L; ++i) pb.bucket[i - 1] = tmp.p.layer[i - 1].bucket;
   pb.crit = crit;
@@ -1378,6 +1326,8 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
   s->d.acts = s->acts.data();
   s->p = make_plan(d);
   s->pdl = env_int("OOO_PDL", 1) != 0;
+  s->comm_stack = d->world_size > 1 || d->nccl_unique_id != nullptr;
+  s->timeout_ms = d->wait_timeout_ms > 0 ? d->wait_timeout_ms : (s->comm_stack ? 120000 : 4000);
   s->test_comm_gate = d->world_size == 1 && s->p.engine && env_int("OOO_TEST_COMM_GATE", 0) != 0;
   s->ws = static_cast<uint8_t *>(d->workspace);
   s->grads = static_cast<uint8_t *>(d->grads);
@@ -1388,11 +1338,6 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
     t_err = msg;
     return st;
   };
-  static std::once_flag init_once;
-  static cudaError_t init_err = cudaSuccess;
-  std::call_once(init_once, [] { init_err = gemm_tc_init(); });
-  if (init_err != cudaSuccess)
-    return cleanup_fail(fail(OOO_ERR_CUDA, "kernel attribute init: %s", cudaGetErrorString(init_err)));
   s->lr.resize(p.L);
   for (int i = 1; i <= p.L; ++i) {
     const LayerPlan &lp = p.layer[i - 1];
@@ -1406,20 +1351,6 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
     r.db = reinterpret_cast<float *>(s->ws + lp.off_db);
     r.gw = s->grads + lp.goff_w * p.elt;
     r.gb = s->grads + lp.goff_b * p.elt;
-    if (p.dtype == OOO_BF16) {
-      ooo_status st;
-      if ((st = make_map(&r.fwdA, r.X, lp.din, p.M, 64, 128)) != OOO_OK ||
-          (st = make_map(&r.fwdB, r.W, lp.dout, lp.din, 64, 64)) != OOO_OK ||
-          (st = make_map(&r.dxA, r.dZ, lp.dout, p.M, 64, 128)) != OOO_OK ||
-          (st = make_map(&r.dxB, r.W, lp.dout, lp.din, 64, lp.dx.bn)) != OOO_OK ||
-          (st = make_map(&r.dwA, r.X, lp.din, p.M, 64, 64)) != OOO_OK ||
-          (st = make_map(&r.dwB, r.dZ, lp.dout, p.M, 64, 64)) != OOO_OK ||
-          (st = make_map(&r.dzX, r.dZ, lp.dout, p.M, 64, 32)) != OOO_OK ||
-          (st = make_map(&r.gwX, r.gw, lp.dout, lp.din, 64, 32)) != OOO_OK ||
-          (r.Z && (st = make_map(&r.fwdZ, r.Z, lp.dout, p.M, 64, 32)) != OOO_OK) ||
-          (r.Xn && (st = make_map(&r.fwdX, r.Xn, lp.dout, p.M, 64, 32)) != OOO_OK))
-        return cleanup_fail(st);
-    }
   }
   if (p.engine) {
     static std::once_flag eng_once;
@@ -1480,13 +1411,13 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     // emulated all-reduce (measurement aid, N = 1): see ooo_stack::emu_n
-    if (d->world_size == 1 && env_int("OOO_EMULATE_AR_N", 0) > 1) {
+    if (!s->comm_stack && env_int("OOO_EMULATE_AR_N", 0) > 1) {
       s->emu_n = env_int("OOO_EMULATE_AR_N", 0);
       if (const char *v = getenv("OOO_EMULATE_AR_GBPS")) s->emu_gbps = atof(v);
       if (const char *v = getenv("OOO_EMULATE_AR_LAT_US")) s->emu_lat_us = atof(v);
     }
     // N > 1 (or its emulation): leave SMs for the NCCL kernels the engine's counters wait on
-    const int reserve = d->world_size > 1 || s->emu_n > 1 ? (d->nccl_max_ctas > 0 ? d->nccl_max_ctas : 16) : 0;
+    const int reserve = s->comm_stack || s->emu_n > 1 ? (d->nccl_max_ctas > 0 ? d->nccl_max_ctas : 16) : 0;
     s->engine_ctas = std::max(1, sms - reserve);
     s->engine_ctas = std::min(s->engine_ctas, env_int("OOO_ENGINE_CTAS", s->engine_ctas));
   }
@@ -1514,7 +1445,7 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
       (e = mk(&s->ev_j_lo)) != cudaSuccess || (e = mk(&s->ev_j_comm)) != cudaSuccess ||
       (e = mk(&s->ev_reset)) != cudaSuccess)
     return cleanup_fail(fail(OOO_ERR_CUDA, "event create: %s", cudaGetErrorString(e)));
-  if (d->world_size > 1) {
+  if (s->comm_stack) {
     const char *why = nullptr;
     s->api = nccl_api(&why);
     if (!s->api) return cleanup_fail(fail(OOO_ERR_NCCL, "NCCL unavailable: %s", why));
@@ -1534,6 +1465,16 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
       s->nccl = nullptr;
       return cleanup_fail(fail(OOO_ERR_NCCL, "ncclCommInitRank: %s", s->api->GetErrorString(r)));
     }
+    // warm-up: every bucket's all-reduce once (lazy channel connection, NVLS
+    // setup) so that no training step pays it under the engine's wait bound
+    ooo_status st = OOO_OK;
+    cudaError_t ce = cudaMemsetAsync(s->grads, 0, (size_t)p.grad_elems * p.elt, s->comm);
+    if (ce != cudaSuccess) st = fail(OOO_ERR_CUDA, "warm-up memset: %s", cudaGetErrorString(ce));
+    for (int b = p.nbuckets - 1; b >= 0 && st == OOO_OK && d->comm_enabled; --b) st = launch_allreduce(s, b);
+    if (st == OOO_OK && (ce = cudaStreamSynchronize(s->comm)) != cudaSuccess)
+      st = fail(OOO_ERR_CUDA, "warm-up all-reduce: %s", cudaGetErrorString(ce));
+    if (st == OOO_OK) st = check_async(s);
+    if (st != OOO_OK) return cleanup_fail(st);
   }
   *out = s;
   return OOO_OK;
@@ -1541,6 +1482,8 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
 
 ooo_status ooo_forward(ooo_stack *s, const void *X, void *Y, void *stream) {
   if (!s || !X || !Y) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
+  OOO_TRY(check_align(s, X, "X"));
+  OOO_TRY(check_align(s, Y, "Y"));
   OOO_TRY(check_async(s));
   return enqueue_forward(s, X, Y, static_cast<cudaStream_t>(stream));
 }
@@ -1553,6 +1496,8 @@ ooo_status ooo_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void *dX
   if (s->d.need_input_grad && !dX) return fail(OOO_ERR_INVALID_ARGUMENT, "need_input_grad set but dX NULL");
   if (!s->d.need_input_grad && dX) return fail(OOO_ERR_INVALID_ARGUMENT, "dX given but need_input_grad = 0");
   if (!s->have_fwd) return fail(OOO_ERR_STATE, "ooo_backward without a preceding ooo_forward");
+  OOO_TRY(check_align(s, dY, "dY"));
+  if (dX) OOO_TRY(check_align(s, dX, "dX"));
   OOO_TRY(check_async(s));
   return enqueue_backward(s, dY, sch, dX, static_cast<cudaStream_t>(stream));
 }
@@ -1562,6 +1507,20 @@ ooo_status ooo_join(ooo_stack *s, void *stream) {
   OOO_TRY(engine_flush(s));
   OOO_TRY(join_into(s, static_cast<cudaStream_t>(stream)));
   return check_async(s);
+}
+
+ooo_status ooo_allreduce_buckets(ooo_stack *s, void *stream) {
+  if (!s) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL stack");
+  if (!s->nccl) return fail(OOO_ERR_STATE, "stack has no communicator");
+  OOO_TRY(check_async(s));
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  OOO_TRY(engine_flush(s));
+  OOO_TRY(fork_from(s, st));
+  if (s->timing) s->rec_cursor = 0;
+  for (int b = s->p.nbuckets - 1; b >= 0; --b) {
+    if (s->d.comm_enabled) OOO_TRY(launch_allreduce(s, b));
+  }
+  return join_into(s, st);
 }
 
 ooo_status ooo_graph_create(ooo_stack *s, const void *X, void *Y, const void *dY, ooo_schedule sch,
@@ -1574,6 +1533,10 @@ ooo_status ooo_graph_create(ooo_stack *s, const void *X, void *Y, const void *dY
   if (sch.k < 0) return fail(OOO_ERR_INVALID_ARGUMENT, "k must be >= 0");
   if (s->d.need_input_grad && !dX) return fail(OOO_ERR_INVALID_ARGUMENT, "need_input_grad set but dX NULL");
   if (!s->d.need_input_grad && dX) return fail(OOO_ERR_INVALID_ARGUMENT, "dX given but need_input_grad = 0");
+  OOO_TRY(check_align(s, X, "X"));
+  OOO_TRY(check_align(s, Y, "Y"));
+  OOO_TRY(check_align(s, dY, "dY"));
+  if (dX) OOO_TRY(check_align(s, dX, "dX"));
   cudaStream_t cap;
   CU_TRY(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
   cudaError_t e = cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal);
@@ -1601,18 +1564,86 @@ ooo_status ooo_graph_create(ooo_stack *s, const void *X, void *Y, const void *dY
   gr->s = s;
   gr->graph = g;
   gr->exec = ex;
+  if (s->timing && s->rec_cursor > 0) {
+    for (size_t j = 0; j < s->rec_cursor; ++j) gr->tinfo.push_back(s->recs[j].info);
+    size_t nn = 0;
+    if (cudaGraphGetNodes(g, nullptr, &nn) == cudaSuccess && nn > 0) {
+      std::vector<cudaGraphNode_t> nodes(nn);
+      if (cudaGraphGetNodes(g, nodes.data(), &nn) == cudaSuccess) {
+        for (cudaGraphNode_t n : nodes) {
+          cudaGraphNodeType ty;
+          cudaEvent_t ev = nullptr;
+          if (cudaGraphNodeGetType(n, &ty) != cudaSuccess || ty != cudaGraphNodeTypeEventRecord) continue;
+          if (cudaGraphEventRecordNodeGetEvent(n, &ev) != cudaSuccess) continue;
+          for (size_t j = 0; j < s->rec_cursor; ++j) {
+            if (s->recs[j].a == ev) gr->tnodes.push_back({n, (int)j, 0});
+            else if (s->recs[j].b == ev) gr->tnodes.push_back({n, (int)j, 1});
+          }
+        }
+      }
+    }
+    (void)cudaGetLastError();
+  }
   *out = gr;
+  return OOO_OK;
+}
+
+ooo_status ooo_graph_set_timing_slots(ooo_graph *g, int32_t slots) {
+  if (!g) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL graph");
+  if (slots < 1) return fail(OOO_ERR_INVALID_ARGUMENT, "slots must be >= 1");
+  if (g->tnodes.empty()) return fail(OOO_ERR_STATE, "graph was captured without timing (ooo_set_timing before ooo_graph_create)");
+  for (cudaEvent_t e : g->sev) cudaEventDestroy(e);
+  g->sev.assign((size_t)slots * g->tinfo.size() * 2, nullptr);
+  for (cudaEvent_t &e : g->sev) CU_TRY(cudaEventCreate(&e));
+  g->slots = slots;
+  g->launches = 0;
+  return OOO_OK;
+}
+
+ooo_status ooo_graph_timing_read(ooo_graph *g, ooo_launch_record *out, int32_t cap, int32_t *n, int32_t *per_launch) {
+  if (!g || !n) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
+  const int nrec = (int)g->tinfo.size();
+  const long used = std::min<long>(g->launches, g->slots);
+  if (per_launch) *per_launch = nrec;
+  int32_t cnt = 0;
+  for (long l = 0; l < used; ++l) {
+    for (int j = 0; j < nrec; ++j, ++cnt) {
+      if (!out || cnt >= cap) continue;
+      cudaEvent_t a = g->sev[((size_t)l * nrec + j) * 2], b = g->sev[((size_t)l * nrec + j) * 2 + 1];
+      out[cnt] = g->tinfo[j];
+      float ms = 0.f, st = 0.f;
+      cudaError_t e = cudaEventElapsedTime(&ms, a, b);
+      out[cnt].ms = e == cudaSuccess ? ms : -1.f;
+      if (e != cudaSuccess) (void)cudaGetLastError();
+      e = cudaEventElapsedTime(&st, g->sev[0], a);
+      out[cnt].start_ms = e == cudaSuccess ? st : -1.f;
+      if (e != cudaSuccess) (void)cudaGetLastError();
+    }
+  }
+  *n = cnt;
   return OOO_OK;
 }
 
 ooo_status ooo_graph_launch(ooo_graph *g, void *stream) {
   if (!g) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL graph");
+  if (g->slots > 0 && g->launches <= g->slots) {
+    // re-point the timing nodes: launch l records into slot l's events; after
+    // the last slot, back to the stack's own events (slots keep their values)
+    const int nrec = (int)g->tinfo.size();
+    for (const ooo_graph::TNode &t : g->tnodes) {
+      cudaEvent_t ev = g->launches < g->slots ? g->sev[((size_t)g->launches * nrec + t.rec) * 2 + t.which]
+                                              : (t.which ? g->s->recs[t.rec].b : g->s->recs[t.rec].a);
+      CU_TRY(cudaGraphExecEventRecordNodeSetEvent(g->exec, t.node, ev));
+    }
+  }
   CU_TRY(cudaGraphLaunch(g->exec, static_cast<cudaStream_t>(stream)));
+  if (g->slots > 0) ++g->launches;
   return OOO_OK;
 }
 
 ooo_status ooo_graph_destroy(ooo_graph *g) {
   if (!g) return OOO_OK;
+  for (cudaEvent_t e : g->sev) cudaEventDestroy(e);
   if (g->exec) cudaGraphExecDestroy(g->exec);
   if (g->graph) cudaGraphDestroy(g->graph);
   delete g;

@@ -1,6 +1,6 @@
 // Shared sm_100a device helpers (PTX wrappers for mbarrier / TMA / tcgen05 /
-// PDL, UMMA descriptors, epilogue math) used by gemm_tc.cu (per-layer
-// kernels) and engine.cu (persistent dataflow kernels).
+// PDL, UMMA descriptors, epilogue math) used by engine.cu (the persistent
+// dataflow kernel of the bf16 path).
 #pragma once
 #include <cuda.h>
 #include <cuda_bf16.h>

@@ -22,7 +22,7 @@ def _i32arr(vals):
 
 
 def _desc(dims, acts, tokens, dtype, need_input_grad=False, bucket_layers=1, max_temp_bytes=0,
-          world_size=1, rank=0, comm_enabled=True, nccl_max_ctas=0):
+          world_size=1, rank=0, comm_enabled=True, nccl_max_ctas=0, wait_timeout_ms=0):
     keep = {}
     d = _lib.StackDesc()
     d.num_layers = len(acts)
@@ -39,6 +39,7 @@ def _desc(dims, acts, tokens, dtype, need_input_grad=False, bucket_layers=1, max
     d.rank = int(rank)
     d.comm_enabled = int(bool(comm_enabled))
     d.nccl_max_ctas = int(nccl_max_ctas)
+    d.wait_timeout_ms = int(wait_timeout_ms)
     return d, keep
 
 
@@ -130,6 +131,11 @@ def broadcast_unique_id(group=None) -> bytes:
     return obj[0]
 
 
+def _record(r) -> dict:
+    return {"kind": _lib.KIND_NAMES.get(r.kind, r.kind), "layer": r.layer, "stream": r.stream, "grid": r.grid,
+            "flops": r.flops, "bytes": r.bytes, "ms": r.ms, "start_ms": r.start_ms}
+
+
 def _stream_handle(stream):
     import torch
     if stream is None:
@@ -148,6 +154,22 @@ class StepGraph:
     def launch(self, stream=None):
         check(load().ooo_graph_launch(self._h, _stream_handle(stream)))
 
+    def set_timing_slots(self, slots: int):
+        """The next `slots` launches each record their own per-kernel CUDA
+        events (graph captured with the stack's timing on)."""
+        check(load().ooo_graph_set_timing_slots(self._h, int(slots)))
+
+    def timing(self) -> list:
+        """Per-launch records of the timed launches: a list (one entry per
+        launch) of lists of record dicts (see OooStack.timing)."""
+        n, per = c_int32(), c_int32()
+        check(load().ooo_graph_timing_read(self._h, None, 0, ctypes.byref(n), ctypes.byref(per)))
+        recs = (_lib.LaunchRecord * max(1, n.value))()
+        check(load().ooo_graph_timing_read(self._h, recs, n.value, ctypes.byref(n), ctypes.byref(per)))
+        flat = [_record(r) for r in recs[: n.value]]
+        p = max(1, per.value)
+        return [flat[i: i + p] for i in range(0, len(flat), p)]
+
     def close(self):
         if self._h:
             load().ooo_graph_destroy(self._h)
@@ -165,7 +187,10 @@ class OooStack:
 
     def __init__(self, dims, acts, tokens, W, b, dtype="bf16", need_input_grad=False, bucket_layers=1,
                  max_temp_bytes=0, world_size=1, rank=0, unique_id: bytes | None = None,
-                 comm_enabled=True, nccl_max_ctas=0):
+                 comm_enabled=True, nccl_max_ctas=0, wait_timeout_ms=0):
+        """unique_id: the NCCL bootstrap id (broadcast_unique_id); required
+        for world_size > 1; with world_size == 1 it makes a one-rank
+        communicator that runs the N > 1 data plane on one GPU."""
         import torch
         lib = load()
         self.dims = [int(x) for x in dims]
@@ -189,7 +214,7 @@ class OooStack:
         self.W, self.b = list(W), list(b)
         self.device = W[0].device
         d, keep = _desc(self.dims, self.acts, self.tokens, dtype, need_input_grad, bucket_layers,
-                        max_temp_bytes, world_size, rank, comm_enabled, nccl_max_ctas)
+                        max_temp_bytes, world_size, rank, comm_enabled, nccl_max_ctas, wait_timeout_ms)
         ws, gb = c_size_t(), c_size_t()
         check(lib.ooo_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)))
         self.workspace = torch.empty(ws.value, dtype=torch.uint8, device=self.device)
@@ -200,9 +225,11 @@ class OooStack:
         d.b = ctypes.cast(keep["b"], ctypes.POINTER(c_void_p))
         d.grads = self.grads_buf.data_ptr()
         d.workspace = self.workspace.data_ptr()
-        if self.world_size > 1:
-            if unique_id is None or len(unique_id) != _lib.UNIQUE_ID_BYTES:
-                raise ValueError("world_size > 1 needs the 128-byte NCCL unique id (broadcast_unique_id)")
+        if self.world_size > 1 and unique_id is None:
+            raise ValueError("world_size > 1 needs the 128-byte NCCL unique id (broadcast_unique_id)")
+        if unique_id is not None:
+            if len(unique_id) != _lib.UNIQUE_ID_BYTES:
+                raise ValueError("the NCCL unique id has 128 bytes")
             keep["uid"] = ctypes.create_string_buffer(unique_id, _lib.UNIQUE_ID_BYTES)
             d.nccl_unique_id = ctypes.cast(keep["uid"], c_void_p)
         self._keep = keep
@@ -245,6 +272,11 @@ class OooStack:
 
     def join(self, stream=None):
         check(load().ooo_join(self._h, _stream_handle(stream)))
+
+    def allreduce_buckets(self, stream=None):
+        """Every bucket's all-reduce back to back on the stack's own
+        communicator (stand-alone S[dW] time; sums `grads` in place again)."""
+        check(load().ooo_allreduce_buckets(self._h, _stream_handle(stream)))
 
     def graph(self, X, Y, dY, kind="first_k", k=0, dX=None) -> StepGraph:
         self._check_act(X, self.tokens, self.dims[0], "X")
@@ -303,12 +335,7 @@ class OooStack:
         check(load().ooo_timing_read(self._h, None, 0, ctypes.byref(n)))
         recs = (_lib.LaunchRecord * max(1, n.value))()
         check(load().ooo_timing_read(self._h, recs, n.value, ctypes.byref(n)))
-        out = []
-        for r in recs[: n.value]:
-            out.append({"kind": _lib.KIND_NAMES.get(r.kind, r.kind), "layer": r.layer, "stream": r.stream,
-                        "grid": r.grid, "flops": r.flops, "bytes": r.bytes, "ms": r.ms,
-                        "start_ms": r.start_ms})
-        return out
+        return [_record(r) for r in recs[: n.value]]
 
     def close(self):
         if getattr(self, "_h", None):

@@ -407,3 +407,131 @@ def test_bf16_narrowest_and_widest_widths():
     inorder = case.run(stk, "in_order", 0)
     assert torch.equal(inorder["raw"], out["raw"])
     stk.close()
+
+
+# ------------------- the N > 1 data plane on one GPU: a one-rank NCCL communicator
+def _nccl_stack(case, monkeypatch, **kw):
+    from paper_conf_eurosys_ohlks22_b200.stack import get_unique_id
+    # the bit-exact setting SURVEY §8e pins for N > 1 (one rank: NCCL's own path)
+    monkeypatch.setenv("NCCL_ALGO", "Ring")
+    monkeypatch.setenv("NCCL_PROTO", "Simple")
+    return case.stack(unique_id=get_unique_id(), **kw)
+
+
+@pytest.mark.parametrize("kind,k", [("first_k", 2), ("in_order", 0), ("first_k", 5)])
+def test_bf16_nccl_one_rank_fused_steps_bit_exact(monkeypatch, kind, k):
+    """A real NCCL communicator (world_size 1, ooo_get_unique_id) drives the
+    whole N > 1 data plane through the captured fused step:
+    per-bucket cuStreamWaitValue32 on the engine's dW counters ->
+    ncclAllReduce -> cuStreamWriteValue32 of the flag F_i(t+1) waits on, with
+    the 16-SM reserve.  Over three steps with fresh inputs the gradients and Y
+    equal the non-communicating stack bit for bit (the all-reduce of one rank
+    is the identity) and the oracle within the bf16 gate; the library's
+    launch records show one all-reduce per bucket."""
+    dims, acts = [256, 512, 256, 256, 512, 256], ["gelu", "id", "id", "gelu", "id"]
+    cases = [Case(dims, acts, 520, "bf16", step=t) for t in range(4)]
+    plain = cases[0].stack(bucket_layers=2)
+    comm = _nccl_stack(cases[0], monkeypatch, bucket_layers=2)
+    Xb = [to_dev(cases[0].X, "bf16") for _ in range(2)]
+    dYb = [to_dev(cases[0].dY, "bf16") for _ in range(2)]
+    Yb = [torch.empty(cases[0].M, dims[-1], dtype=torch.bfloat16, device="cuda") for _ in range(2)]
+    plain.forward(Xb[0], Yb[0])
+    comm.forward(Xb[1], Yb[1])
+    comm.set_timing(True)                    # launch records captured into the graph
+    g = [plain.graph(Xb[0], Yb[0], dYb[0], kind, k), comm.graph(Xb[1], Yb[1], dYb[1], kind, k)]
+    for t in range(3):
+        for j in range(2):                   # step t's dY, step t+1's X into the captured buffers
+            dYb[j].copy_(to_dev(cases[t].dY, "bf16"))
+            Xb[j].copy_(to_dev(cases[t + 1].X, "bf16"))
+            g[j].launch()
+        torch.cuda.synchronize()
+        assert torch.equal(comm.grads_buf, plain.grads_buf), t
+        assert torch.equal(Yb[0], Yb[1]), t
+        ref = cases[t].oracle(k if kind == "first_k" else 0)
+        _check(max_err({"Y": ref.Y[0], "dW": [to_np(w) for w in comm.dW], "db": [to_np(v) for v in comm.db],
+                        "dX": None}, ref), BF16_TOL)
+        assert rel_fro(to_np(Yb[1]), cases[t + 1].oracle().Y[0]) <= BF16_TOL
+    recs = comm.timing()
+    assert sum(r["kind"] == "allreduce" for r in recs) == 3, recs     # ceil(5 / 2) buckets
+    comm.set_timing(False)
+    for x in g:
+        x.close()
+    # the stand-alone all-reduce of every bucket (bench's AR_ms): identity at one rank
+    before = comm.grads_buf.clone()
+    comm.allreduce_buckets()
+    torch.cuda.synchronize()
+    assert torch.equal(comm.grads_buf, before)
+    plain.close()
+    comm.close()
+
+
+def test_bf16_nccl_one_rank_eager_rules(monkeypatch):
+    """Eager use of a communicating stack: backward + join (all-reduces after
+    the engine) is bit-exact with the plain stack; an eager fused step
+    (forward with a backward pending) is refused with OOO_ERR_UNSUPPORTED
+    (ooo.h), and the stack stays usable after the refusal."""
+    from paper_conf_eurosys_ohlks22_b200._lib import OooError
+    case = Case([256, 512, 256, 256], ["gelu", "id", "id"], 264, "bf16")
+    plain = case.stack()
+    comm = _nccl_stack(case, monkeypatch)
+    a = case.run(plain, "first_k", 1)
+    b = case.run(comm, "first_k", 1)
+    assert torch.equal(a["raw"], b["raw"])
+    X, dY = to_dev(case.X, "bf16"), to_dev(case.dY, "bf16")
+    comm.forward(X)
+    comm.backward(dY, "first_k", 1)
+    with pytest.raises(OooError, match="UNSUPPORTED"):
+        comm.forward(X)
+    comm.join()
+    torch.cuda.synchronize()
+    assert torch.equal(comm.grads_buf, plain.grads_buf)
+    plain.close()
+    comm.close()
+
+
+def test_bf16_misaligned_activation_rejected():
+    """the engine stores 32-byte row vectors, so a 16-byte aligned
+    view of Y (or X, dY, dX) is rejected before anything is enqueued."""
+    from paper_conf_eurosys_ohlks22_b200._lib import OooError
+    case = Case([256, 256], ["id"], 64, "bf16")
+    stk = case.stack()
+    X = to_dev(case.X, "bf16")
+    big = torch.empty(64 * 256 + 8, dtype=torch.bfloat16, device="cuda")
+    Ymis = big[8:].view(64, 256)                 # 16-byte offset
+    with pytest.raises(OooError, match="aligned"):
+        stk.forward(X, Ymis)
+    stk.forward(X)
+    stk.close()
+
+
+def test_graph_timing_slots_every_launch():
+    """ooo_graph_set_timing_slots: each of the timed launches of a captured
+    step keeps its own per-kernel CUDA-event durations (bench.py's roofline
+    takes the engine kernel's mean over all timed launches); the slots do
+    not change the results."""
+    case = Case([256, 512, 256, 256], ["gelu", "id", "id"], 520, "bf16")
+    stk = case.stack()
+    base = case.run(stk, "first_k", 1, graph=True, launches=1)
+    X, dY = to_dev(case.X, "bf16"), to_dev(case.dY, "bf16")
+    Y = stk.forward(X)
+    stk.set_timing(True)
+    g = stk.graph(X, Y, dY, "first_k", 1)
+    stk.set_timing(False)
+    g.set_timing_slots(6)
+    for _ in range(8):
+        g.launch()
+    torch.cuda.synchronize()
+    per = g.timing()
+    assert len(per) == 6
+    kinds = [r["kind"] for r in per[0]]
+    assert "engine_step" in kinds and "seed" in kinds, kinds
+    for recs in per:
+        assert [r["kind"] for r in recs] == kinds
+        assert all(r["ms"] > 0 for r in recs)
+    starts = [recs[0]["start_ms"] for recs in per]
+    assert starts == sorted(starts) and starts[-1] > starts[0]
+    g.close()
+    stk.join()
+    torch.cuda.synchronize()
+    assert torch.equal(stk.grads_buf, base["raw"])
+    stk.close()

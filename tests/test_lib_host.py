@@ -33,7 +33,7 @@ def test_library_exports_every_declared_symbol(lib):
     for name in declared:
         assert hasattr(lib, name), name
     assert set(_lib.EXPORTS) == declared
-    assert lib.ooo_abi_version() == 1
+    assert lib.ooo_abi_version() == 2
 
 
 @pytest.mark.parametrize("L", [1, 2, 3, 5, 8, 13, 72, 144])
