@@ -59,7 +59,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample-tokens", type=int, default=0)
-    ap.add_argument("--runs", type=int, default=5, help="extra timed runs for mean +- s.e.")
+    ap.add_argument("--runs", type=int, default=10,
+                    help="the K timed steps run as this many back-to-back runs (mean +- s.e. over runs), "
+                         "interleaved with as many in_order runs")
     return ap.parse_args()
 
 
@@ -204,6 +206,86 @@ def run_reference(args):
 
 
 # ------------------------------------------------------------------ ours
+def split_runs(steps: int, runs: int) -> list:
+    """K timed steps as R back-to-back runs (mean +- s.e. over runs)."""
+    runs = max(1, min(runs, steps))
+    base, extra = divmod(steps, runs)
+    return [base + (1 if r < extra else 0) for r in range(runs)]
+
+
+def dp_selfcheck(world, rank, dev, stream, dist, bucket_layers=2):
+    """N > 1: the library's data plane checks itself before anything is timed.
+    A small stack with the bit-exact NCCL setting SURVEY §8e pins
+    (NCCL_ALGO=Ring NCCL_PROTO=Simple), per-rank seeded shards (synth), shared
+    W: (1) in_order and ooo_first_k(2) give bit-identical gradients on every
+    rank (fixed all-reduce order); (2) every rank holds the same bytes
+    (gathered sha256); (3) the all-reduced gradient equals the sum over ranks
+    of each rank's local 1/N-scaled gradient (comm-off stack of the same
+    library, summed in fp32 by torch.distributed) within the bf16 gate --
+    i.e. every bucket was really reduced across ranks before F_i read it.
+    Runs through captured steps (eager fused steps are refused at N > 1).
+    At N = 1 the same check runs on a one-rank communicator (the N > 1 data
+    plane on one GPU), so its code is exercised by every single-GPU bench."""
+    import hashlib
+
+    import torch
+    from paper_conf_eurosys_ohlks22_b200 import synth
+    from paper_conf_eurosys_ohlks22_b200.stack import OooStack, broadcast_unique_id, get_unique_id
+    uid = broadcast_unique_id if world > 1 else get_unique_id
+    dims, acts, M = [256, 512, 256, 256, 512, 256], ["gelu", "id", "id", "gelu", "id"], 264
+    Wn, bn = synth.weights(dims, acts, "bf16")
+    tb = lambda a: torch.from_numpy(a).to(torch.bfloat16).to(dev).contiguous()  # noqa: E731
+    W, b = [tb(w) for w in Wn], [tb(x) for x in bn]
+    X = tb(synth.x_shard(M, dims[0], rank, "bf16"))
+    dY = tb(synth.dy_shard(M, dims[-1], rank, "bf16"))
+    Y = torch.empty(M, dims[-1], dtype=torch.bfloat16, device=dev)
+    saved = {k: os.environ.get(k) for k in ("NCCL_ALGO", "NCCL_PROTO")}
+    os.environ.update({"NCCL_ALGO": "Ring", "NCCL_PROTO": "Simple"})
+    try:
+        on = OooStack(dims, acts, M, W, b, bucket_layers=bucket_layers, world_size=world, rank=rank,
+                      unique_id=uid())
+        off = OooStack(dims, acts, M, W, b, bucket_layers=bucket_layers, world_size=world, rank=rank,
+                       unique_id=uid(), comm_enabled=False)
+    finally:
+        for k, v in saved.items():
+            if v is None:
+                os.environ.pop(k, None)
+            else:
+                os.environ[k] = v
+    out = {}
+    for name, stk in (("on", on), ("off", off)):
+        for sch in (("in_order", 0), ("first_k", 2)):
+            stk.forward(X, Y)
+            g = stk.graph(X, Y, dY, *sch)
+            g.launch(stream)
+            torch.cuda.synchronize()
+            out[(name, sch[0])] = stk.grads_buf.clone()
+            g.close()
+    bit_exact = bool(torch.equal(out[("on", "in_order")], out[("on", "first_k")]) and
+                     torch.equal(out[("off", "in_order")], out[("off", "first_k")]))
+    h = hashlib.sha256(out[("on", "first_k")].cpu().numpy().tobytes()).hexdigest()
+    hs = [h] * world
+    local = out[("off", "first_k")].view(torch.bfloat16).float()
+    if world > 1:
+        dist.all_gather_object(hs, h)
+        dist.all_reduce(local)                          # fp32 sum of the ranks' 1/N-scaled local gradients
+    got = out[("on", "first_k")].view(torch.bfloat16).float()
+    errs = []
+    offs_w = [(w.data_ptr() - on.grads_buf.data_ptr()) // 2 for w in on.dW]
+    offs_b = [(x.data_ptr() - on.grads_buf.data_ptr()) // 2 for x in on.db]
+    for i in range(len(acts)):
+        for o, n in ((offs_w[i], on.dW[i].numel()), (offs_b[i], on.db[i].numel())):
+            r = local[o: o + n]
+            errs.append(float((got[o: o + n] - r).norm() / r.norm().clamp_min(1e-30)))
+    on.close()
+    off.close()
+    res = {"stack": f"{len(acts)} layers {dims}, {M} tokens/rank, bucket_layers {bucket_layers}",
+           "nccl_env": "NCCL_ALGO=Ring NCCL_PROTO=Simple", "in_order_eq_first_k_bit_exact": bit_exact,
+           "ranks_identical": len(set(hs)) == 1, "max_rel_err_vs_sum_of_local_grads": max(errs)}
+    res["ok"] = bool(bit_exact and res["ranks_identical"] and res["max_rel_err_vs_sum_of_local_grads"] <= 1e-2)
+    return res
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -221,7 +303,28 @@ def main():
     cfg = configs.get(args.config)
     dt = cfg.dtype
     M = cfg.tokens
+    L = cfg.L
     peaks = load_peaks()
+    stream = torch.cuda.current_stream()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(xs):
+        """Elementwise max over ranks of a list of floats (device-timed values)."""
+        if world == 1:
+            return list(xs)
+        t = torch.tensor(list(xs), dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return t.tolist()
+
+    try:
+        selfcheck = dp_selfcheck(world, rank, dev, stream, dist)
+    except Exception as e:  # noqa: BLE001 -- reported in the line (and fatal at N > 1 below)
+        selfcheck = {"ok": False, "error": str(e)[:300]}
+    if not selfcheck.get("ok"):
+        print(f"WARNING: data-parallel self-check failed: {selfcheck}", file=sys.stderr, flush=True)
 
     W, b = synth.weights_torch(cfg.dims, cfg.acts, dt, dev)
     uid = broadcast_unique_id() if world > 1 else None
@@ -230,45 +333,45 @@ def main():
     X = synth.activations_torch(M, cfg.dims[0], dt, dev, synth.SEED, rank, 0)
     dY = synth.activations_torch(M, cfg.dims[-1], dt, dev, synth.SEED, rank, 1)
     Y = torch.empty(M, cfg.dims[-1], dtype=X.dtype, device=dev)
-    stream = torch.cuda.current_stream()
 
-    def barrier():
-        if world > 1:
-            dist.barrier()
-
-    def max_over_ranks(x: float) -> float:
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
-
-    def timed(graph, steps, sampler=None):
+    def interleaved(graphs, steps, runs, sampler=None):
+        """Time `steps` launches of every graph in `graphs` as `runs`
+        back-to-back runs per graph, interleaved A B A B ... (no host sync or
+        idle inside the region), bracketed by barrier + synchronize; CUDA
+        events on the launching stream; per-run times max over ranks.
+        Returns per graph the list of per-run ms per step."""
+        sizes = split_runs(steps, runs)
+        ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in sizes]
+              for _ in graphs]
         barrier()
         torch.cuda.synchronize()
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
         if sampler:
             sampler.__enter__()
-            time.sleep(0.2)
-        e0.record(stream)
-        for _ in range(steps):
-            graph.launch(stream)
-        e1.record(stream)
+        for r, n in enumerate(sizes):
+            for gi, g in enumerate(graphs):
+                ev[gi][r][0].record(stream)
+                for _ in range(n):
+                    g.launch(stream)
+                ev[gi][r][1].record(stream)
         torch.cuda.synchronize()
         if sampler:
             sampler.__exit__(None, None, None)
         barrier()
-        return max_over_ranks(e0.elapsed_time(e1) / steps)
+        flat = [ev[gi][r][0].elapsed_time(ev[gi][r][1]) for gi in range(len(graphs)) for r in range(len(sizes))]
+        flat = max_over_ranks(flat)
+        return [[flat[gi * len(sizes) + r] / sizes[r] for r in range(len(sizes))] for gi in range(len(graphs))]
+
+    def summary(per_run, steps, runs):
+        sizes = split_runs(steps, runs)
+        total = sum(ms * n for ms, n in zip(per_run, sizes))
+        mean = total / sum(sizes)
+        sem = statistics.stdev(per_run) / math.sqrt(len(per_run)) if len(per_run) > 1 else None
+        return {"ms_per_step": mean, "value": 1e3 / mean, "runs": len(per_run), "run_steps": sizes,
+                "run_ms_per_step": per_run, "sem_ms": sem}
 
     stk.forward(X, Y)
     torch.cuda.synchronize()
     graphs = {}
-
-    def s_graph(Xb, Yb, dYb, sch):
-        stk.forward(Xb, Yb)          # the graph's backward needs a forward on these buffers
-        torch.cuda.synchronize()
-        return stk.graph(Xb, Yb, dYb, *sch)
 
     def graph_for(kind, k, s=stk):
         key = (id(s), kind, k)
@@ -277,7 +380,6 @@ def main():
         return graphs[key]
 
     # ---- choose k: the paper's heuristic search (§5.1) on measured throughput
-    L = cfg.L
     if args.k == "auto":
         from paper_conf_eurosys_ohlks22_b200.ksearch import search_k
         probe = max(5, min(20, args.steps // 2))
@@ -286,7 +388,7 @@ def main():
             g = graph_for("first_k", k)
             for _ in range(2):
                 g.launch(stream)
-            return 1e3 / timed(g, probe)
+            return 1e3 / interleaved([g], probe, 1)[0][0]
         k_best, visited = search_k(L, tput)
     else:
         k_best, visited = int(args.k), []
@@ -294,7 +396,7 @@ def main():
     sched = ("first_k", k_best)
     # ---- N = 1: the paper's single-GPU method -- multi-stream ooo with
     # Algorithm 1 regions (§4.1), planned from profiled co-run
-    # speedups; the better of it and reverse first-k is the measured schedule
+    # speedups; the better of it and reverse first-k (ABAB probe) is timed
     regions = None
     plan = None
     if world == 1 and args.regions > 0 and dt == "bf16":    # profiles the bf16 engine
@@ -308,13 +410,14 @@ def main():
         torch.cuda.synchronize()
     if plan is not None:
         g_reg = graph_for("regions", 0)
-        probe = max(10, min(30, args.steps))
         for _ in range(3):
             g_reg.launch(stream)
             g_fk.launch(stream)
-        ms_r, ms_f = timed(g_reg, probe), timed(g_fk, probe)
+        pr = interleaved([g_reg, g_fk], max(20, min(60, args.steps)), 4)
+        ms_r, ms_f = statistics.mean(pr[0]), statistics.mean(pr[1])
         regions = {"region_layers": args.regions, "n_regions": plan["n_regions"], "k_pre": plan["k_pre"],
-                   "plan_seconds": t_plan, "probe_ms_per_step": ms_r, "first_k_probe_ms_per_step": ms_f}
+                   "D": plan["D"], "plan_seconds": t_plan, "probe_ms_per_step": ms_r,
+                   "first_k_probe_ms_per_step": ms_f}
         if ms_r < ms_f:
             sched = ("regions", 0)
     g_ooo = graph_for(*sched)
@@ -324,56 +427,65 @@ def main():
         g_in.launch(stream)
     torch.cuda.synchronize()
 
+    # ---- the timed region: K steps of the ooo schedule and K of in_order,
+    # as R runs each, interleaved ABAB (drift hits both alike)
     sampler = ClockSampler(local)
-    ms_ooo = timed(g_ooo, args.steps, sampler)
+    per = interleaved([g_ooo, g_in], args.steps, args.runs, sampler)
     clocks = sampler.summary()
-    ms_in = timed(g_in, args.steps)
-    ms_fk = ms_ooo if sched[0] == "first_k" else timed(g_fk, args.steps)
-    if plan is not None:
-        regions["ms_per_step"] = ms_ooo if sched[0] == "regions" else timed(graph_for("regions", 0), args.steps)
-    # repeat runs (mean +- standard error) and the dual-stream
-    # control ooo_first_k(0) (no reordering)
-    reps = [timed(g_ooo, args.steps) for _ in range(args.runs)]
+    main_s, in_s = summary(per[0], args.steps, args.runs), summary(per[1], args.steps, args.runs)
+    ms_ooo, ms_in = main_s["ms_per_step"], in_s["ms_per_step"]
+    # secondary comparisons (own ABAB regions): the other ooo schedule and the
+    # dual-stream control ooo_first_k(0) (no reordering)
+    half = max(10, args.steps // 2)
     g_k0 = graph_for("first_k", 0)
-    for _ in range(3):
-        g_k0.launch(stream)
-    ms_k0 = timed(g_k0, args.steps)
+    others = [("first_k", k_best)] if sched[0] == "regions" else ([("regions", 0)] if plan is not None else [])
+    og = [g_k0] + [graph_for(*o) for o in others]
+    for g in og:
+        for _ in range(3):
+            g.launch(stream)
+    po = interleaved([g_ooo] + og, half, max(2, args.runs // 2))
+    ms_k0 = statistics.mean(po[1])
+    ms_other = {f"{o[0]}": statistics.mean(po[2 + j]) for j, o in enumerate(others)}
+    ms_fk = ms_ooo if sched[0] == "first_k" else ms_other.get("first_k")
+    if regions is not None and plan is not None:
+        regions["ms_per_step"] = ms_ooo if sched[0] == "regions" else ms_other.get("regions")
 
-    # ---- exposed communication: same graph with the all-reduce skipped (comm-off control)
+    # ---- N > 1: exposed communication = same graphs with the all-reduce
+    # skipped (comm-off stack, ABAB with the comm-on graphs), and the
+    # stand-alone all-reduce of the library's own buckets on its own communicator
     exposed = None
     ar_ms = None
     if world > 1:
         stk_off = OooStack(cfg.dims, cfg.acts, M, W, b, dtype=dt, bucket_layers=args.bucket_layers,
-                           world_size=world, rank=rank, unique_id=broadcast_unique_id(), comm_enabled=False)
+                           world_size=world, rank=rank, unique_id=broadcast_unique_id(), comm_enabled=False,
+                           nccl_max_ctas=args.nccl_max_ctas)
         stk_off.forward(X, Y)
-        g_off = stk_off.graph(X, Y, dY, "first_k", k_best)
-        for _ in range(3):
-            g_off.launch(stream)
-        ms_off = timed(g_off, args.steps)
-        exposed = {"ooo_first_k": ms_ooo - ms_off}
+        g_off = stk_off.graph(X, Y, dY, *sched)
         g_off_in = stk_off.graph(X, Y, dY, "in_order", 0)
-        for _ in range(3):
-            g_off_in.launch(stream)
-        exposed["in_order"] = ms_in - timed(g_off_in, args.steps)
-        # standalone all-reduce time: every bucket back to back, no compute
-        views = []
-        for i in range(L):
-            views.append(stk.dW[i].view(-1))
-            views.append(stk.db[i])
-        torch.cuda.synchronize()
-        barrier()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        ar_reps = 5
-        e0.record(stream)
-        for _ in range(ar_reps):
-            for v in views:
-                dist.all_reduce(v)
-        e1.record(stream)
-        torch.cuda.synchronize()
-        ar_ms = max_over_ranks(e0.elapsed_time(e1) / ar_reps)
+        for g in (g_off, g_off_in):
+            for _ in range(3):
+                g.launch(stream)
+        pe = interleaved([g_ooo, g_off, g_in, g_off_in], half, max(2, args.runs // 2))
+        m = [statistics.mean(x) for x in pe]
+        exposed = {"ooo": m[0] - m[1], "in_order": m[2] - m[3], "ooo_comm_on_ms": m[0], "ooo_comm_off_ms": m[1],
+                   "in_order_comm_on_ms": m[2], "in_order_comm_off_ms": m[3]}
         g_off.close()
         g_off_in.close()
         stk_off.close()
+        reps = 10
+        stk.allreduce_buckets(stream)                   # warm
+        torch.cuda.synchronize()
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(reps):
+            stk.allreduce_buckets(stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        barrier()
+        ar_ms = max_over_ranks([e0.elapsed_time(e1) / reps])[0]
+        stk.forward(X, Y)                               # grads were summed again: fresh step state
+        torch.cuda.synchronize()
 
     # ---- N = 1: exposed communication against an EMULATED n-rank ring all-reduce
     # (no NCCL, no data moved: the comm stream is held for each bucket's ring
@@ -387,21 +499,28 @@ def main():
             ar_total = sum(2.0 * (n - 1) / n * (cfg.dims[i] * cfg.dims[i + 1] + cfg.dims[i + 1]) * elt / (gbps * 1e9) * 1e3
                            for i in range(L)) + nbk * lat * 1e-3
             ks = sorted({0, max(1, L // 24), L // 6, L // 2, L})
-            times = {}
+            gs = {}
+            stacks = []
             for label, bw, la in (("on", gbps, lat), ("off", 1e9, 0.0)):
                 os.environ.update({"OOO_EMULATE_AR_N": str(n), "OOO_EMULATE_AR_GBPS": str(bw),
                                    "OOO_EMULATE_AR_LAT_US": str(la)})
                 se = OooStack(cfg.dims, cfg.acts, M, W, b, dtype=dt, bucket_layers=args.bucket_layers)
+                stacks.append(se)
                 se.forward(X, Y)
                 for kind, k in [("in_order", 0)] + [("first_k", k) for k in ks]:
                     g = se.graph(X, Y, dY, kind, k)
                     for _ in range(3):
                         g.launch(stream)
-                    times[(label, kind, k)] = min(timed(g, max(10, args.steps // 2)) for _ in range(2))
-                    g.close()
-                se.close()
+                    gs[(label, kind, k)] = g
             for key in ("OOO_EMULATE_AR_N", "OOO_EMULATE_AR_GBPS", "OOO_EMULATE_AR_LAT_US"):
                 os.environ.pop(key, None)
+            keys = list(gs)
+            pe = interleaved([gs[k] for k in keys], max(10, args.steps // 4), 2)
+            times = {k: statistics.mean(v) for k, v in zip(keys, pe)}
+            for g in gs.values():
+                g.close()
+            for se in stacks:
+                se.close()
             sweep = {}
             for kind, k in [("in_order", 0)] + [("first_k", k) for k in ks]:
                 on, off = times[("on", kind, k)], times[("off", kind, k)]
@@ -411,7 +530,8 @@ def main():
             emulated = {"n": n, "link_GBps_per_direction": gbps, "latency_us_per_bucket": lat,
                         "bucket_layers": args.bucket_layers,
                         "note": "EMULATED all-reduce on one GPU (comm stream held for the ring time; no NCCL, no "
-                                "data moved); the engine keeps the 16-SM NCCL reserve",
+                                "data moved); the engine keeps the 16-SM NCCL reserve; all graphs timed "
+                                "interleaved (2 runs each)",
                         "allreduce_total_ms": ar_total, "in_order_ms": sweep["in_order(0)"]["ms"], "best": best,
                         "best_ms": sweep[best]["ms"], "best_exposed_ms": sweep[best]["exposed_ms"],
                         "best_hidden_fraction": sweep[best]["hidden_fraction"],
@@ -422,38 +542,51 @@ def main():
             for key in ("OOO_EMULATE_AR_N", "OOO_EMULATE_AR_GBPS", "OOO_EMULATE_AR_LAT_US"):
                 os.environ.pop(key, None)
 
-    # ---- per-kernel durations: instrumented replay of the same step (CUDA events per launch)
+    # ---- per-kernel durations: the same step captured with per-launch CUDA
+    # events (stream-ordered on the stream each kernel runs on), every launch of
+    # a K-step back-to-back region keeping its own events (timing slots)
     stk.set_timing(True)
+    stk.forward(X, Y)
     g_t = stk.graph(X, Y, dY, *sched)
+    stk.set_timing(False)
     for _ in range(3):
         g_t.launch(stream)
-    ms_timed = timed(g_t, max(3, args.steps // 2))
-    recs = stk.timing()
+    n_t = args.steps
+    g_t.set_timing_slots(n_t)
+    ms_timed = statistics.mean(interleaved([g_t], n_t, 1)[0])
+    per_launch = g_t.timing()
     g_t.close()
-    stk.set_timing(False)
     by_kind = {}
-    for r in recs:
-        d = by_kind.setdefault(r["kind"], {"ms": 0.0, "flops": 0.0, "bytes": 0.0, "n": 0})
-        d["ms"] += max(r["ms"], 0.0)
-        d["flops"] += r["flops"]
-        d["bytes"] += r["bytes"]
-        d["n"] += 1
+    for recs in per_launch:
+        for r in recs:
+            d = by_kind.setdefault(r["kind"], {"ms": [], "flops": r["flops"], "bytes": r["bytes"], "per_launch": 0})
+            d["ms"].append(max(r["ms"], 0.0))
+    for recs in per_launch[:1]:
+        for r in recs:
+            by_kind[r["kind"]]["per_launch"] += 1
     ours = {k: v for k, v in by_kind.items() if k not in ("allreduce", "copy")}
-    dom = max(ours, key=lambda k: ours[k]["ms"])
+    dom = max(ours, key=lambda k: sum(ours[k]["ms"]))
     dd = ours[dom]
-    launches_per_step = sum(v["n"] for v in ours.values())
+    n_launch = len(per_launch)
+    launches_per_step = sum(v["per_launch"] for v in ours.values())
+    dom_ms = statistics.mean(dd["ms"])                      # mean over every timed launch
+    dom_step_ms = sum(dd["ms"]) / max(1, n_launch)          # per step (if several launches per step)
     if dd["flops"] > 0:
-        achieved = dd["flops"] / (dd["ms"] * 1e-3) / 1e12
+        achieved = dd["flops"] / (dom_ms * 1e-3) / 1e12
         peak = peaks["bf16_tflops_sustained"] if dt == "bf16" else 75.0
         roof = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak}
     else:
-        achieved = dd["bytes"] / (dd["ms"] * 1e-3) / 1e9
+        achieved = dd["bytes"] / (dom_ms * 1e-3) / 1e9
         peak = peaks["hbm_gbs"]
         roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak}
     roof["kernel"] = dom
-    roof["launches_per_step"] = dd["n"]
-    roof["avg_launch_us"] = dd["ms"] * 1e3 / max(1, dd["n"])
-    roof["share_of_step"] = dd["ms"] / ms_timed
+    roof["algorithmic_work_per_launch"] = dd["flops"] if dd["flops"] > 0 else dd["bytes"]
+    roof["timed_launches"] = len(dd["ms"])
+    roof["avg_launch_us"] = dom_ms * 1e3
+    roof["launch_us_sem"] = (statistics.stdev(dd["ms"]) / math.sqrt(len(dd["ms"])) * 1e3) if len(dd["ms"]) > 1 else None
+    roof["share_of_step"] = dom_step_ms / ms_timed
+    roof["share_ok"] = roof["share_of_step"] <= 1.0 + 1e-3
+    roof["instrumented_ms_per_step"] = ms_timed
     roof["peak_source"] = f"{peaks['source']} ({'bf16_tflops_sustained' if dd['flops'] > 0 else 'hbm_gbs'})"
     traffic = None
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -465,11 +598,12 @@ def main():
             traffic = None
     roof["traffic"] = traffic
 
-    # ---- north-star roofline of the whole step: max(GEMM FLOP at peak, ring AR bytes at link bw)
+    # ---- north-star roofline of the whole step: max(GEMM FLOP at peak, ring AR bytes at 900 GB/s)
     flops = cfg.gemm_flops()
     t_tensor = flops / (peaks["bf16_tflops_sustained"] * 1e12) * 1e3 if dt == "bf16" else None
     grad_bytes = cfg.params() * (2 if dt == "bf16" else 4)
-    t_ar = 2 * (world - 1) / world * grad_bytes / 770e9 * 1e3 if world > 1 else 0.0
+    link = 900e9
+    t_ar = 2 * (world - 1) / world * grad_bytes / link * 1e3 if world > 1 else 0.0
     step_roof_ms = max(t_tensor or 0.0, t_ar)
     hbm_bytes = cfg.hbm_min_bytes()
     t_hbm = hbm_bytes / (peaks["hbm_gbs"] * 1e9) * 1e3
@@ -485,7 +619,12 @@ def main():
         sets = []
         for p in range(2):
             Xp, dYp, Yp = (X, dY, Y) if p == 0 else (torch.empty_like(X), torch.empty_like(dY), torch.empty_like(Y))
-            g = g_ooo if p == 0 else s_graph(Xp, Yp, dYp, sched)
+            if p == 0:
+                g = g_ooo
+            else:
+                stk.forward(Xp, Yp)
+                torch.cuda.synchronize()
+                g = stk.graph(Xp, Yp, dYp, *sched)
             hX = torch.empty(X.shape, dtype=X.dtype, pin_memory=True)
             hdY = torch.empty(dY.shape, dtype=dY.dtype, pin_memory=True)
             hY = torch.empty(Y.shape, dtype=Y.dtype, pin_memory=True)
@@ -525,7 +664,7 @@ def main():
         run_steps(args.steps, e0, e1)
         torch.cuda.synchronize()
         barrier()
-        ms_e2e = max_over_ranks(e0.elapsed_time(e1) / args.steps)
+        ms_e2e = max_over_ranks([e0.elapsed_time(e1) / args.steps])[0]
         ebytes = X.element_size()
         e2e = {"value": 1e3 / ms_e2e, "unit": UNIT,
                "h2d_bytes_per_step": (X.numel() + dY.numel()) * ebytes, "d2h_bytes_per_step": Y.numel() * ebytes,
@@ -540,6 +679,15 @@ def main():
                "sample": f"one fp64 (bf16-storage) forward+backward of {tok} of {M} tokens of {cfg.name}, "
                          f"{sec:.1f} s, scaled by {tok}/{M}"}
 
+    nccl = None
+    if world > 1:
+        try:
+            ver = torch.cuda.nccl.version()
+        except Exception:  # noqa: BLE001
+            ver = None
+        nccl = {"version": ".".join(map(str, ver)) if isinstance(ver, tuple) else ver,
+                "env": {k: v for k, v in sorted(os.environ.items()) if k.startswith("NCCL_")},
+                "library_communicator_max_ctas": args.nccl_max_ctas or 16}
     value = 1e3 / ms_ooo
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -551,26 +699,32 @@ def main():
                                 else "ooo_first_k"),
                    "k": k_best, "k_search_visited": visited,
                    "bucket_layers": args.bucket_layers, "parallelism": f"dp{world}",
+                   "timing": f"{args.steps} steps as {len(main_s['run_steps'])} back-to-back runs, interleaved "
+                             f"with as many in_order runs (ABAB); value = steps / summed run time",
                    "l2": "working set (weights+activations+grads) >> 126 MB L2; no flush"},
         "tokens_per_s": value * M * world,
-        "in_order": {"value": 1e3 / ms_in, "ms_per_step": ms_in},
+        "runs": {"n": main_s["runs"], "mean_ms": ms_ooo, "sem_ms": main_s["sem_ms"],
+                 "run_ms_per_step": main_s["run_ms_per_step"]},
+        "in_order": {"value": in_s["value"], "ms_per_step": ms_in, "sem_ms": in_s["sem_ms"]},
         "ooo_speedup_vs_in_order": ms_in / ms_ooo,
         "exposed_allreduce_ms": exposed,
         "allreduce_standalone_ms": ar_ms,
-        "hidden_fraction": (None if not exposed or not ar_ms else 1.0 - exposed["ooo_first_k"] / ar_ms),
-        "runs": {"n": len(reps), "mean_ms": statistics.mean(reps) if reps else None,
-                 "sem_ms": (statistics.stdev(reps) / math.sqrt(len(reps))) if len(reps) > 1 else None},
+        "allreduce_standalone_note": ("the library's own buckets on its own communicator (ooo_allreduce_buckets), "
+                                      "back to back, no compute" if world > 1 else None),
+        "hidden_fraction": (None if not exposed or not ar_ms else 1.0 - max(0.0, exposed["ooo"]) / ar_ms),
+        "dp_selfcheck": selfcheck,
+        "nccl": nccl,
         "ooo_first_k0": {"value": 1e3 / ms_k0, "ms_per_step": ms_k0},
-        "ooo_first_k": {"k": k_best, "value": 1e3 / ms_fk, "ms_per_step": ms_fk},
+        "ooo_first_k": {"k": k_best, "value": 1e3 / ms_fk if ms_fk else None, "ms_per_step": ms_fk},
         "regions": regions,
         "emulated_dp": emulated,
         "step_roofline": {"ms": step_roof_ms, "frac": step_roof_ms / ms_ooo if step_roof_ms else None,
-                          "tensor_ms": t_tensor, "allreduce_ms_at_770GBps": t_ar, "gemm_flops": flops,
+                          "tensor_ms": t_tensor, "allreduce_ms_at_900GBps": t_ar, "gemm_flops": flops,
                           "hbm_min_bytes": hbm_bytes, "hbm_ms": t_hbm,
                           "hbm_inclusive_ms": max(step_roof_ms, t_hbm)},
         "roofline": roof,
-        "kernels": {k: {"ms_per_step": v["ms"], "launches": v["n"]} for k, v in by_kind.items()},
-        "instrumented_ms_per_step": ms_timed,
+        "kernels": {k: {"mean_ms_per_launch": statistics.mean(v["ms"]), "launches_per_step": v["per_launch"]}
+                    for k, v in by_kind.items()},
         "gpu_launches": launches_per_step * args.steps,
         "clocks": clocks,
         "e2e": e2e,

@@ -20,13 +20,16 @@ Modules
                a backward schedule D, data-parallel averaging, bf16 storage
                rounding (§2, §3, §5.1).
 ``schedule``   Algorithm 2 (reverse first-k), the k memory clamp
-               (**parity unpinned**: the formula is garbled) and the
-               k heuristic search (**parity unpinned**: prose only).
+               (the formula is garbled -- reading Q3) and the k
+               heuristic search (prose only -- reading Q4).
 ``unit_sim``   unit-time list-scheduling simulator used to pin the dependency
                rules against the paper's worked examples (Fig. 4, P:164/P:180/
                P:206; Fig. 5, P:226/P:232/P:236).
 
 Pin status: every function is pinned by a
-``-m "not gpu"`` test against something other than itself, except
-``schedule.max_k`` and ``schedule.search_k`` which say "parity unpinned".
+``-m "not gpu"`` test against something other than itself.
+``schedule.max_k`` and ``schedule.search_k`` are pinned to their readings
+(Q3, Q4: the paper gives no numeric example, so the readings themselves rest
+on the text alone) by traces expanded by hand from the readings' wording
+(tests/golden/alg2_kclamp_ksearch.json).
 """

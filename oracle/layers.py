@@ -98,6 +98,28 @@ def act_grad(name: str, z: np.ndarray) -> np.ndarray:
     raise ValueError(name)
 
 
+# ------------------------------------------------- single steps (per op)
+# The arithmetic of one op from given inputs, in float64 without storage
+# rounding.  forward / op_dO / op_dW below are built from these, so every pin
+# of the full stack (finite differences, fp64 autograd, P:99 invariance) also
+# pins them; the teacher-forced GPU tests call them on the
+# GPU's own stored inputs of each step.
+def step_F(X: np.ndarray, W: np.ndarray, b: np.ndarray) -> np.ndarray:
+    """F_i (§2): Z_i = X_i W_i + 1 b_i^T."""
+    return X @ W + b[None, :]
+
+
+def step_dO(G: np.ndarray, W: np.ndarray, factor: np.ndarray | None) -> np.ndarray:
+    """dO_i: (G_i W_i^T) * act_{i-1}'(Z_{i-1}); factor None = dX (i == 1)."""
+    P = G @ W.T
+    return P if factor is None else P * factor
+
+
+def step_dW(X: np.ndarray, G: np.ndarray) -> tuple:
+    """dW_i: (X_i^T G_i, 1^T G_i)."""
+    return X.T @ G, G.sum(axis=0)
+
+
 # ------------------------------------------------------------------ forward
 @dataclass
 class ForwardState:
@@ -114,7 +136,7 @@ def forward(X1: np.ndarray, W: list, b: list, acts: list, dtype: str = "fp64") -
     Xs = [storage_round(X1, dtype)]
     Zs = []
     for i in range(L):
-        Z = storage_round(Xs[i] @ W[i] + b[i][None, :], dtype)
+        Z = storage_round(step_F(Xs[i], W[i], b[i]), dtype)
         Zs.append(Z)
         Xs.append(storage_round(act_fwd(acts[i], Z), dtype))
     return ForwardState(X=Xs, Z=Zs)
@@ -142,11 +164,10 @@ def op_dO(i: int, bs: BackwardState, state: ForwardState, W: list, acts: list, d
     (or dX for i == 1)."""
     if i not in bs.G:
         raise RuntimeError(f"dO_{i} scheduled before G_{i} exists (violates P:84 dependency)")
-    P = bs.G[i] @ W[i - 1].T
     if i == 1:
-        bs.dX = storage_round(P, dtype)
+        bs.dX = storage_round(step_dO(bs.G[i], W[i - 1], None), dtype)
     else:
-        bs.G[i - 1] = storage_round(P * act_grad(acts[i - 2], state.Z[i - 2]), dtype)
+        bs.G[i - 1] = storage_round(step_dO(bs.G[i], W[i - 1], act_grad(acts[i - 2], state.Z[i - 2])), dtype)
     bs.order.append(+i)
 
 
@@ -156,8 +177,7 @@ def op_dW(i: int, bs: BackwardState, state: ForwardState) -> None:
     ``dp_average`` (S[dW_i], §5.1)."""
     if i not in bs.G:
         raise RuntimeError(f"dW_{i} scheduled before G_{i} exists (violates P:84 dependency)")
-    bs.dW[i] = state.X[i - 1].T @ bs.G[i]
-    bs.db[i] = bs.G[i].sum(axis=0)
+    bs.dW[i], bs.db[i] = step_dW(state.X[i - 1], bs.G[i])
     bs.order.append(-i)
 
 

@@ -80,6 +80,17 @@ def max_err(gpu, ref) -> dict:
     return errs
 
 
+def record_parity(name: str, data: dict) -> None:
+    """Append measured errors to $OOO_PARITY_OUT (JSON lines) when set, so a
+    GPU run can commit the table of measured errors (profiles/r02_parity.md)."""
+    import json
+    import os
+    path = os.environ.get("OOO_PARITY_OUT")
+    if path:
+        with open(path, "a") as f:
+            f.write(json.dumps({"test": name, **data}) + "\n")
+
+
 def bf16_floor(L: int) -> float:
     """Random-walk floor of two independently rounded bf16 pipelines
     (SURVEY §8c G3): sqrt(2L) * 2^-9 / sqrt(3)."""

@@ -12,7 +12,7 @@ import torch
 
 from paper_conf_eurosys_ohlks22_b200 import configs
 from oracle.layers import rel_fro
-from tests.gpu_helpers import TDT, Case, bf16_floor, max_err, to_dev, to_np
+from tests.gpu_helpers import TDT, Case, bf16_floor, max_err, record_parity, to_dev, to_np
 
 pytestmark = pytest.mark.gpu
 
@@ -122,6 +122,8 @@ def test_bf16_mlp96_full_config():
     stk = case.stack()
     out = case.run(stk, "first_k", 48, graph=True)
     errs = max_err(out, ref)
+    record_parity("g3_MLP96", {"config": c.name, "layers": c.L, "errors": errs, "floor": bf16_floor(c.L),
+                               "gate": max(BF16_TOL, 2 * bf16_floor(c.L))})
     _check(errs, max(BF16_TOL, 2 * bf16_floor(c.L)))
     base = case.run(stk, "in_order", 0)
     assert torch.equal(out["raw"], base["raw"])
@@ -138,6 +140,8 @@ def test_bf16_bert_base_full_config_end_to_end():
     out = case.run(stk, "first_k", 24, graph=True)
     errs = max_err(out, ref)
     print("bert_base full-size errors", errs, "floor", bf16_floor(c.L))
+    record_parity("g3_BERT-base", {"config": c.name, "layers": c.L, "errors": errs, "floor": bf16_floor(c.L),
+                                   "gate": max(BF16_TOL, 2 * bf16_floor(c.L))})
     _check(errs, max(BF16_TOL, 2 * bf16_floor(c.L)))
     # bench.py's N = 1 schedule: Algorithm 1 regions of one block (§4.1), graph-captured
     stk.forward(to_dev(case.X, "bf16"))
@@ -341,6 +345,8 @@ def test_bf16_144_layer_full_configs_end_to_end(cfg):
     out = case.run(stk, "first_k", cfg.L // 6, graph=True)
     errs = max_err(out, ref)
     print(cfg.name, "full-size errors", errs, "floor", bf16_floor(cfg.L))
+    record_parity(f"g3_{cfg.name}", {"config": cfg.name, "layers": cfg.L, "errors": errs,
+                                      "floor": bf16_floor(cfg.L), "gate": max(BF16_TOL, 2 * bf16_floor(cfg.L))})
     _check(errs, max(BF16_TOL, 2 * bf16_floor(cfg.L)))
     stk.forward(to_dev(case.X, "bf16"))
     stk.plan_regions(region_layers=6)

@@ -286,3 +286,39 @@ def test_fig4_data_parallel_unit_counts():
     t = {k: U.dp_iteration(L, S.reverse_first_k(L, k), c, "preemptive") for k in range(L + 1)}
     best = min(t.values())
     assert sorted(k for k, v in t.items() if v == best) == g["optimal_k"]
+
+
+def test_max_k_and_search_k_hand_expanded_traces():
+    """Alg. 2 l.1 (reading Q3) and the k search (P:212-214,
+    reading Q4) against traces expanded by hand from the readings' text
+    (tests/golden/alg2_kclamp_ksearch.json): the oracle's f(j), max_k, visit
+    order and best k, and the library's (ooo_max_k / ooo_k_search) -- two
+    implementations pinned to the same hand-computed numbers."""
+    import json
+    import os
+    from oracle import schedule as S
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "alg2_kclamp_ksearch.json")))
+    fns = {"-(k-7)^2": lambda k: -(k - 7) ** 2, "-|k-40|": lambda k: -abs(k - 40),
+           "-(k-11)^2": lambda k: -(k - 11) ** 2, "-(k-3)^2": lambda k: -(k - 3) ** 2, "1 (flat)": lambda k: 1.0}
+    lib_ok = True
+    try:
+        from paper_conf_eurosys_ohlks22_b200 import stack
+        from paper_conf_eurosys_ohlks22_b200.ksearch import search_k as lib_search
+        stack.max_k(0, [1], [1], 0)
+    except Exception:  # noqa: BLE001 -- library not built: the oracle half still runs
+        lib_ok = False
+    for c in g["max_k"]["cases"]:
+        L = len(c["m_dO"])
+        assert [S.f_mem(j, c["m_fwd"], c["m_dO"], c["m_dW"]) for j in range(L + 1)] == c["f"]
+        for mxm, want in c["mxm_to_max_k"]:
+            assert S.max_k(c["m_fwd"], c["m_dO"], c["m_dW"], mxm) == want, (c, mxm)
+            if lib_ok:
+                assert stack.max_k(c["m_fwd"], c["m_dO"], c["m_dW"], mxm) == want, (c, mxm)
+    for c in g["search_k"]["cases"]:
+        f = fns[c["throughput"]]
+        visited = []
+        assert S.search_k(c["L"], f, visited) == c["best"], c
+        assert visited == c["visited"], (c, visited)
+        if lib_ok:
+            best, vis = lib_search(c["L"], f)
+            assert (best, vis) == (c["best"], c["visited"]), (c, best, vis)
