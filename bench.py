@@ -56,6 +56,10 @@ def parse():
                     help="consecutive layers per all-reduce bucket (6 = one transformer block: per-call latency; "
                          "measured with the emulated all-reduce, DESIGN.md §5c)")
     ap.add_argument("--nccl-max-ctas", type=int, default=0)
+    ap.add_argument("--comm-priority", type=int, default=0,
+                    help="1: prioritised, partitioned all-reduce issue (Fig. 4(b), P:180) for the timed stack")
+    ap.add_argument("--comm-chunk-mb", type=float, default=4.0,
+                    help="all-reduce partition size (MB) of the prioritised communication")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-sample-tokens", type=int, default=0)
@@ -328,8 +332,10 @@ def main():
 
     W, b = synth.weights_torch(cfg.dims, cfg.acts, dt, dev)
     uid = broadcast_unique_id() if world > 1 else None
+    chunk = int(args.comm_chunk_mb * 2 ** 20)
+    comm_kw = {"comm_priority": args.comm_priority, "comm_chunk_bytes": chunk if args.comm_priority else 0}
     stk = OooStack(cfg.dims, cfg.acts, M, W, b, dtype=dt, bucket_layers=args.bucket_layers,
-                   world_size=world, rank=rank, unique_id=uid, nccl_max_ctas=args.nccl_max_ctas)
+                   world_size=world, rank=rank, unique_id=uid, nccl_max_ctas=args.nccl_max_ctas, **comm_kw)
     X = synth.activations_torch(M, cfg.dims[0], dt, dev, synth.SEED, rank, 0)
     dY = synth.activations_torch(M, cfg.dims[-1], dt, dev, synth.SEED, rank, 1)
     Y = torch.empty(M, cfg.dims[-1], dtype=X.dtype, device=dev)
@@ -458,7 +464,7 @@ def main():
     if world > 1:
         stk_off = OooStack(cfg.dims, cfg.acts, M, W, b, dtype=dt, bucket_layers=args.bucket_layers,
                            world_size=world, rank=rank, unique_id=broadcast_unique_id(), comm_enabled=False,
-                           nccl_max_ctas=args.nccl_max_ctas)
+                           nccl_max_ctas=args.nccl_max_ctas, **comm_kw)
         stk_off.forward(X, Y)
         g_off = stk_off.graph(X, Y, dY, *sched)
         g_off_in = stk_off.graph(X, Y, dY, "in_order", 0)
@@ -501,10 +507,13 @@ def main():
             ks = sorted({0, max(1, L // 24), L // 6, L // 2, L})
             gs = {}
             stacks = []
-            for label, bw, la in (("on", gbps, lat), ("off", 1e9, 0.0)):
+            # "prio": the same emulated link with the prioritised, partitioned
+            # issue order (NEXT-4, Fig. 4(b)); the zero-time control is shared
+            for label, bw, la, pr in (("on", gbps, lat, 0), ("prio", gbps, lat, 1), ("off", 1e9, 0.0, 0)):
                 os.environ.update({"OOO_EMULATE_AR_N": str(n), "OOO_EMULATE_AR_GBPS": str(bw),
                                    "OOO_EMULATE_AR_LAT_US": str(la)})
-                se = OooStack(cfg.dims, cfg.acts, M, W, b, dtype=dt, bucket_layers=args.bucket_layers)
+                se = OooStack(cfg.dims, cfg.acts, M, W, b, dtype=dt, bucket_layers=args.bucket_layers,
+                              comm_priority=pr, comm_chunk_bytes=chunk if pr else 0)
                 stacks.append(se)
                 se.forward(X, Y)
                 for kind, k in [("in_order", 0)] + [("first_k", k) for k in ks]:
@@ -523,10 +532,13 @@ def main():
                 se.close()
             sweep = {}
             for kind, k in [("in_order", 0)] + [("first_k", k) for k in ks]:
-                on, off = times[("on", kind, k)], times[("off", kind, k)]
-                sweep[f"{kind}({k})"] = {"ms": on, "exposed_ms": max(0.0, on - off),
-                                         "hidden_fraction": 1.0 - max(0.0, on - off) / ar_total}
-            best = min((v["ms"], key) for key, v in sweep.items() if key.startswith("first_k"))[1]
+                off = times[("off", kind, k)]
+                for label, tag in (("on", ""), ("prio", "+prio")):
+                    on = times[(label, kind, k)]
+                    sweep[f"{kind}({k}){tag}"] = {"ms": on, "exposed_ms": max(0.0, on - off),
+                                                  "hidden_fraction": 1.0 - max(0.0, on - off) / ar_total}
+            best = min((v["ms"], key) for key, v in sweep.items() if key.startswith("first_k") and "+prio" not in key)[1]
+            best_p = min((v["ms"], key) for key, v in sweep.items() if "+prio" in key)[1]
             emulated = {"n": n, "link_GBps_per_direction": gbps, "latency_us_per_bucket": lat,
                         "bucket_layers": args.bucket_layers,
                         "note": "EMULATED all-reduce on one GPU (comm stream held for the ring time; no NCCL, no "
@@ -535,7 +547,11 @@ def main():
                         "allreduce_total_ms": ar_total, "in_order_ms": sweep["in_order(0)"]["ms"], "best": best,
                         "best_ms": sweep[best]["ms"], "best_exposed_ms": sweep[best]["exposed_ms"],
                         "best_hidden_fraction": sweep[best]["hidden_fraction"],
-                        "ooo_speedup_vs_in_order": sweep["in_order(0)"]["ms"] / sweep[best]["ms"], "k_sweep": sweep}
+                        "ooo_speedup_vs_in_order": sweep["in_order(0)"]["ms"] / sweep[best]["ms"],
+                        "prioritised": {"chunk_mb": args.comm_chunk_mb, "best": best_p, "best_ms": sweep[best_p]["ms"],
+                                        "best_hidden_fraction": sweep[best_p]["hidden_fraction"],
+                                        "speedup_vs_fifo_best": sweep[best]["ms"] / sweep[best_p]["ms"]},
+                        "k_sweep": sweep}
         except Exception as e:  # noqa: BLE001 -- the bench line must still be printed
             emulated = {"error": str(e)[:200]}
         finally:
@@ -699,6 +715,8 @@ def main():
                                 else "ooo_first_k"),
                    "k": k_best, "k_search_visited": visited,
                    "bucket_layers": args.bucket_layers, "parallelism": f"dp{world}",
+                   "comm": (f"prioritised, {args.comm_chunk_mb} MB chunks (Fig. 4(b))" if args.comm_priority
+                            else "FIFO in D's dW order"),
                    "timing": f"{args.steps} steps as {len(main_s['run_steps'])} back-to-back runs, interleaved "
                              f"with as many in_order runs (ABAB); value = steps / summed run time",
                    "l2": "working set (weights+activations+grads) >> 126 MB L2; no flush"},

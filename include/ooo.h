@@ -155,6 +155,20 @@ typedef struct {
                                   drive): beyond it the kernel traps and the CUDA context reports an
                                   error instead of hanging.  <= 0 = default: 4000 ms for a stack
                                   without a communicator, 120000 ms with one. */
+  int32_t comm_priority;       /* issue order of the all-reduce chunks on the comm stream (§5.1 P:180,
+                                  Fig. 4; ooo_comm_schedule): 0 = FIFO in D's dW order (Fig. 4(a)/(c));
+                                  1 = prioritised: the ready chunk of the lowest-layer bucket first
+                                  (Fig. 4(b)), planned per step from the engine planner's predicted dW
+                                  completion times (bf16 engine; the fp32 path stays FIFO) */
+  int32_t comm_model_gbps;     /* chunk-duration model of the prioritised order: ring bytes
+                                  2(N-1)/N x chunk bytes at this many GB/s + 8 us per call;
+                                  <= 0 = 700 (the emulated all-reduce uses its own parameters) */
+  int64_t comm_chunk_bytes;    /* > 0: every bucket's all-reduce is partitioned into chunks of at most
+                                  this many bytes (rounded down to 256 elements), with boundaries
+                                  fixed per stack -- so every schedule reduces the same element ranges
+                                  and stays bit-exact -- and the channel can switch buckets between
+                                  chunks (the partitioning of [28, 38] behind P:180); <= 0 = one
+                                  all-reduce per bucket */
 } ooo_stack_desc;
 
 /* ---------------------------------------------------------------- info */
@@ -215,6 +229,23 @@ ooo_status ooo_region_schedule(int32_t n_regions, const double *t_main, int32_t 
  * throughput is NULL.  Pure host function. */
 int32_t ooo_k_search(int32_t L, double (*throughput)(int32_t k, void *ctx), void *ctx, int32_t *visited,
                      int32_t *n_visited);
+
+/* Issue order of partitioned all-reduces on one FIFO channel (§5.1 P:180,
+ * Fig. 4(b); readings C1-C3 in DESIGN.md).  Pure host function.
+ *   n_buckets B; ready[B] = time bucket b's dW ops are complete; n_chunks[B]
+ *   >= 1; dur = chunk durations, bucket after bucket (sum n_chunks entries);
+ *   prio[B] = priority key (lower = more urgent: the bucket's first layer);
+ *   fifo_rank[B] = position in the FIFO order (NULL = bucket index).
+ *   policy 0 = FIFO: buckets by fifo_rank, chunks in order, each chunk
+ *   starting at max(channel free, ready); 1 = PRIORITY: whenever the channel
+ *   is free the next chunk of the ready bucket with the lowest prio (ties:
+ *   lower index) goes, an idle channel waits for the earliest ready bucket.
+ * Outputs (caller-owned): order_b / order_c = the (bucket, chunk) issue
+ * order (sum n_chunks entries); done[B] (may be NULL) = completion time of
+ * each bucket's last chunk.  OOO_ERR_INVALID_ARGUMENT on bad sizes. */
+ooo_status ooo_comm_schedule(int32_t n_buckets, const double *ready, const int32_t *n_chunks, const double *dur,
+                             const int32_t *prio, const int32_t *fifo_rank, int32_t policy, int32_t *order_b,
+                             int32_t *order_c, double *done);
 
 /* Extra bytes kept alive by deferring dW_1..dW_k (the memory cost of
  * deferral, §3; E8 at P:352-354): sum_{i=2..k} |dZ_i|. */
@@ -277,6 +308,12 @@ ooo_status ooo_join(ooo_stack *s, void *stream);
  * Buckets are issued from the last (layer L) to the first.  `stream` waits
  * for the all-reduces.  OOO_ERR_STATE for a stack without communicator. */
 ooo_status ooo_allreduce_buckets(ooo_stack *s, void *stream);
+
+/* The (bucket, chunk) order in which the most recently enqueued step issued
+ * its all-reduces on the comm stream (engine path; ooo_comm_schedule with
+ * desc.comm_priority).  *n = count (only the first `cap` are written).  An
+ * empty list for a stack that does not communicate. */
+ooo_status ooo_comm_issue_order(const ooo_stack *s, int32_t *bucket, int32_t *chunk, int32_t cap, int32_t *n);
 
 /* Plans OOO_SCHED_REGIONS (single-GPU multi-stream ooo, §4.1) for
  * this stack, by the paper's steps 1-5:

@@ -43,6 +43,9 @@ class StackDesc(ctypes.Structure):
         ("comm_enabled", c_int32),
         ("nccl_max_ctas", c_int32),
         ("wait_timeout_ms", c_int32),
+        ("comm_priority", c_int32),
+        ("comm_model_gbps", c_int32),
+        ("comm_chunk_bytes", c_int64),
     ]
 
 
@@ -72,7 +75,8 @@ EXPORTS = [
     "ooo_forward", "ooo_backward", "ooo_join", "ooo_graph_create", "ooo_graph_launch",
     "ooo_graph_destroy", "ooo_destroy", "ooo_tensor", "ooo_set_timing", "ooo_timing_read",
     "ooo_engine_plan", "ooo_region_schedule", "ooo_plan_regions", "ooo_region_plan", "ooo_k_search",
-    "ooo_allreduce_buckets", "ooo_graph_set_timing_slots", "ooo_graph_timing_read",
+    "ooo_allreduce_buckets", "ooo_graph_set_timing_slots", "ooo_graph_timing_read", "ooo_comm_schedule",
+    "ooo_comm_issue_order",
 ]
 
 _lib = None
@@ -145,6 +149,12 @@ def load() -> ctypes.CDLL:
     lib.ooo_tensor.argtypes = [c_void_p, c_int32, c_int32, POINTER(c_void_p), POINTER(c_int64)]
     lib.ooo_set_timing.restype = S
     lib.ooo_set_timing.argtypes = [c_void_p, c_int32]
+    lib.ooo_comm_issue_order.restype = S
+    lib.ooo_comm_issue_order.argtypes = [c_void_p, POINTER(c_int32), POINTER(c_int32), c_int32, POINTER(c_int32)]
+    lib.ooo_comm_schedule.restype = S
+    lib.ooo_comm_schedule.argtypes = [c_int32, POINTER(c_double), POINTER(c_int32), POINTER(c_double),
+                                      POINTER(c_int32), POINTER(c_int32), c_int32, POINTER(c_int32),
+                                      POINTER(c_int32), POINTER(c_double)]
     lib.ooo_graph_set_timing_slots.restype = S
     lib.ooo_graph_set_timing_slots.argtypes = [c_void_p, c_int32]
     lib.ooo_graph_timing_read.restype = S

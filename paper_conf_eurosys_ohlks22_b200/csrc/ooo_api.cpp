@@ -92,6 +92,7 @@ struct Plan {
   int L = 0, M = 0, dtype = 0, elt = 2, R = 0, nbuckets = 0;
   std::vector<LayerPlan> layer;  // index i-1
   std::vector<int> bucket_first, bucket_last;
+  std::vector<std::vector<int64_t>> chunk_start;   // [bucket] element offsets (in grads) of its chunks, + end
   size_t off_wpart = 0, wpart_bytes = 0;
   size_t workspace_bytes = 0;
   int64_t grad_elems = 0;
@@ -261,9 +262,17 @@ Plan make_plan(const ooo_stack_desc *d) {
   p.grad_elems = goff;
   p.bucket_first.resize(p.nbuckets);
   p.bucket_last.resize(p.nbuckets);
+  p.chunk_start.resize(p.nbuckets);
   for (int b = 0; b < p.nbuckets; ++b) {
     p.bucket_first[b] = b * d->bucket_layers + 1;
     p.bucket_last[b] = std::min(p.L, (b + 1) * d->bucket_layers);
+    // fixed chunk boundaries (schedule independent): NEXT-4 partitioning
+    const int64_t e0 = p.layer[p.bucket_first[b] - 1].goff_w;
+    const int64_t e1 = p.layer[p.bucket_last[b] - 1].goff_b + p.layer[p.bucket_last[b] - 1].dout;
+    int64_t ce = d->comm_chunk_bytes > 0 ? d->comm_chunk_bytes / p.elt / 256 * 256 : 0;
+    if (ce <= 0) ce = e1 - e0;
+    for (int64_t e = e0; e < e1; e += ce) p.chunk_start[b].push_back(e);
+    p.chunk_start[b].push_back(e1);
   }
   return p;
 }
@@ -377,6 +386,8 @@ struct ooo_stack {
   void *eng_dX = nullptr;
   bool eng_in_order = false;
   bool eng_comm = false;                      // the deferred backward's per-bucket S[dW] still to enqueue
+  std::vector<double> pred_dw;                // planner: predicted dW_i completion (us) of the last launch
+  std::vector<int> comm_b, comm_c;            // the last step's all-reduce chunk issue order (introspection)
   // region plan (OOO_SCHED_REGIONS, §4.1; ooo_plan_regions)
   bool has_regions = false;
   std::vector<int> reg_D;          // backward order D of the plan
@@ -540,11 +551,9 @@ ooo_status launch_seed_op(ooo_stack *s, const void *dY, cudaStream_t st, int pri
   return end_rec(tr, st, grid, 0, bytes);
 }
 
-ooo_status launch_allreduce(ooo_stack *s, int b) {
-  const int first = s->p.bucket_first[b], last = s->p.bucket_last[b];
-  const LayerPlan &f = s->p.layer[first - 1];
-  const LayerPlan &l = s->p.layer[last - 1];
-  const int64_t e0 = f.goff_w, e1 = l.goff_b + l.dout;
+// S[dW] of chunk c of bucket b (the whole bucket when it is not partitioned).
+ooo_status launch_allreduce(ooo_stack *s, int b, int c) {
+  const int64_t e0 = s->p.chunk_start[b][c], e1 = s->p.chunk_start[b][c + 1];
   if (s->emu_n > 1) {
     TimedRec *tr;
     OOO_TRY(begin_rec(s, s->comm, 5, b, 2, &tr));
@@ -567,6 +576,10 @@ ooo_status launch_allreduce(ooo_stack *s, int b) {
     const double n = s->d.world_size;
     OOO_TRY(end_rec(tr, s->comm, 0, 0, 2.0 * (n - 1) / n * (double)(e1 - e0) * s->p.elt));
   }
+  return OOO_OK;
+}
+ooo_status launch_allreduce(ooo_stack *s, int b) {
+  for (int c = 0; c + 1 < (int)s->p.chunk_start[b].size(); ++c) OOO_TRY(launch_allreduce(s, b, c));
   return OOO_OK;
 }
 
@@ -756,7 +769,7 @@ ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const 
   for (int i = 1; i <= p.L; ++i) pb.bucket[i - 1] = p.layer[i - 1].bucket;
   pb.crit = crit;
   pb.defer = defer;
-  const std::vector<pl::Unit> order = pl::schedule(pb, plan_model(), ooo::eng::kMaxOps);
+  const std::vector<pl::Unit> order = pl::schedule(pb, plan_model(), ooo::eng::kMaxOps, &s->pred_dw);
   if (order.empty()) return fail(OOO_ERR_UNSUPPORTED, "engine queue does not fit the op table (%d ops)", ooo::eng::kMaxOps);
   ooo::eng::Params P = {};
   P.M = p.M;
@@ -813,23 +826,60 @@ ooo_status engine_comm(ooo_stack *s) {
   static StreamValueFn wait_fn = stream_value_fn("cuStreamWaitValue32");
   static StreamValueFn write_fn = stream_value_fn("cuStreamWriteValue32");
   if (!wait_fn || !write_fn) return fail(OOO_ERR_CUDA, "stream memory operations unavailable");
-  std::vector<int> left(p.nbuckets), tiles(p.nbuckets, 0);
-  for (int b = 0; b < p.nbuckets; ++b) left[b] = p.bucket_last[b] - p.bucket_first[b] + 1;
+  const int nb = p.nbuckets;
+  std::vector<int> left(nb), tiles(nb, 0), rank(nb, 0), nch(nb);
+  for (int b = 0; b < nb; ++b) {
+    left[b] = p.bucket_last[b] - p.bucket_first[b] + 1;
+    nch[b] = (int)p.chunk_start[b].size() - 1;
+  }
   for (int i = 1; i <= L; ++i) {
     const LayerPlan &lp = p.layer[i - 1];
     tiles[lp.bucket] += ((lp.din + 127) / 128) * ((lp.dout + lp.ebn_dw - 1) / lp.ebn_dw);
   }
-  for (int op : s->D) {
-    if (op > 0) continue;
-    const int b = p.layer[-op - 1].bucket;
-    if (--left[b] != 0) continue;
-    CUresult r = wait_fn(s->comm, reinterpret_cast<CUdeviceptr>(s->ctr + p.cl.bucket_done + b),
-                         (cuuint32_t)tiles[b], CU_STREAM_WAIT_VALUE_GEQ);
-    if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWaitValue32 failed (%d)", (int)r);
-    OOO_TRY(launch_allreduce(s, b));
-    r = write_fn(s->comm, reinterpret_cast<CUdeviceptr>(s->ctr + p.cl.ar_done + b), 1, 0);
-    if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWriteValue32 failed (%d)", (int)r);
+  int pos = 0;   // FIFO = the order in which D completes each bucket's dW ops
+  for (int op : s->D)
+    if (op < 0 && --left[p.layer[-op - 1].bucket] == 0) rank[p.layer[-op - 1].bucket] = pos++;
+  // chunk issue order (§5.1, ooo_comm_schedule): FIFO, or prioritised
+  // from the planner's predicted bucket ready times and a ring-time model
+  std::vector<double> ready(nb, 0.0), dur;
+  std::vector<int32_t> prio(nb);
+  const bool emu = s->emu_n > 1;
+  const double n = emu ? s->emu_n : s->d.world_size;
+  const double gbps = emu ? s->emu_gbps : (s->d.comm_model_gbps > 0 ? s->d.comm_model_gbps : 700.0);
+  const double lat = emu ? s->emu_lat_us : 8.0;
+  for (int b = 0; b < nb; ++b) {
+    prio[b] = p.bucket_first[b];
+    for (int i = p.bucket_first[b]; i <= p.bucket_last[b]; ++i)
+      if (i - 1 < (int)s->pred_dw.size()) ready[b] = std::max(ready[b], s->pred_dw[i - 1]);
+    for (int c = 0; c < nch[b]; ++c) {
+      const double bytes = (double)(p.chunk_start[b][c + 1] - p.chunk_start[b][c]) * p.elt;
+      dur.push_back(lat + 2.0 * (n - 1) / n * bytes / (gbps * 1e3));   // us
+    }
   }
+  const int total = (int)dur.size();
+  std::vector<int32_t> ob(total), oc(total);
+  OOO_TRY(ooo_comm_schedule(nb, ready.data(), nch.data(), dur.data(), prio.data(), rank.data(),
+                            s->d.comm_priority ? 1 : 0, ob.data(), oc.data(), nullptr));
+  // per chunk: the bucket's dW counter (before its first chunk), the
+  // all-reduce, and after its last chunk the flag F_i waits on
+  std::vector<int> todo = nch;
+  std::vector<char> waited(nb, 0);
+  for (int j = 0; j < total; ++j) {
+    const int b = ob[j];
+    if (!waited[b]) {
+      CUresult r = wait_fn(s->comm, reinterpret_cast<CUdeviceptr>(s->ctr + p.cl.bucket_done + b),
+                           (cuuint32_t)tiles[b], CU_STREAM_WAIT_VALUE_GEQ);
+      if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWaitValue32 failed (%d)", (int)r);
+      waited[b] = 1;
+    }
+    OOO_TRY(launch_allreduce(s, b, oc[j]));
+    if (--todo[b] == 0) {
+      CUresult r = write_fn(s->comm, reinterpret_cast<CUdeviceptr>(s->ctr + p.cl.ar_done + b), 1, 0);
+      if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWriteValue32 failed (%d)", (int)r);
+    }
+  }
+  s->comm_b.assign(ob.begin(), ob.end());
+  s->comm_c.assign(oc.begin(), oc.end());
   return OOO_OK;
 }
 
@@ -1507,6 +1557,17 @@ ooo_status ooo_join(ooo_stack *s, void *stream) {
   OOO_TRY(engine_flush(s));
   OOO_TRY(join_into(s, static_cast<cudaStream_t>(stream)));
   return check_async(s);
+}
+
+ooo_status ooo_comm_issue_order(const ooo_stack *s, int32_t *bucket, int32_t *chunk, int32_t cap, int32_t *n) {
+  if (!s || !n) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
+  const int m = (int)s->comm_b.size();
+  for (int j = 0; j < m && j < cap; ++j) {
+    if (bucket) bucket[j] = s->comm_b[j];
+    if (chunk) chunk[j] = s->comm_c[j];
+  }
+  *n = m;
+  return OOO_OK;
 }
 
 ooo_status ooo_allreduce_buckets(ooo_stack *s, void *stream) {

@@ -211,7 +211,7 @@ std::vector<Unit> merge(const std::vector<Unit> &v) {
 //    workers it needs when its rows become ready);
 //  * else the critical row anyway (its worker waits), or the dW group if the
 //    chain cannot proceed.
-std::vector<Unit> plan_once(const Problem &pb, const Model &m, int group_rows) {
+std::vector<Unit> plan_once(const Problem &pb, const Model &m, int group_rows, std::vector<double> *dw_done) {
   Sim sim(pb, m, true);
   std::vector<Unit> def;   // dW ops split into row groups
   for (const Unit &u : pb.defer)
@@ -269,16 +269,20 @@ std::vector<Unit> plan_once(const Problem &pb, const Model &m, int group_rows) {
       out.push_back(def[di++]);
     }
   }
+  if (dw_done) {
+    dw_done->assign(pb.L, 0.0);
+    for (int i = 1; i <= pb.L; ++i) (*dw_done)[i - 1] = sim.op_done(WGRAD, i);
+  }
   return merge(out);
 }
 
 }  // namespace
 
-std::vector<Unit> schedule(const Problem &pb, const Model &m, int max_units) {
+std::vector<Unit> schedule(const Problem &pb, const Model &m, int max_units, std::vector<double> *dw_done) {
   int maxrows = 1;
   for (const Unit &u : pb.defer) maxrows = std::max(maxrows, u.mt);
   for (int g = 1;; g *= 2) {
-    std::vector<Unit> q = plan_once(pb, m, std::min(g, maxrows));
+    std::vector<Unit> q = plan_once(pb, m, std::min(g, maxrows), dw_done);
     if (q.empty() || (int)q.size() <= max_units || g >= maxrows) return (int)q.size() <= max_units ? q : std::vector<Unit>{};
   }
 }

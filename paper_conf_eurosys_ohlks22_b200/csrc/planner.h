@@ -60,7 +60,10 @@ struct Problem {
 // Returns the FIFO order as units (adjacent units of one op merged when
 // their rows are contiguous), using at most `max_units` entries (coarser dW
 // row groups if needed).  Empty on failure (dependency cycle).
-std::vector<Unit> schedule(const Problem &pb, const Model &m, int max_units);
+// dw_done (optional): predicted completion time (us from the launch) of every
+// dW_i in this launch (index i-1; 0 for dW ops not in it) -- the ready times
+// of the prioritised all-reduce order (comm_order.cpp).
+std::vector<Unit> schedule(const Problem &pb, const Model &m, int max_units, std::vector<double> *dw_done = nullptr);
 
 // True iff every unit's dependencies are emitted before it (test hook).
 bool topological(const Problem &pb, const std::vector<Unit> &order);

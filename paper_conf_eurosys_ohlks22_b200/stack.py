@@ -22,7 +22,8 @@ def _i32arr(vals):
 
 
 def _desc(dims, acts, tokens, dtype, need_input_grad=False, bucket_layers=1, max_temp_bytes=0,
-          world_size=1, rank=0, comm_enabled=True, nccl_max_ctas=0, wait_timeout_ms=0):
+          world_size=1, rank=0, comm_enabled=True, nccl_max_ctas=0, wait_timeout_ms=0, comm_priority=0,
+          comm_chunk_bytes=0, comm_model_gbps=0):
     keep = {}
     d = _lib.StackDesc()
     d.num_layers = len(acts)
@@ -40,6 +41,9 @@ def _desc(dims, acts, tokens, dtype, need_input_grad=False, bucket_layers=1, max
     d.comm_enabled = int(bool(comm_enabled))
     d.nccl_max_ctas = int(nccl_max_ctas)
     d.wait_timeout_ms = int(wait_timeout_ms)
+    d.comm_priority = int(comm_priority)
+    d.comm_chunk_bytes = int(comm_chunk_bytes)
+    d.comm_model_gbps = int(comm_model_gbps)
     return d, keep
 
 
@@ -117,6 +121,23 @@ def region_schedule(t_main, t_sub, speedup, ready, last_region=None, nbytes=None
     return S, kp.value
 
 
+def comm_schedule(ready, dur, prio, policy="priority", fifo_rank=None):
+    """The library's all-reduce chunk issue order (``ooo_comm_schedule``,
+    §5.1).  dur[b] = list of bucket b's chunk durations.  Returns
+    (order as [(b, c), ...], done[b])."""
+    B = len(ready)
+    nch = [len(d) for d in dur]
+    tot = sum(nch)
+    flat = [float(x) for d in dur for x in d]
+    ob, oc = (c_int32 * max(1, tot))(), (c_int32 * max(1, tot))()
+    done = (ctypes.c_double * max(1, B))()
+    fr = _i32arr(fifo_rank) if fifo_rank is not None else None
+    check(load().ooo_comm_schedule(int(B), (ctypes.c_double * max(1, B))(*ready), _i32arr(nch),
+                                   (ctypes.c_double * max(1, tot))(*flat), _i32arr(prio), fr,
+                                   {"fifo": 0, "priority": 1}[policy], ob, oc, done))
+    return [(ob[j], oc[j]) for j in range(tot)], list(done[:B])
+
+
 def get_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(_lib.UNIQUE_ID_BYTES)
     check(load().ooo_get_unique_id(buf))
@@ -187,7 +208,8 @@ class OooStack:
 
     def __init__(self, dims, acts, tokens, W, b, dtype="bf16", need_input_grad=False, bucket_layers=1,
                  max_temp_bytes=0, world_size=1, rank=0, unique_id: bytes | None = None,
-                 comm_enabled=True, nccl_max_ctas=0, wait_timeout_ms=0):
+                 comm_enabled=True, nccl_max_ctas=0, wait_timeout_ms=0, comm_priority=0, comm_chunk_bytes=0,
+                 comm_model_gbps=0):
         """unique_id: the NCCL bootstrap id (broadcast_unique_id); required
         for world_size > 1; with world_size == 1 it makes a one-rank
         communicator that runs the N > 1 data plane on one GPU."""
@@ -214,7 +236,8 @@ class OooStack:
         self.W, self.b = list(W), list(b)
         self.device = W[0].device
         d, keep = _desc(self.dims, self.acts, self.tokens, dtype, need_input_grad, bucket_layers,
-                        max_temp_bytes, world_size, rank, comm_enabled, nccl_max_ctas, wait_timeout_ms)
+                        max_temp_bytes, world_size, rank, comm_enabled, nccl_max_ctas, wait_timeout_ms,
+                        comm_priority, comm_chunk_bytes, comm_model_gbps)
         ws, gb = c_size_t(), c_size_t()
         check(lib.ooo_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)))
         self.workspace = torch.empty(ws.value, dtype=torch.uint8, device=self.device)
@@ -272,6 +295,14 @@ class OooStack:
 
     def join(self, stream=None):
         check(load().ooo_join(self._h, _stream_handle(stream)))
+
+    def comm_issue_order(self) -> list:
+        """(bucket, chunk) issue order of the last enqueued step's all-reduces."""
+        n = c_int32()
+        check(load().ooo_comm_issue_order(self._h, None, None, 0, ctypes.byref(n)))
+        b, c = (c_int32 * max(1, n.value))(), (c_int32 * max(1, n.value))()
+        check(load().ooo_comm_issue_order(self._h, b, c, n.value, ctypes.byref(n)))
+        return [(b[j], c[j]) for j in range(n.value)]
 
     def allreduce_buckets(self, stream=None):
         """Every bucket's all-reduce back to back on the stack's own

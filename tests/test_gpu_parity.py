@@ -541,3 +541,61 @@ def test_graph_timing_slots_every_launch():
     torch.cuda.synchronize()
     assert torch.equal(stk.grads_buf, base["raw"])
     stk.close()
+
+
+# ------------------- NEXT-4: prioritised, partitioned all-reduce issue (§5.1)
+def _valid_chunk_order(order, nchunks):
+    seen = {}
+    for b, c in order:
+        assert c == seen.get(b, 0), order
+        seen[b] = c + 1
+    assert seen == nchunks, (seen, nchunks)
+
+
+@pytest.mark.parametrize("mode", ["nccl", "emulated"])
+def test_bf16_prioritised_partitioned_comm_bit_exact(monkeypatch, mode):
+    """comm_priority=1 with 64 KiB chunks: the captured fused steps issue
+    every bucket's all-reduce as fixed chunks in the prioritised order (a
+    valid chunk order: each bucket's chunks in sequence, all present), and
+    give gradients / Y bit-identical to the plain stack over three steps,
+    for both schedules -- a one-rank NCCL communicator (real ncclAllReduce
+    per chunk) and the emulated 8-rank link."""
+    dims, acts = [256, 512, 256, 256, 512, 256], ["gelu", "id", "id", "gelu", "id"]
+    cases = [Case(dims, acts, 520, "bf16", step=t) for t in range(4)]
+    kw = dict(bucket_layers=2, comm_priority=1, comm_chunk_bytes=64 * 1024)
+    if mode == "nccl":
+        comm = _nccl_stack(cases[0], monkeypatch, **kw)
+    else:
+        monkeypatch.setenv("OOO_EMULATE_AR_N", "8")
+        monkeypatch.setenv("OOO_EMULATE_AR_GBPS", "50")
+        comm = cases[0].stack(**kw)
+        monkeypatch.delenv("OOO_EMULATE_AR_N")
+        monkeypatch.delenv("OOO_EMULATE_AR_GBPS")
+    plain = cases[0].stack(bucket_layers=2)
+    # chunk count per bucket: bucket bytes / 64 KiB (32768 bf16 elements), rounded up
+    nel = [dims[i] * dims[i + 1] + dims[i + 1] for i in range(len(acts))]
+    buckets = [sum(nel[j] for j in range(b, min(b + 2, len(acts)))) for b in range(0, len(acts), 2)]
+    nchunks = {b: -(-e // 32768) for b, e in enumerate(buckets)}
+    for kind, k in (("first_k", 5), ("in_order", 0)):
+        Xb = [to_dev(cases[0].X, "bf16") for _ in range(2)]
+        dYb = [to_dev(cases[0].dY, "bf16") for _ in range(2)]
+        Yb = [torch.empty(cases[0].M, dims[-1], dtype=torch.bfloat16, device="cuda") for _ in range(2)]
+        plain.forward(Xb[0], Yb[0])
+        comm.forward(Xb[1], Yb[1])
+        g = [plain.graph(Xb[0], Yb[0], dYb[0], kind, k), comm.graph(Xb[1], Yb[1], dYb[1], kind, k)]
+        _valid_chunk_order(comm.comm_issue_order(), nchunks)
+        for t in range(3):
+            for j in range(2):
+                dYb[j].copy_(to_dev(cases[t].dY, "bf16"))
+                Xb[j].copy_(to_dev(cases[t + 1].X, "bf16"))
+                g[j].launch()
+            torch.cuda.synchronize()
+            assert torch.equal(comm.grads_buf, plain.grads_buf), (kind, t)
+            assert torch.equal(Yb[0], Yb[1]), (kind, t)
+        for x in g:
+            x.close()
+    ref = cases[2].oracle(0)
+    _check(max_err({"Y": ref.Y[0], "dW": [to_np(w) for w in comm.dW], "db": [to_np(v) for v in comm.db],
+                    "dX": None}, ref), BF16_TOL)
+    plain.close()
+    comm.close()
