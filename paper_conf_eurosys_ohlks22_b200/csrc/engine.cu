@@ -406,6 +406,19 @@ __device__ __forceinline__ void prefetch_b(const CUtensorMap *mB, uint32_t sbase
   }
 }
 
+// L2 prefetch of the B operand (= W_j) slice a chain tile of layer j would
+// load: this CTA's columns [bn0, bn0 + bh) over all nkb k-blocks.
+template <int CG, bool B_MN>
+__device__ __forceinline__ void prefetch_b_l2(const CUtensorMap *mB, int bn0, int bh, int nkb) {
+  for (int kb = 0; kb < nkb; ++kb) {
+    if (B_MN) {
+      for (int c = 0; c < (bh + 63) / 64; ++c) tma_prefetch_l2_2d(mB, bn0 + 64 * c, kb * BK);
+    } else {
+      tma_prefetch_l2_2d(mB, kb * BK, bn0);
+    }
+  }
+}
+
 // Producer k-loop of one task, specialised per operand layout (no per-k-block
 // branches; stage / phase advanced incrementally): waits for a free ring
 // stage, then TMA-loads this CTA's A rows and its share of B, completing on
@@ -577,6 +590,22 @@ __global__ void __launch_bounds__(kThreads, 1)
           case 1: produce<CG, false, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, t, npre); break;
           case 0: produce<CG, false, false>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, t, npre); break;
           default: produce<CG, true, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, t, npre); break;
+        }
+        if (p.pf_dist > 0 && T.kind != EPI_WGRAD && T.m0 == 0) {
+          // the weights pf_dist layers ahead on this chain (F: upwards, dO:
+          // downwards), this tile's column slice -- issued after the tile's
+          // own loads, so they never queue behind the prefetch
+          const int j = T.kind == EPI_FWD ? T.layer + p.pf_dist : T.layer - p.pf_dist;
+          if (j >= 1 && j <= cl.L && o.mapB >= 0) {
+            const LayerDev &Lj = p.layers[j - 1];
+            const CUtensorMap *mBj = p.maps + o.mapB + (j - T.layer) * p.maps_per_layer;
+            const int nj = T.kind == EPI_FWD ? Lj.dout : Lj.din;        // output width of op j
+            const int kj = T.kind == EPI_FWD ? Lj.din : Lj.dout;        // its reduction length
+            if (bn0 < nj) {
+              if (b_mn) prefetch_b_l2<CG, true>(mBj, bn0, min(bh, nj - bn0), (kj + BK - 1) / BK);
+              else prefetch_b_l2<CG, false>(mBj, bn0, bh, (kj + BK - 1) / BK);
+            }
+          }
         }
       }
     }

@@ -89,6 +89,10 @@ struct Params {
                            // up to 8 when all tokens fit one 128-row tile (1-CTA tiles): the
                            // MMA's rows beyond it read stale smem and are never stored
   uint64_t timeout_ns;     // bound of every in-kernel wait (trap beyond it)
+  int32_t pf_dist;         // > 0: a chain tile of F_i (dO_i) also prefetches into L2 its slice of the
+                           // weights of layer i + pf_dist (i - pf_dist) -- skinny stacks, where every
+                           // chain op streams its W from HBM (W does not depend on the chain)
+  int32_t maps_per_layer;  // map-table slots per layer (the map of layer j = the op's map + (j-i) x this)
   const CUtensorMap *maps;
   int32_t *ctr;            // counter array base
   const LayerDev *layers;  // index i-1

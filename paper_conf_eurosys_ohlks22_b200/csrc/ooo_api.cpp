@@ -781,6 +781,11 @@ ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const 
   P.copy_nt = (s->dims[0] + copy_bn(s->dims[0]) - 1) / copy_bn(s->dims[0]);
   P.a_rows = a_box_rows(p);
   P.timeout_ns = (uint64_t)s->timeout_ms * 1000000ull;
+  // skinny stacks (the tokens fill at most two tile rows: C4, C5): every chain
+  // op streams its W_i from HBM; prefetch the weights a few layers ahead into
+  // L2 (OOO_PF_DIST overrides; 0 = off)
+  P.pf_dist = env_int("OOO_PF_DIST", pb.rows <= 2 ? 4 : 0);
+  P.maps_per_layer = MS_COUNT;
   P.maps = s->dmaps;
   P.ctr = s->ctr;
   P.layers = s->dlayers;
