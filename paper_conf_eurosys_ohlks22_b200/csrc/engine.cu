@@ -124,10 +124,28 @@ constexpr uint32_t TMEM_COLS = 512;
 // barrier; every wait follows that barrier.
 __shared__ uint64_t s_timeout_ns;
 
+#ifndef OOO_CG1_MAXBN
+#define OOO_CG1_MAXBN 256   // experiment: widest B share a 1-CTA stage holds
+#endif
+#ifndef OOO_CG1_STAGES
+#define OOO_CG1_STAGES 4
+#endif
+// 64-deep k-blocks per ring stage: 2 = one full-barrier wait and one MMA
+// commit per 128-deep stage (the MMA issuer's per-stage overhead halves; C4
+// 3.11 -> 2.92 ms, C2 neutral); 1-CTA stacks keep 1 (only 2 stages would fit:
+// C5 +2.7 %)
+#ifndef OOO_KPS2
+#define OOO_KPS2 2
+#endif
+#ifndef OOO_KPS1
+#define OOO_KPS1 1
+#endif
 template <int CG> struct Cfg {
-  static constexpr int B_BYTES = (kMaxBN / CG) * BK * 2;   // this CTA's share of B
-  static constexpr int STAGE = A_BYTES + B_BYTES;
-  static constexpr int STAGES = CG == 2 ? (kEpiWarps > 8 ? 5 : 6) : (kEpiWarps > 8 ? 3 : 4);
+  static constexpr int KPS = CG == 2 ? OOO_KPS2 : OOO_KPS1;
+  static constexpr int B_BYTES = (CG == 1 ? OOO_CG1_MAXBN : kMaxBN / CG) * BK * 2;   // this CTA's share of B
+  static constexpr int SUB = A_BYTES + B_BYTES;      // one k-block: A rows, then this CTA's B share
+  static constexpr int STAGE = SUB * KPS;
+  static constexpr int STAGES = (CG == 2 ? (kEpiWarps > 8 ? 5 : 6) : (kEpiWarps > 8 ? 3 : OOO_CG1_STAGES)) / KPS;
   static constexpr int RING = STAGE * STAGES;
   static constexpr int STG_OFF = RING;
   static constexpr int BAR_OFF = STG_OFF + STG_BYTES;
@@ -391,14 +409,17 @@ __device__ __forceinline__ void load_b(const CUtensorMap *mB, uint32_t sb, uint3
 template <int CG, bool B_MN>
 __device__ __forceinline__ void prefetch_b(const CUtensorMap *mB, uint32_t sbase, uint32_t bar_empty,
                                            uint32_t bar_full, uint32_t L_full, bool leader, uint32_t bytes, int bn0,
-                                           int bh, int it, int npre) {
+                                           int bh, int it, int npre, int nkb) {
   using C = Cfg<CG>;
   int s = it % C::STAGES;
   uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;
-  for (int kb = 0; kb < npre; ++kb) {
-    if (it + kb >= C::STAGES) mbar_wait_b(bar_empty + 8 * s, ph ^ 1u);
-    if (leader) mbar_expect_tx(bar_full + 8 * s, bytes);
-    load_b<CG, B_MN>(mB, sbase + s * C::STAGE + A_BYTES, L_full + 8 * s, bn0, bh, kb * BK);
+  for (int st = 0; st < npre; ++st) {
+    const int kc = min(C::KPS, nkb - st * C::KPS);        // k-blocks in this stage
+    if (it + st >= C::STAGES) mbar_wait_b(bar_empty + 8 * s, ph ^ 1u);
+    if (leader) mbar_expect_tx(bar_full + 8 * s, bytes * kc);
+    for (int sub = 0; sub < kc; ++sub)
+      load_b<CG, B_MN>(mB, sbase + s * C::STAGE + sub * C::SUB + A_BYTES, L_full + 8 * s, bn0, bh,
+                       (st * C::KPS + sub) * BK);
     if (++s == C::STAGES) {
       s = 0;
       ph ^= 1u;
@@ -429,30 +450,38 @@ __device__ __forceinline__ void produce(const TaskRt &T, const CUtensorMap *mA, 
                                         uint32_t bar_empty, uint32_t bar_full, uint32_t L_full, bool leader,
                                         uint32_t bytes, int am, int bn0, int bh, int &it, int t, int npre) {
   using C = Cfg<CG>;
+  const int nst = (T.nkb + C::KPS - 1) / C::KPS;         // ring stages of this task
   int s = it % C::STAGES;
   uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;   // phase of the stage's next fill
-  for (int kb = 0; kb < npre; ++kb) {
-    ktrace(t, kb, 0);
-    load_a<CG, A_MN>(mA, sbase + s * C::STAGE, L_full + 8 * s, am, kb * BK);
+  for (int st = 0; st < npre; ++st) {
+    const int kc = min(C::KPS, T.nkb - st * C::KPS);
+    for (int sub = 0; sub < kc; ++sub) {
+      ktrace(t, st * C::KPS + sub, 0);
+      load_a<CG, A_MN>(mA, sbase + s * C::STAGE + sub * C::SUB, L_full + 8 * s, am, (st * C::KPS + sub) * BK);
+    }
     if (++s == C::STAGES) {
       s = 0;
       ph ^= 1u;
     }
   }
-  for (int kb = npre; kb < T.nkb; ++kb) {
-    if (it + kb >= C::STAGES) mbar_wait_b(bar_empty + 8 * s, ph ^ 1u);
-    ktrace(t, kb, 0);
-    if (leader) mbar_expect_tx(bar_full + 8 * s, bytes);
+  for (int st = npre; st < nst; ++st) {
+    const int kc = min(C::KPS, T.nkb - st * C::KPS);
+    if (it + st >= C::STAGES) mbar_wait_b(bar_empty + 8 * s, ph ^ 1u);
+    if (leader) mbar_expect_tx(bar_full + 8 * s, bytes * kc);
     const uint32_t lb = L_full + 8 * s;
-    const uint32_t sa = sbase + s * C::STAGE;
-    load_a<CG, A_MN>(mA, sa, lb, am, kb * BK);
-    load_b<CG, B_MN>(mB, sa + A_BYTES, lb, bn0, bh, kb * BK);
+    for (int sub = 0; sub < kc; ++sub) {
+      const int kb = st * C::KPS + sub;
+      ktrace(t, kb, 0);
+      const uint32_t sa = sbase + s * C::STAGE + sub * C::SUB;
+      load_a<CG, A_MN>(mA, sa, lb, am, kb * BK);
+      load_b<CG, B_MN>(mB, sa + A_BYTES, lb, bn0, bh, kb * BK);
+    }
     if (++s == C::STAGES) {
       s = 0;
       ph ^= 1u;
     }
   }
-  it += T.nkb;
+  it += nst;
 }
 
 template <int CG>
@@ -579,9 +608,9 @@ __global__ void __launch_bounds__(kThreads, 1)
             wgate(p, T);
             asm volatile("fence.proxy.async.global;" ::: "memory");
           }
-          npre = min(T.nkb, C::STAGES);
-          if (b_mn) prefetch_b<CG, true>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre);
-          else prefetch_b<CG, false>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre);
+          npre = min((T.nkb + C::KPS - 1) / C::KPS, C::STAGES);   // ring stages claimed for W
+          if (b_mn) prefetch_b<CG, true>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre, T.nkb);
+          else prefetch_b<CG, false>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre, T.nkb);
         }
         deps<true>(p, T, T.mblk0 + (int)rank);    // this CTA's row block (no-op after a ready claim)
         asm volatile("fence.proxy.async.global;" ::: "memory");   // TMA reads see the producers' data
@@ -648,7 +677,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         int s = it % C::STAGES;
         uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;
 #if OOO_EARLY_WAIT
-        if (CG == 2) {
+        if (CG == 2 && C::KPS == 1) {
           // the barrier wait (+ fence) of k-block kb + 1 runs while kb's last
           // two MMAs execute, so the issuer's per-k-block overhead is covered
           // by queued tensor work; kb's stage is released right after
@@ -678,35 +707,40 @@ __global__ void __launch_bounds__(kThreads, 1)
           continue;
         }
 #endif
-        for (int kb = 0; kb < T.nkb; ++kb) {
-          ktrace(t, kb, 2);
+        const int nst = (T.nkb + C::KPS - 1) / C::KPS;
+        for (int st = 0; st < nst; ++st) {
+          const int kb0 = st * C::KPS;
+          const int kc = min(C::KPS, T.nkb - kb0);
+          ktrace(t, kb0, 2);
           mbar_wait_b(bar_full + 8 * s, ph);
-          ktrace(t, kb, 3);
-          if (kb == 0) etrace_gt(t, 6);           // first k-block landed
-          if (kb == T.nkb - 1) etrace_gt(t, 7);   // last k-block landed
+          ktrace(t, kb0, 3);
+          if (st == 0) etrace_gt(t, 6);           // first k-block landed
+          if (st == nst - 1) etrace_gt(t, 7);     // last k-block landed
           fence_after();
-          const uint64_t soff = (uint64_t)(s * (C::STAGE >> 4));
-          const uint64_t ad = a0 + soff, bd = b0 + soff;
-          if (CG == 2) {
-            umma_bf16_pair(dtm, ad, bd, ID, kb != 0 ? 1u : 0u);
-            umma_bf16_pair(dtm, ad + astep, bd + bstep, ID, 1u);
-            umma_bf16_pair(dtm, ad + 2 * astep, bd + 2 * bstep, ID, 1u);
-            umma_bf16_pair(dtm, ad + 3 * astep, bd + 3 * bstep, ID, 1u);
-            umma_commit_pair(bar_empty + 8 * s);
-            ktrace(t, kb, 4);
-          } else {
-            umma_bf16(dtm, ad, bd, ID, kb != 0 ? 1u : 0u);
-            umma_bf16(dtm, ad + astep, bd + bstep, ID, 1u);
-            umma_bf16(dtm, ad + 2 * astep, bd + 2 * bstep, ID, 1u);
-            umma_bf16(dtm, ad + 3 * astep, bd + 3 * bstep, ID, 1u);
-            umma_commit(bar_empty + 8 * s);
+          for (int sub = 0; sub < kc; ++sub) {
+            const uint64_t soff = (uint64_t)((s * C::STAGE + sub * C::SUB) >> 4);
+            const uint64_t ad = a0 + soff, bd = b0 + soff;
+            const uint32_t acc0 = (kb0 + sub) != 0 ? 1u : 0u;
+            if (CG == 2) {
+              umma_bf16_pair(dtm, ad, bd, ID, acc0);
+              umma_bf16_pair(dtm, ad + astep, bd + bstep, ID, 1u);
+              umma_bf16_pair(dtm, ad + 2 * astep, bd + 2 * bstep, ID, 1u);
+              umma_bf16_pair(dtm, ad + 3 * astep, bd + 3 * bstep, ID, 1u);
+            } else {
+              umma_bf16(dtm, ad, bd, ID, acc0);
+              umma_bf16(dtm, ad + astep, bd + bstep, ID, 1u);
+              umma_bf16(dtm, ad + 2 * astep, bd + 2 * bstep, ID, 1u);
+              umma_bf16(dtm, ad + 3 * astep, bd + 3 * bstep, ID, 1u);
+            }
           }
+          if (CG == 2) umma_commit_pair(bar_empty + 8 * s); else umma_commit(bar_empty + 8 * s);
+          ktrace(t, kb0, 4);
           if (++s == C::STAGES) {
             s = 0;
             ph ^= 1u;
           }
         }
-        it += T.nkb;
+        it += nst;
         if (CG == 2) umma_commit_pair(bar_tfull + 8 * acc); else umma_commit(bar_tfull + 8 * acc);
         etrace_gt(t, 5);                         // last MMA issued
       }

@@ -13,7 +13,7 @@
 using namespace ooo::tc;
 
 __global__ void __launch_bounds__(128, 1) probe(int iters, int bn, int a_mn, int b_mn, int wait_each,
-                                                long long *out) {
+                                                long long *out, int bm) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = smem_raw + ((1024u - (smem_u32(smem_raw) & 1023u)) & 1023u);
   const uint32_t sa = smem_u32(smem), sb = sa + 16384, bar = sa + 16384 + 32768;
@@ -35,7 +35,7 @@ __global__ void __launch_bounds__(128, 1) probe(int iters, int bn, int a_mn, int
   const uint32_t tmem = tslot;
   if (threadIdx.x == 0) {
     const uint32_t ID = (1u << 4) | (1u << 7) | (1u << 10) | ((a_mn ? 1u : 0u) << 15) | ((b_mn ? 1u : 0u) << 16) |
-                        ((uint32_t)(bn >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+                        ((uint32_t)(bn >> 3) << 17) | ((uint32_t)(bm >> 4) << 24);
     long long t0 = clock64();
     uint32_t ph = 0;
     for (int it = 0; it < iters; ++it) {
@@ -67,22 +67,29 @@ int main() {
   const int smem = 16384 + 32768 + 64 + 1024;
   cudaFuncSetAttribute(probe, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   const int iters = 4000;
-  struct C { int bn, a_mn, b_mn, wait; const char *name; } cs[] = {
-      {256, 0, 1, 0, "F   (A K-major, B MN-major) N=256"},
-      {256, 0, 0, 0, "dO  (A K-major, B K-major)  N=256"},
-      {256, 1, 1, 0, "dW  (A MN-major, B MN-major) N=256"},
-      {128, 0, 1, 0, "F   N=128"},
-      {256, 0, 1, 1, "F   N=256, commit+wait each k-block"},
+  struct C { int bn, a_mn, b_mn, wait, bm; const char *name; } cs[] = {
+      {256, 0, 1, 0, 128, "F   (A K-major, B MN-major) N=256"},
+      {256, 0, 0, 0, 128, "dO  (A K-major, B K-major)  N=256"},
+      {256, 1, 1, 0, 128, "dW  (A MN-major, B MN-major) N=256"},
+      {128, 0, 1, 0, 128, "F   N=128"},
+      {64, 0, 1, 0, 128, "F   N=64"},
+      {64, 0, 0, 0, 128, "dO  N=64"},
+      {32, 0, 0, 0, 128, "dO  N=32"},
+      {256, 0, 0, 0, 64, "dO  M=64 N=256"},
+      {64, 0, 0, 0, 64, "dO  M=64 N=64"},
+      {64, 0, 1, 0, 64, "F   M=64 N=64"},
+      {256, 0, 1, 1, 128, "F   N=256, commit+wait each k-block"},
+      {64, 0, 1, 1, 128, "F   N=64, commit+wait each k-block"},
   };
   for (auto &c : cs) {
-    probe<<<148, 128, smem>>>(iters, c.bn, c.a_mn, c.b_mn, c.wait, d);
+    probe<<<148, 128, smem>>>(iters, c.bn, c.a_mn, c.b_mn, c.wait, d, c.bm);
     cudaError_t e = cudaDeviceSynchronize();
     long long h[148];
     cudaMemcpy(h, d, sizeof(h), cudaMemcpyDeviceToHost);
     double m = 0;
     for (int i = 0; i < 148; ++i) m += h[i];
     m /= 148;
-    const double flop = 2.0 * 128 * c.bn * 64;   // per k-block per SM
+    const double flop = 2.0 * c.bm * c.bn * 64;   // per k-block per SM
     printf("%-40s %7.1f cycles per 64-deep k-block (%s); ideal %5.0f at 8192 FLOP/clk/SM\n", c.name, m / iters,
            cudaGetErrorString(e), flop / 8192);
   }
