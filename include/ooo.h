@@ -169,6 +169,9 @@ typedef struct {
                                   and stays bit-exact -- and the channel can switch buckets between
                                   chunks (the partitioning of [28, 38] behind P:180); <= 0 = one
                                   all-reduce per bucket */
+  int32_t engine_ctas;         /* > 0: at most this many CTAs (SMs) for the bf16 engine kernels of this
+                                  stack (one SM partition per pipeline stage, ooo_pipeline_*); <= 0 = all
+                                  SMs (minus the NCCL reserve of a communicating stack) */
 } ooo_stack_desc;
 
 /* ---------------------------------------------------------------- info */
@@ -299,6 +302,17 @@ ooo_status ooo_backward(ooo_stack *s, const void *dY, ooo_schedule sch, void *dX
 /* `stream` waits for all outstanding backward work, all-reduces included. */
 ooo_status ooo_join(ooo_stack *s, void *stream);
 
+/* Gradient fast-forwarding across pipeline stages (§5.2.1): make
+ * `stream` wait until the input gradient dX of this stack's last
+ * ooo_backward is complete -- in the middle of the engine kernel, as soon as
+ * the dO chain has produced dX and before the deferrable dW ops finish -- so
+ * the previous stage can start on it.  Launches the deferred backward kernel
+ * if it has not run yet (as ooo_join would, without joining it).  bf16
+ * engine stacks with need_input_grad only (OOO_ERR_UNSUPPORTED otherwise);
+ * OOO_ERR_STATE without a backward.  Like every mid-kernel wait on another
+ * stream, run it inside a captured graph (see ooo_forward). */
+ooo_status ooo_input_grad_wait(ooo_stack *s, void *stream);
+
 /* S[dW] of every bucket back to back on the stack's comm stream and
  * communicator, no compute (collective: every rank calls it): the
  * stand-alone all-reduce time the hidden fraction is measured against
@@ -354,6 +368,50 @@ ooo_status ooo_graph_launch(ooo_graph *g, void *stream);
 ooo_status ooo_graph_destroy(ooo_graph *g);
 
 ooo_status ooo_destroy(ooo_stack *s);             /* joins, then frees host/NCCL resources */
+
+/* --------------------------------------- cross-layer model parallelism (§5.2) */
+/* A stack of L layers split into groups of group_layers consecutive layers
+ * (the unit of allocation; the paper allocates transformer blocks),
+ * groups allocated to n_stages pipeline stages (GPUs): placement 0 =
+ * contiguous (G/n consecutive groups per stage, the conventional allocation,
+ * P:234), 1 = modulo (group j on stage j mod n, "modulo layer allocation",
+ * P:234-238).  One training iteration (no micro-batches, §5.2.1) = the
+ * forward of every group in layer order, then the backward from the last
+ * group: with fast_forward = 0 conventional backprop (each group in order, a
+ * stage starts after the next group's whole backward, P:101 / Fig. 5(a));
+ * with fast_forward = 1 gradient fast-forwarding (each group's dO chain first
+ * and its dX released mid-kernel to the previous group, whose backward
+ * overlaps this group's dW ops, Fig. 5(b)/(c)).
+ * This build runs the stages as SM partitions of the current GPU (148 / n SMs
+ * each, one stream per stage; the stage-to-stage activation / gradient
+ * hand-off is the receiving group's X_1 copy / seed read of the sender's
+ * buffer): the data plane of n GPUs on one device.  Gradients of group j are
+ * in its own gradient buffer (ooo_pipeline_grads_offset). */
+typedef struct ooo_pipeline ooo_pipeline;
+typedef struct {
+  int32_t num_layers;          /* L */
+  const int32_t *dims;         /* L+1 widths (as ooo_stack_desc) */
+  const int32_t *acts;         /* L activations */
+  int32_t tokens;              /* M */
+  int32_t group_layers;        /* >= 1, divides L */
+  int32_t n_stages;            /* >= 1; n_stages <= number of groups */
+  int32_t placement;           /* 0 contiguous, 1 modulo */
+  const void *const *W, *const *b;   /* L device pointers (bf16) */
+  void *workspace;             /* device, ooo_pipeline_query_sizes, 256-B aligned */
+  void *grads;                 /* device, ooo_pipeline_query_sizes: groups' gradient buffers back to back */
+} ooo_pipeline_desc;
+ooo_status ooo_pipeline_query_sizes(const ooo_pipeline_desc *d, size_t *workspace_bytes, size_t *grads_bytes);
+/* byte offset of group j's gradient buffer (layout of ooo_grad_offsets for the group's layers) */
+ooo_status ooo_pipeline_grads_offset(const ooo_pipeline_desc *d, int32_t group, int64_t *offset);
+ooo_status ooo_pipeline_create(const ooo_pipeline_desc *d, ooo_pipeline **out);
+/* Captures one iteration [forward(X) -> Y; backward(dY)] into a graph
+ * (launch / destroy with ooo_graph_launch / ooo_graph_destroy).  X [M][d_0],
+ * dY [M][d_L], Y [M][d_L]: caller device buffers, baked into the graph. */
+ooo_status ooo_pipeline_graph_create(ooo_pipeline *p, const void *X, const void *dY, void *Y, int32_t fast_forward,
+                                     ooo_graph **out);
+/* Stage of group j under the pipeline's placement; -1 if out of range. */
+int32_t ooo_pipeline_stage_of(const ooo_pipeline *p, int32_t group);
+ooo_status ooo_pipeline_destroy(ooo_pipeline *p);
 
 /* ------------------------------------------------- introspection / timing */
 /* Device pointer of an internal store (teacher-forced parity tests):

@@ -46,6 +46,23 @@ class StackDesc(ctypes.Structure):
         ("comm_priority", c_int32),
         ("comm_model_gbps", c_int32),
         ("comm_chunk_bytes", c_int64),
+        ("engine_ctas", c_int32),
+    ]
+
+
+class PipelineDesc(ctypes.Structure):
+    _fields_ = [
+        ("num_layers", c_int32),
+        ("dims", POINTER(c_int32)),
+        ("acts", POINTER(c_int32)),
+        ("tokens", c_int32),
+        ("group_layers", c_int32),
+        ("n_stages", c_int32),
+        ("placement", c_int32),
+        ("W", POINTER(c_void_p)),
+        ("b", POINTER(c_void_p)),
+        ("workspace", c_void_p),
+        ("grads", c_void_p),
     ]
 
 
@@ -76,7 +93,8 @@ EXPORTS = [
     "ooo_graph_destroy", "ooo_destroy", "ooo_tensor", "ooo_set_timing", "ooo_timing_read",
     "ooo_engine_plan", "ooo_region_schedule", "ooo_plan_regions", "ooo_region_plan", "ooo_k_search",
     "ooo_allreduce_buckets", "ooo_graph_set_timing_slots", "ooo_graph_timing_read", "ooo_comm_schedule",
-    "ooo_comm_issue_order",
+    "ooo_comm_issue_order", "ooo_input_grad_wait", "ooo_pipeline_query_sizes", "ooo_pipeline_grads_offset",
+    "ooo_pipeline_create", "ooo_pipeline_graph_create", "ooo_pipeline_stage_of", "ooo_pipeline_destroy",
 ]
 
 _lib = None
@@ -149,6 +167,20 @@ def load() -> ctypes.CDLL:
     lib.ooo_tensor.argtypes = [c_void_p, c_int32, c_int32, POINTER(c_void_p), POINTER(c_int64)]
     lib.ooo_set_timing.restype = S
     lib.ooo_set_timing.argtypes = [c_void_p, c_int32]
+    lib.ooo_input_grad_wait.restype = S
+    lib.ooo_input_grad_wait.argtypes = [c_void_p, c_void_p]
+    lib.ooo_pipeline_query_sizes.restype = S
+    lib.ooo_pipeline_query_sizes.argtypes = [POINTER(PipelineDesc), POINTER(c_size_t), POINTER(c_size_t)]
+    lib.ooo_pipeline_grads_offset.restype = S
+    lib.ooo_pipeline_grads_offset.argtypes = [POINTER(PipelineDesc), c_int32, POINTER(c_int64)]
+    lib.ooo_pipeline_create.restype = S
+    lib.ooo_pipeline_create.argtypes = [POINTER(PipelineDesc), POINTER(c_void_p)]
+    lib.ooo_pipeline_graph_create.restype = S
+    lib.ooo_pipeline_graph_create.argtypes = [c_void_p, c_void_p, c_void_p, c_void_p, c_int32, POINTER(c_void_p)]
+    lib.ooo_pipeline_stage_of.restype = c_int32
+    lib.ooo_pipeline_stage_of.argtypes = [c_void_p, c_int32]
+    lib.ooo_pipeline_destroy.restype = S
+    lib.ooo_pipeline_destroy.argtypes = [c_void_p]
     lib.ooo_comm_issue_order.restype = S
     lib.ooo_comm_issue_order.argtypes = [c_void_p, POINTER(c_int32), POINTER(c_int32), c_int32, POINTER(c_int32)]
     lib.ooo_comm_schedule.restype = S

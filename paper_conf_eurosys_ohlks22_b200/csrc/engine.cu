@@ -918,6 +918,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (et == 0 && mrow0 < T.M) {
           if (T.kind == EPI_FWD) red_release_add(ctr + cl.fwd_rows + (T.layer - 1) * cl.MT + mblk, 1);
           else if (T.layer >= 2) red_release_add(ctr + cl.dz_rows + (T.layer - 2) * cl.MT + mblk, 1);
+          else red_release_add(ctr + cl.dx_total, 1);   // dX (the input gradient a previous stage waits for)
           if (leader) etrace(t, 3);
         }
       }

@@ -69,12 +69,12 @@ static_assert(sizeof(LayerDev) == 128, "LayerDev layout");
 // Counter layout (int32, one region in the workspace; indices are absolute):
 //   [0] dispenser | [1] unused | fwd_rows[L][MT]: tiles done of row block m of X_{i+1} |
 //   xcopy[MT]: X_1 rows copied | dz_rows[L][MT] | dz_total[L] | dw_done[L] |
-//   bucket_done[nb] | ar_done[nb]
+//   bucket_done[nb] | ar_done[nb] | dx_total: tiles of dO_1's output (dX) published
 // A forward-only launch resets [0, fwd_end); a backward resets [0, total).
 struct CounterLayout {
   int L, MT, nb;
   int fwd_rows, xcopy, fwd_end;
-  int dz_rows, dz_total, dw_done, bucket_done, ar_done, total;
+  int dz_rows, dz_total, dw_done, bucket_done, ar_done, dx_total, total;
 };
 
 struct Params {

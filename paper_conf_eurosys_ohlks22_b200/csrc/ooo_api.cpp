@@ -255,7 +255,8 @@ Plan make_plan(const ooo_stack_desc *d) {
     cl.dw_done = cl.dz_total + p.L;
     cl.bucket_done = cl.dw_done + p.L;
     cl.ar_done = cl.bucket_done + p.nbuckets;
-    cl.total = cl.ar_done + p.nbuckets;
+    cl.dx_total = cl.ar_done + p.nbuckets;
+    cl.total = cl.dx_total + 1;
     p.off_ctr = take((size_t)cl.total * 4);
   }
   p.workspace_bytes = std::max<size_t>(off, 256);
@@ -1475,6 +1476,7 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
     const int reserve = s->comm_stack || s->emu_n > 1 ? (d->nccl_max_ctas > 0 ? d->nccl_max_ctas : 16) : 0;
     s->engine_ctas = std::max(1, sms - reserve);
     s->engine_ctas = std::min(s->engine_ctas, env_int("OOO_ENGINE_CTAS", s->engine_ctas));
+    if (d->engine_ctas > 0) s->engine_ctas = std::min(s->engine_ctas, d->engine_ctas);
   }
   int least = 0, greatest = 0;
   cudaError_t e = cudaDeviceGetStreamPriorityRange(&least, &greatest);
@@ -1563,6 +1565,23 @@ ooo_status ooo_join(ooo_stack *s, void *stream) {
   OOO_TRY(join_into(s, static_cast<cudaStream_t>(stream)));
   return check_async(s);
 }
+
+ooo_status ooo_input_grad_wait(ooo_stack *s, void *stream) {
+  if (!s) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL stack");
+  if (!s->p.engine || !s->d.need_input_grad)
+    return fail(OOO_ERR_UNSUPPORTED, "input-gradient wait needs a bf16 engine stack with need_input_grad");
+  if (!s->bwd_pending) return fail(OOO_ERR_STATE, "no backward to wait for");
+  OOO_TRY(engine_flush(s));   // the deferred backward kernel runs now (on hi)
+  static StreamValueFn wait_fn = stream_value_fn("cuStreamWaitValue32");
+  if (!wait_fn) return fail(OOO_ERR_CUDA, "stream memory operations unavailable");
+  // every 128-row block of dO_1's output, once per column tile (engine.cu: dx_total)
+  const uint32_t target = (uint32_t)(s->p.cl.MT * ((s->dims[0] + s->p.layer[0].ebn_dx - 1) / s->p.layer[0].ebn_dx));
+  CUresult r = wait_fn(static_cast<cudaStream_t>(stream), reinterpret_cast<CUdeviceptr>(s->ctr + s->p.cl.dx_total),
+                       target, CU_STREAM_WAIT_VALUE_GEQ);
+  if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWaitValue32 failed (%d)", (int)r);
+  return OOO_OK;
+}
+
 
 ooo_status ooo_comm_issue_order(const ooo_stack *s, int32_t *bucket, int32_t *chunk, int32_t cap, int32_t *n) {
   if (!s || !n) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
@@ -1824,6 +1843,17 @@ ooo_status ooo_region_plan(const ooo_stack *s, int32_t *n_regions, int32_t *k_pr
 }
 
 }  // extern "C"
+
+// ---- internal (pipeline.cpp): error message and graph wrapping
+namespace ooo {
+ooo_status set_error(ooo_status st, const char *msg) { return fail(st, "%s", msg); }
+ooo_graph *wrap_graph(cudaGraph_t g, cudaGraphExec_t e) {
+  ooo_graph *gr = new ooo_graph();
+  gr->graph = g;
+  gr->exec = e;
+  return gr;
+}
+}  // namespace ooo
 
 #ifdef OOO_TRACE
 // Debug builds only (libooo_trace.so): device buffer of [task][4] u64 stamps

@@ -23,7 +23,7 @@ def _i32arr(vals):
 
 def _desc(dims, acts, tokens, dtype, need_input_grad=False, bucket_layers=1, max_temp_bytes=0,
           world_size=1, rank=0, comm_enabled=True, nccl_max_ctas=0, wait_timeout_ms=0, comm_priority=0,
-          comm_chunk_bytes=0, comm_model_gbps=0):
+          comm_chunk_bytes=0, comm_model_gbps=0, engine_ctas=0):
     keep = {}
     d = _lib.StackDesc()
     d.num_layers = len(acts)
@@ -44,6 +44,7 @@ def _desc(dims, acts, tokens, dtype, need_input_grad=False, bucket_layers=1, max
     d.comm_priority = int(comm_priority)
     d.comm_chunk_bytes = int(comm_chunk_bytes)
     d.comm_model_gbps = int(comm_model_gbps)
+    d.engine_ctas = int(engine_ctas)
     return d, keep
 
 
@@ -209,7 +210,7 @@ class OooStack:
     def __init__(self, dims, acts, tokens, W, b, dtype="bf16", need_input_grad=False, bucket_layers=1,
                  max_temp_bytes=0, world_size=1, rank=0, unique_id: bytes | None = None,
                  comm_enabled=True, nccl_max_ctas=0, wait_timeout_ms=0, comm_priority=0, comm_chunk_bytes=0,
-                 comm_model_gbps=0):
+                 comm_model_gbps=0, engine_ctas=0):
         """unique_id: the NCCL bootstrap id (broadcast_unique_id); required
         for world_size > 1; with world_size == 1 it makes a one-rank
         communicator that runs the N > 1 data plane on one GPU."""
@@ -237,7 +238,7 @@ class OooStack:
         self.device = W[0].device
         d, keep = _desc(self.dims, self.acts, self.tokens, dtype, need_input_grad, bucket_layers,
                         max_temp_bytes, world_size, rank, comm_enabled, nccl_max_ctas, wait_timeout_ms,
-                        comm_priority, comm_chunk_bytes, comm_model_gbps)
+                        comm_priority, comm_chunk_bytes, comm_model_gbps, engine_ctas)
         ws, gb = c_size_t(), c_size_t()
         check(lib.ooo_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)))
         self.workspace = torch.empty(ws.value, dtype=torch.uint8, device=self.device)
@@ -371,6 +372,80 @@ class OooStack:
     def close(self):
         if getattr(self, "_h", None):
             load().ooo_destroy(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class Pipeline:
+    """Cross-layer model parallelism (§5.2.1): ooo_pipeline_create over
+    caller-owned torch buffers.  placement 'contiguous' | 'modulo'; the
+    stages are SM partitions of the current GPU (include/ooo.h)."""
+
+    def __init__(self, dims, acts, tokens, W, b, group_layers, n_stages, placement="modulo"):
+        import torch
+        lib = load()
+        self.dims, self.acts, self.tokens = [int(x) for x in dims], list(acts), int(tokens)
+        self.L = len(self.acts)
+        self.group_layers, self.n_stages = int(group_layers), int(n_stages)
+        self.G = self.L // self.group_layers
+        keep = {"dims": _i32arr(self.dims), "acts": _i32arr([_lib.ACTS[a] if isinstance(a, str) else a
+                                                             for a in self.acts])}
+        d = _lib.PipelineDesc()
+        d.num_layers = self.L
+        d.dims = ctypes.cast(keep["dims"], ctypes.POINTER(c_int32))
+        d.acts = ctypes.cast(keep["acts"], ctypes.POINTER(c_int32))
+        d.tokens = self.tokens
+        d.group_layers = self.group_layers
+        d.n_stages = self.n_stages
+        d.placement = {"contiguous": 0, "modulo": 1}[placement]
+        ws, gb = c_size_t(), c_size_t()
+        check(lib.ooo_pipeline_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)))
+        dev = W[0].device
+        self.workspace = torch.empty(ws.value, dtype=torch.uint8, device=dev)
+        self.grads_buf = torch.zeros(gb.value, dtype=torch.uint8, device=dev)
+        self.W, self.b = list(W), list(b)
+        keep["W"] = (c_void_p * self.L)(*[w.data_ptr() for w in self.W])
+        keep["b"] = (c_void_p * self.L)(*[x.data_ptr() for x in self.b])
+        d.W = ctypes.cast(keep["W"], ctypes.POINTER(c_void_p))
+        d.b = ctypes.cast(keep["b"], ctypes.POINTER(c_void_p))
+        d.workspace = self.workspace.data_ptr()
+        d.grads = self.grads_buf.data_ptr()
+        self._keep, self._desc = keep, d
+        h = c_void_p()
+        check(lib.ooo_pipeline_create(ctypes.byref(d), ctypes.byref(h)))
+        self._h = h
+        # gradient views: group j's buffer, laid out as ooo_grad_offsets of its layers
+        g = self.grads_buf.view(torch.bfloat16)
+        self.dW, self.db = [], []
+        for j in range(self.G):
+            off = c_int64()
+            check(lib.ooo_pipeline_grads_offset(ctypes.byref(d), j, ctypes.byref(off)))
+            lo = j * self.group_layers
+            offs = grad_offsets(self.dims[lo: lo + self.group_layers + 1], self.acts[lo: lo + self.group_layers],
+                                self.tokens)
+            base = off.value // 2
+            for i, (ow, ob) in enumerate(offs):
+                din, dout = self.dims[lo + i], self.dims[lo + i + 1]
+                self.dW.append(g[base + ow: base + ow + din * dout].view(din, dout))
+                self.db.append(g[base + ob: base + ob + dout])
+
+    def stage_of(self, group: int) -> int:
+        return int(load().ooo_pipeline_stage_of(self._h, int(group)))
+
+    def graph(self, X, dY, Y, fast_forward=True) -> StepGraph:
+        h = c_void_p()
+        check(load().ooo_pipeline_graph_create(self._h, c_void_p(X.data_ptr()), c_void_p(dY.data_ptr()),
+                                               c_void_p(Y.data_ptr()), int(bool(fast_forward)), ctypes.byref(h)))
+        return StepGraph(self, h, (X, dY, Y))
+
+    def close(self):
+        if getattr(self, "_h", None):
+            load().ooo_pipeline_destroy(self._h)
             self._h = None
 
     def __del__(self):

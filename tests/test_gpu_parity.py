@@ -599,3 +599,48 @@ def test_bf16_prioritised_partitioned_comm_bit_exact(monkeypatch, mode):
                     "dX": None}, ref), BF16_TOL)
     plain.close()
     comm.close()
+
+
+# ------------------- NEXT-3: cross-layer model parallelism (§5.2.1)
+@pytest.mark.parametrize("n_stages,placement", [(2, "modulo"), (2, "contiguous"), (3, "modulo")])
+def test_bf16_pipeline_fast_forward_and_modulo_bit_exact(n_stages, placement):
+    """Groups of 6 layers (BERT-shaped blocks at width 256, identity at every
+    group boundary) on n SM-partition stages: conventional backprop and
+    gradient fast-forwarding give bit-identical gradients and Y, equal to the
+    oracle's partitioned step (oracle/pipeline.py) within the bf16 gate, and
+    dW bit-identical to the unpartitioned engine stack (reading M2), over two
+    captured iterations."""
+    from oracle import pipeline as PL
+    from paper_conf_eurosys_ohlks22_b200.stack import Pipeline
+    h, blocks = 256, 6
+    dims, acts = [h], []
+    for _ in range(blocks):
+        dims += [h, h, h, h, 4 * h, h]
+        acts += ["id", "id", "id", "id", "gelu", "id"]
+    case = Case(dims, acts, 264, "bf16")
+    Wt = [to_dev(w, "bf16") for w in case.W]
+    bt = [to_dev(v, "bf16") for v in case.b]
+    X, dY = to_dev(case.X, "bf16"), to_dev(case.dY, "bf16")
+    outs = {}
+    for ff in (False, True):
+        pipe = Pipeline(dims, acts, case.M, Wt, bt, group_layers=6, n_stages=n_stages, placement=placement)
+        Y = torch.empty(case.M, dims[-1], dtype=torch.bfloat16, device="cuda")
+        g = pipe.graph(X, dY, Y, fast_forward=ff)
+        for _ in range(2):
+            g.launch()
+        torch.cuda.synchronize()
+        outs[ff] = (Y.clone(), pipe.grads_buf.clone(), [to_np(w) for w in pipe.dW], [to_np(v) for v in pipe.db])
+        g.close()
+        pipe.close()
+    assert torch.equal(outs[False][0], outs[True][0]) and torch.equal(outs[False][1], outs[True][1])
+    Yo, gW, gb = PL.mp_step(case.X, case.dY, case.W, case.b, acts, 6, "bf16")
+    _check({"Y": rel_fro(to_np(outs[True][0]), Yo),
+            "dW": max(rel_fro(a, r) for a, r in zip(outs[True][2], gW)),
+            "db": max(rel_fro(a, r) for a, r in zip(outs[True][3], gb))}, BF16_TOL)
+    stk = case.stack()
+    whole = case.run(stk, "first_k", 0)
+    stk.close()
+    assert all(np.array_equal(a, r) for a, r in zip(outs[True][2], whole["dW"]))
+    # db of a group's top layer comes from the seed kernel's column sums (another fp32
+    # summation order than the engine epilogue's): equal up to the final bf16 rounding
+    assert max(rel_fro(a, r) for a, r in zip(outs[True][3], whole["db"])) < 4e-3
