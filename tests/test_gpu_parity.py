@@ -634,9 +634,10 @@ def test_bf16_pipeline_fast_forward_and_modulo_bit_exact(n_stages, placement):
         pipe.close()
     assert torch.equal(outs[False][0], outs[True][0]) and torch.equal(outs[False][1], outs[True][1])
     Yo, gW, gb = PL.mp_step(case.X, case.dY, case.W, case.b, acts, 6, "bf16")
+    # 36 bf16 layers end to end: the G3 gate max(1e-2, 2 x the rounding random-walk floor)
     _check({"Y": rel_fro(to_np(outs[True][0]), Yo),
             "dW": max(rel_fro(a, r) for a, r in zip(outs[True][2], gW)),
-            "db": max(rel_fro(a, r) for a, r in zip(outs[True][3], gb))}, BF16_TOL)
+            "db": max(rel_fro(a, r) for a, r in zip(outs[True][3], gb))}, max(BF16_TOL, 2 * bf16_floor(len(acts))))
     stk = case.stack()
     whole = case.run(stk, "first_k", 0)
     stk.close()

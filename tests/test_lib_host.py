@@ -133,3 +133,32 @@ def test_degenerate_sizes_without_gpu(lib):
     for kind, k in [("in_order", 0), ("first_k", 0), ("first_k", 1), ("first_k", 5)]:
         assert stack.schedule_order(1, kind, k) == [-1]
         assert sorted(stack.schedule_order(1, kind, k, need_input_grad=True)) == [-1, 1]
+
+
+def test_pipeline_host_validation(lib):
+    """ooo_pipeline_* (cross-layer MP, §5.2.1): sizes and gradient offsets
+    without a GPU; invalid groupings are rejected."""
+    import ctypes
+    from paper_conf_eurosys_ohlks22_b200 import stack
+    dims, acts = [256] * 13, ["id"] * 12
+    d = _lib.PipelineDesc()
+    keep = (stack._i32arr(dims), stack._i32arr([0] * 12))
+    d.num_layers, d.tokens, d.group_layers, d.n_stages, d.placement = 12, 64, 3, 2, 1
+    d.dims = ctypes.cast(keep[0], ctypes.POINTER(ctypes.c_int32))
+    d.acts = ctypes.cast(keep[1], ctypes.POINTER(ctypes.c_int32))
+    ws, gb = ctypes.c_size_t(), ctypes.c_size_t()
+    assert lib.ooo_pipeline_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)) == 0
+    per_group = 3 * (256 * 256 + 256) * 2
+    assert gb.value >= 4 * per_group
+    offs = []
+    for j in range(4):
+        o = ctypes.c_int64()
+        assert lib.ooo_pipeline_grads_offset(ctypes.byref(d), j, ctypes.byref(o)) == 0
+        offs.append(o.value)
+    assert offs == sorted(offs) and all(b - a >= per_group for a, b in zip(offs, offs[1:]))
+    d.group_layers = 5                     # does not divide 12
+    assert lib.ooo_pipeline_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)) == 1
+    d.group_layers, d.n_stages = 3, 5      # more stages than groups
+    assert lib.ooo_pipeline_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)) == 1
+    d.n_stages, d.placement = 3, 0         # contiguous: stages must divide the groups
+    assert lib.ooo_pipeline_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)) == 1
