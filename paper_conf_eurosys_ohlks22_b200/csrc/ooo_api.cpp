@@ -113,7 +113,7 @@ int env_int(const char *name, int dflt) {
 // Engine tile width for an output of width N: the widest of 256/192/128/64
 // that divides N (the dataflow pipeline hides wave quantisation, so wider
 // tiles -- better MMA efficiency, less L2 traffic per FLOP -- win).
-int engine_bn(int N, bool chain, int cg, int row_tiles, int workers) {
+int engine_bn(int N, bool chain, int cg, int row_tiles, int workers, int K = 0) {
   int forced = env_int(chain ? "OOO_EBN_CHAIN" : "OOO_EBN_DW", 0);
   if (!forced) forced = env_int("OOO_EBN", 0);
   if (forced && N % forced == 0 && (cg == 1 || forced % 64 == 0) && (cg == 1 || forced >= 128)) return forced;
@@ -126,6 +126,18 @@ int engine_bn(int N, bool chain, int cg, int row_tiles, int workers) {
   if (chain && cg == 2 && N % 128 == 0 && row_tiles * (N / 128) <= workers) return 128;
   const int narrow = env_int("OOO_EBN_NARROW", 0);   // experiment: 192-wide tiles for N <= this
   if (narrow && cg == 1 && N <= narrow && N % 192 == 0) return 192;
+  // CTA-pair chain tiles: 192 wide when that still fits one wave and the op
+  // is not faster with 256 (a chain op is latency-bound: waves x (first load +
+  // k-blocks at the MMA issue rate, the same for N = 192 and 256 + an
+  // epilogue proportional to the width); OOO_CHAIN192=0 turns it off)
+  if (chain && cg == 2 && K > 0 && N % 256 == 0 && N % 192 == 0 && env_int("OOO_CHAIN192", 1)) {
+    auto cost = [&](int bn) {
+      const int tiles = row_tiles * ((N + bn - 1) / bn);
+      const int waves = (tiles + workers - 1) / workers;
+      return waves * (1.0 + ((K + 63) / 64) * 0.45 + 2.8 * bn / 256.0);
+    };
+    if (cost(192) < cost(256) * 0.98) return 192;
+  }
   // CTA pairs split B in halves of >= 64 columns: bn in {128, 256}
   return N % 256 == 0 ? 256 : 128;
 }
@@ -237,8 +249,8 @@ Plan make_plan(const ooo_stack_desc *d) {
     const int PT = (MT + p.cg - 1) / p.cg;                      // tile rows of F_i / dO_i
     for (int i = 1; i <= p.L; ++i) {
       LayerPlan &lp = p.layer[i - 1];
-      lp.ebn_fwd = engine_bn(lp.dout, true, p.cg, PT, workers);
-      lp.ebn_dx = engine_bn(lp.din, true, p.cg, PT, workers);
+      lp.ebn_fwd = engine_bn(lp.dout, true, p.cg, PT, workers, lp.din);
+      lp.ebn_dx = engine_bn(lp.din, true, p.cg, PT, workers, lp.dout);
       lp.ebn_dw = engine_bn(lp.dout, false, p.cg, PT, workers);
     }
     p.off_maps = take((size_t)p.L * MS_COUNT * sizeof(CUtensorMap));
