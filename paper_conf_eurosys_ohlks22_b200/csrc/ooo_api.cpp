@@ -126,11 +126,12 @@ int engine_bn(int N, bool chain, int cg, int row_tiles, int workers, int K = 0) 
   if (chain && cg == 2 && N % 128 == 0 && row_tiles * (N / 128) <= workers) return 128;
   const int narrow = env_int("OOO_EBN_NARROW", 0);   // experiment: 192-wide tiles for N <= this
   if (narrow && cg == 1 && N <= narrow && N % 192 == 0) return 192;
-  // CTA-pair chain tiles: 192 wide when that still fits one wave and the op
-  // is not faster with 256 (a chain op is latency-bound: waves x (first load +
-  // k-blocks at the MMA issue rate, the same for N = 192 and 256 + an
-  // epilogue proportional to the width); OOO_CHAIN192=0 turns it off)
-  if (chain && cg == 2 && K > 0 && N % 256 == 0 && N % 192 == 0 && env_int("OOO_CHAIN192", 1)) {
+  // experiment (off: OOO_CHAIN192=1 turns it on): CTA-pair chain tiles 192
+  // wide when that still fits one wave and the cost model (waves x (first
+  // load + k-blocks at the MMA issue rate + an epilogue proportional to the
+  // width)) prefers it.  Measured on C2: first-k neutral (2.285 vs 2.283 ms),
+  // in-order +5 % (3.46 vs 3.28); C3 unaffected (1024 % 192 != 0)
+  if (chain && cg == 2 && K > 0 && N % 256 == 0 && N % 192 == 0 && env_int("OOO_CHAIN192", 0)) {
     auto cost = [&](int bn) {
       const int tiles = row_tiles * ((N + bn - 1) / bn);
       const int waves = (tiles + workers - 1) / workers;
