@@ -367,6 +367,19 @@ ooo_status ooo_graph_create(ooo_stack *s, const void *X, void *Y, const void *dY
 ooo_status ooo_graph_launch(ooo_graph *g, void *stream);
 ooo_status ooo_graph_destroy(ooo_graph *g);
 
+/* A training step with HOST buffers (the end-to-end path): ooo_graph_upload
+ * copies the step's inputs X [M][d_0] and dY [M][d_L] from host memory into
+ * the device buffers baked into the graph, on `copy_stream`, after the
+ * graph's previous launch has finished reading them; ooo_graph_launch_host
+ * launches the step on `stream` once that upload is complete and then copies
+ * Y [M][d_L] back to host memory on `copy_stream` (Y_host is written when
+ * copy_stream reaches that point).  Pinned host memory makes the copies
+ * asynchronous.  Two graphs over two buffer sets, used alternately
+ * (upload(t+1); launch_host(t)), overlap the copies with the compute.  Stack
+ * step graphs only (not pipeline graphs: OOO_ERR_UNSUPPORTED). */
+ooo_status ooo_graph_upload(ooo_graph *g, const void *X_host, const void *dY_host, void *copy_stream);
+ooo_status ooo_graph_launch_host(ooo_graph *g, void *Y_host, void *stream, void *copy_stream);
+
 ooo_status ooo_destroy(ooo_stack *s);             /* joins, then frees host/NCCL resources */
 
 /* --------------------------------------- cross-layer model parallelism (§5.2) */

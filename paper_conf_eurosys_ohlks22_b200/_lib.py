@@ -95,6 +95,7 @@ EXPORTS = [
     "ooo_allreduce_buckets", "ooo_graph_set_timing_slots", "ooo_graph_timing_read", "ooo_comm_schedule",
     "ooo_comm_issue_order", "ooo_input_grad_wait", "ooo_pipeline_query_sizes", "ooo_pipeline_grads_offset",
     "ooo_pipeline_create", "ooo_pipeline_graph_create", "ooo_pipeline_stage_of", "ooo_pipeline_destroy",
+    "ooo_graph_upload", "ooo_graph_launch_host",
 ]
 
 _lib = None
@@ -167,6 +168,10 @@ def load() -> ctypes.CDLL:
     lib.ooo_tensor.argtypes = [c_void_p, c_int32, c_int32, POINTER(c_void_p), POINTER(c_int64)]
     lib.ooo_set_timing.restype = S
     lib.ooo_set_timing.argtypes = [c_void_p, c_int32]
+    lib.ooo_graph_upload.restype = S
+    lib.ooo_graph_upload.argtypes = [c_void_p, c_void_p, c_void_p, c_void_p]
+    lib.ooo_graph_launch_host.restype = S
+    lib.ooo_graph_launch_host.argtypes = [c_void_p, c_void_p, c_void_p, c_void_p]
     lib.ooo_input_grad_wait.restype = S
     lib.ooo_input_grad_wait.argtypes = [c_void_p, c_void_p]
     lib.ooo_pipeline_query_sizes.restype = S

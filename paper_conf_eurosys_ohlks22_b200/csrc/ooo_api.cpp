@@ -429,6 +429,12 @@ struct ooo_graph {
   std::vector<cudaEvent_t> sev;    // [slot][rec][2]
   int slots = 0;
   long launches = 0;
+  // host-buffer steps (ooo_graph_upload / ooo_graph_launch_host): the
+  // device buffers baked into the graph and the events ordering the copies
+  void *dX = nullptr, *dY = nullptr, *dYout = nullptr;
+  size_t x_bytes = 0, dy_bytes = 0, y_bytes = 0;
+  cudaEvent_t ev_in = nullptr, ev_done = nullptr;
+  bool launched = false;
 };
 
 namespace {
@@ -1662,6 +1668,11 @@ ooo_status ooo_graph_create(ooo_stack *s, const void *X, void *Y, const void *dY
   gr->s = s;
   gr->graph = g;
   gr->exec = ex;
+  gr->dX = const_cast<void *>(X);
+  gr->dY = const_cast<void *>(dY);
+  gr->dYout = Y;
+  gr->x_bytes = (size_t)s->p.M * s->dims[0] * s->p.elt;
+  gr->dy_bytes = gr->y_bytes = (size_t)s->p.M * s->dims[s->p.L] * s->p.elt;
   if (s->timing && s->rec_cursor > 0) {
     for (size_t j = 0; j < s->rec_cursor; ++j) gr->tinfo.push_back(s->recs[j].info);
     size_t nn = 0;
@@ -1739,8 +1750,38 @@ ooo_status ooo_graph_launch(ooo_graph *g, void *stream) {
   return OOO_OK;
 }
 
+ooo_status ooo_graph_upload(ooo_graph *g, const void *X_host, const void *dY_host, void *copy_stream) {
+  if (!g || !X_host || !dY_host) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (!g->dX) return fail(OOO_ERR_UNSUPPORTED, "not a stack step graph");
+  cudaStream_t cs = static_cast<cudaStream_t>(copy_stream);
+  if (!g->ev_in) {
+    CU_TRY(cudaEventCreateWithFlags(&g->ev_in, cudaEventDisableTiming));
+    CU_TRY(cudaEventCreateWithFlags(&g->ev_done, cudaEventDisableTiming));
+  }
+  if (g->launched) CU_TRY(cudaStreamWaitEvent(cs, g->ev_done, 0));   // the last launch has read X / dY
+  CU_TRY(cudaMemcpyAsync(g->dX, X_host, g->x_bytes, cudaMemcpyHostToDevice, cs));
+  CU_TRY(cudaMemcpyAsync(g->dY, dY_host, g->dy_bytes, cudaMemcpyHostToDevice, cs));
+  CU_TRY(cudaEventRecord(g->ev_in, cs));
+  return OOO_OK;
+}
+
+ooo_status ooo_graph_launch_host(ooo_graph *g, void *Y_host, void *stream, void *copy_stream) {
+  if (!g || !Y_host) return fail(OOO_ERR_INVALID_ARGUMENT, "NULL argument");
+  if (!g->ev_in) return fail(OOO_ERR_STATE, "ooo_graph_upload must precede ooo_graph_launch_host");
+  cudaStream_t st = static_cast<cudaStream_t>(stream), cs = static_cast<cudaStream_t>(copy_stream);
+  CU_TRY(cudaStreamWaitEvent(st, g->ev_in, 0));
+  OOO_TRY(ooo_graph_launch(g, stream));
+  CU_TRY(cudaEventRecord(g->ev_done, st));
+  g->launched = true;
+  CU_TRY(cudaStreamWaitEvent(cs, g->ev_done, 0));
+  CU_TRY(cudaMemcpyAsync(Y_host, g->dYout, g->y_bytes, cudaMemcpyDeviceToHost, cs));
+  return OOO_OK;
+}
+
 ooo_status ooo_graph_destroy(ooo_graph *g) {
   if (!g) return OOO_OK;
+  if (g->ev_in) cudaEventDestroy(g->ev_in);
+  if (g->ev_done) cudaEventDestroy(g->ev_done);
   for (cudaEvent_t e : g->sev) cudaEventDestroy(e);
   if (g->exec) cudaGraphExecDestroy(g->exec);
   if (g->graph) cudaGraphDestroy(g->graph);

@@ -176,6 +176,18 @@ class StepGraph:
     def launch(self, stream=None):
         check(load().ooo_graph_launch(self._h, _stream_handle(stream)))
 
+    def upload(self, X_host, dY_host, copy_stream):
+        """Host -> device copy of the step's inputs (pinned CPU tensors) into
+        the graph's buffers, on copy_stream (ooo_graph_upload)."""
+        check(load().ooo_graph_upload(self._h, c_void_p(X_host.data_ptr()), c_void_p(dY_host.data_ptr()),
+                                      _stream_handle(copy_stream)))
+
+    def launch_host(self, Y_host, stream=None, copy_stream=None):
+        """Launch after the upload, then copy Y back into the pinned CPU
+        tensor Y_host on copy_stream (ooo_graph_launch_host)."""
+        check(load().ooo_graph_launch_host(self._h, c_void_p(Y_host.data_ptr()), _stream_handle(stream),
+                                           _stream_handle(copy_stream)))
+
     def set_timing_slots(self, slots: int):
         """The next `slots` launches each record their own per-kernel CUDA
         events (graph captured with the stack's timing on)."""

@@ -645,3 +645,44 @@ def test_bf16_pipeline_fast_forward_and_modulo_bit_exact(n_stages, placement):
     # db of a group's top layer comes from the seed kernel's column sums (another fp32
     # summation order than the engine epilogue's): equal up to the final bf16 rounding
     assert max(rel_fro(a, r) for a, r in zip(outs[True][3], whole["db"])) < 4e-3
+
+
+def test_graph_host_buffer_steps():
+    """ooo_graph_upload / ooo_graph_launch_host (the e2e path bench.py times):
+    two graphs over two buffer sets used alternately with pinned host
+    buffers give, step for step, the Y (read back to host) and gradients of
+    the device-buffer path."""
+    cases = [Case([256, 512, 256, 256], ["gelu", "id", "id"], 264, "bf16", step=t) for t in range(4)]
+    ref = cases[0].stack()
+    stk = cases[0].stack()
+    bufs = []
+    for p in range(2):
+        X = to_dev(cases[0].X, "bf16")
+        dY = to_dev(cases[0].dY, "bf16")
+        Y = stk.forward(X)
+        torch.cuda.synchronize()
+        bufs.append({"g": stk.graph(X, Y, dY, "first_k", 1),
+                     "hX": torch.empty(X.shape, dtype=X.dtype, pin_memory=True),
+                     "hdY": torch.empty(dY.shape, dtype=dY.dtype, pin_memory=True),
+                     "hY": torch.empty(Y.shape, dtype=Y.dtype, pin_memory=True)})
+    # both graphs' buffers hold forward(cases[0].X) state; the stack's stores hold the last forward
+    cs = torch.cuda.Stream()
+    Xr = to_dev(cases[0].X, "bf16")
+    ref.forward(Xr)
+    for t in range(3):
+        b = bufs[t % 2]
+        b["hX"].copy_(torch.from_numpy(cases[t + 1].X).to(torch.bfloat16))
+        b["hdY"].copy_(torch.from_numpy(cases[t].dY).to(torch.bfloat16))
+        b["g"].upload(b["hX"], b["hdY"], cs)
+        b["g"].launch_host(b["hY"], torch.cuda.current_stream(), cs)
+        torch.cuda.synchronize()
+        ref.backward(to_dev(cases[t].dY, "bf16"), "first_k", 1)
+        ref.join()
+        Yr = ref.forward(to_dev(cases[t + 1].X, "bf16"))
+        torch.cuda.synchronize()
+        assert torch.equal(b["hY"], Yr.cpu()), t
+        assert torch.equal(stk.grads_buf, ref.grads_buf), t
+    for b in bufs:
+        b["g"].close()
+    stk.close()
+    ref.close()
