@@ -395,11 +395,21 @@ ooo_status ooo_destroy(ooo_stack *s);             /* joins, then frees host/NCCL
  * with fast_forward = 1 gradient fast-forwarding (each group's dO chain first
  * and its dX released mid-kernel to the previous group, whose backward
  * overlaps this group's dW ops, Fig. 5(b)/(c)).
- * This build runs the stages as SM partitions of the current GPU (148 / n SMs
- * each, one stream per stage; the stage-to-stage activation / gradient
- * hand-off is the receiving group's X_1 copy / seed read of the sender's
- * buffer): the data plane of n GPUs on one device.  Gradients of group j are
- * in its own gradient buffer (ooo_pipeline_grads_offset). */
+ * Two modes.  Without a communicator (nccl_unique_id NULL, world_size 1) the
+ * stages are SM partitions of the current GPU (148 / n SMs each, one stream
+ * per stage, hand-offs through device buffers): the data plane of n GPUs on
+ * one device.  With a communicator every rank is one stage (n_stages ==
+ * world_size), holds only its groups (ooo_pipeline_query_sizes then sizes
+ * that rank's buffers), uses all SMs but an NCCL reserve of 16, and hands
+ * activations and input gradients to the neighbouring stages with
+ * ncclSend / ncclRecv on a comm stream -- after the group's forward, and
+ * after its dX (fast-forwarding: ooo_input_grad_wait on the comm stream,
+ * mid-kernel) or its whole backward (conventional).  Every rank walks the
+ * groups in the same global order, so each pair of ranks posts matching
+ * send / recv sequences.  world_size 1 with a communicator = loopback: every
+ * group boundary is a send / recv to itself (the P2P data plane on one GPU).
+ * Gradients of group j (owned groups only) are in its own gradient buffer
+ * (ooo_pipeline_grads_offset). */
 typedef struct ooo_pipeline ooo_pipeline;
 typedef struct {
   int32_t num_layers;          /* L */
@@ -412,9 +422,13 @@ typedef struct {
   const void *const *W, *const *b;   /* L device pointers (bf16) */
   void *workspace;             /* device, ooo_pipeline_query_sizes, 256-B aligned */
   void *grads;                 /* device, ooo_pipeline_query_sizes: groups' gradient buffers back to back */
+  int32_t world_size;          /* 1, or the number of ranks (= n_stages) with a communicator */
+  int32_t rank;
+  const void *nccl_unique_id;  /* NULL: SM-partition stages on one GPU; else OOO_UNIQUE_ID_BYTES (rank 0's) */
 } ooo_pipeline_desc;
 ooo_status ooo_pipeline_query_sizes(const ooo_pipeline_desc *d, size_t *workspace_bytes, size_t *grads_bytes);
-/* byte offset of group j's gradient buffer (layout of ooo_grad_offsets for the group's layers) */
+/* byte offset of group j's gradient buffer (layout of ooo_grad_offsets for the group's layers);
+ * OOO_ERR_INVALID_ARGUMENT for a group another rank owns */
 ooo_status ooo_pipeline_grads_offset(const ooo_pipeline_desc *d, int32_t group, int64_t *offset);
 ooo_status ooo_pipeline_create(const ooo_pipeline_desc *d, ooo_pipeline **out);
 /* Captures one iteration [forward(X) -> Y; backward(dY)] into a graph

@@ -63,6 +63,9 @@ class PipelineDesc(ctypes.Structure):
         ("b", POINTER(c_void_p)),
         ("workspace", c_void_p),
         ("grads", c_void_p),
+        ("world_size", c_int32),
+        ("rank", c_int32),
+        ("nccl_unique_id", c_void_p),
     ]
 
 

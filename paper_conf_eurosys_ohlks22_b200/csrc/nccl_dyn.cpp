@@ -27,6 +27,10 @@ void load() {
   OOO_SYM(GetUniqueId, "ncclGetUniqueId")
   OOO_SYM(CommInitRank, "ncclCommInitRank")
   OOO_SYM(AllReduce, "ncclAllReduce")
+  OOO_SYM(Send, "ncclSend")
+  OOO_SYM(Recv, "ncclRecv")
+  OOO_SYM(GroupStart, "ncclGroupStart")
+  OOO_SYM(GroupEnd, "ncclGroupEnd")
   OOO_SYM(CommDestroy, "ncclCommDestroy")
   OOO_SYM(CommAbort, "ncclCommAbort")
   OOO_SYM(CommGetAsyncError, "ncclCommGetAsyncError")

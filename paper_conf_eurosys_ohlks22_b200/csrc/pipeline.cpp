@@ -15,10 +15,11 @@
 //             dO chain of group j has produced dX_j, in the middle of its
 //             engine kernel (ooo_input_grad_wait), so group j's dW ops overlap
 //             group j-1's backward on another stage (Fig. 5(b)/(c)).
-// Each group is an ooo_stack (the same engine kernels), restricted to its
-// stage's SM partition (engine_ctas = SMs / n); every stage has one stream.
-// The hand-off buffers (group outputs, input gradients) are in the
-// pipeline's workspace; on n GPUs they would be the NCCL send/recv buffers.
+// Each group is an ooo_stack (the same engine kernels).  Without a
+// communicator the stages are SM partitions of one GPU (engine_ctas = SMs /
+// n, one stream per stage, hand-offs through device buffers).  With one, each
+// rank is a stage holding only its groups and the hand-offs are ncclSend /
+// ncclRecv on a comm stream (loopback at world_size 1: self send / recv).
 #include <cuda_runtime.h>
 #include <string.h>
 
@@ -28,6 +29,7 @@
 
 #include "../../include/ooo.h"
 #include "internal.h"
+#include "nccl_dyn.h"
 
 namespace {
 
@@ -37,6 +39,8 @@ struct GroupDesc {
   int first = 0, nl = 0;    // first layer (0-based) and layer count
   std::vector<int32_t> dims, acts;
 };
+
+bool comm_mode(const ooo_pipeline_desc *d) { return d->nccl_unique_id != nullptr; }
 
 ooo_status check_desc(const ooo_pipeline_desc *d) {
   if (!d || !d->dims || !d->acts) return ooo::set_error(OOO_ERR_INVALID_ARGUMENT, "NULL pipeline desc");
@@ -48,6 +52,11 @@ ooo_status check_desc(const ooo_pipeline_desc *d) {
   if (d->placement != 0 && d->placement != 1) return ooo::set_error(OOO_ERR_INVALID_ARGUMENT, "placement 0 or 1");
   if (d->placement == 0 && G % d->n_stages != 0)
     return ooo::set_error(OOO_ERR_INVALID_ARGUMENT, "contiguous placement: n_stages must divide the groups");
+  if (d->world_size < 1 || d->rank < 0 || d->rank >= d->world_size)
+    return ooo::set_error(OOO_ERR_INVALID_ARGUMENT, "world_size / rank invalid");
+  if (comm_mode(d) ? d->n_stages != d->world_size : d->world_size != 1)
+    return ooo::set_error(OOO_ERR_INVALID_ARGUMENT,
+                          "with a communicator n_stages == world_size (one stage per rank); without one world_size 1");
   return OOO_OK;
 }
 
@@ -67,6 +76,12 @@ int stage_of(const ooo_pipeline_desc *d, int j) {
   if (j < 0 || j >= G) return -1;
   return d->placement == 1 ? j % d->n_stages : j / (G / d->n_stages);
 }
+// this process computes group j
+bool owned(const ooo_pipeline_desc *d, int j) { return !comm_mode(d) || stage_of(d, j) == d->rank; }
+// the boundary between groups j and j + 1 is an NCCL transfer
+bool xfer(const ooo_pipeline_desc *d, int j) {
+  return comm_mode(d) && (d->world_size == 1 || stage_of(d, j) != stage_of(d, j + 1));
+}
 
 ooo_stack_desc stack_desc(const ooo_pipeline_desc *d, const GroupDesc &g, int j, int sms) {
   ooo_stack_desc s;
@@ -80,11 +95,14 @@ ooo_stack_desc stack_desc(const ooo_pipeline_desc *d, const GroupDesc &g, int j,
   s.bucket_layers = g.nl;
   s.world_size = 1;
   s.comm_enabled = 1;
-  s.engine_ctas = std::max(2, sms / d->n_stages / 2 * 2);   // whole CTA pairs per stage partition
+  // one SM partition per stage; with NCCL, all SMs but the P2P kernels' reserve
+  s.engine_ctas = comm_mode(d) ? std::max(2, (sms - 16) / 2 * 2) : std::max(2, sms / d->n_stages / 2 * 2);
   if (d->W) s.W = d->W + g.first;
   if (d->b) s.b = d->b + g.first;
   return s;
 }
+
+size_t act_bytes(const ooo_pipeline_desc *d, int width) { return (size_t)d->tokens * width * 2; }
 
 }  // namespace
 
@@ -92,44 +110,62 @@ struct ooo_pipeline {
   ooo_pipeline_desc d;
   std::vector<int32_t> dims, acts;
   std::vector<GroupDesc> g;
-  std::vector<ooo_stack *> stk;
-  std::vector<cudaStream_t> st;              // one per stage
-  std::vector<void *> out, dx;               // group j's output (j < G-1) / input gradient (j > 0)
-  std::vector<cudaEvent_t> ev_f, ev_b;       // forward done / input gradient released, per group
-  cudaEvent_t ev_fork = nullptr;
+  std::vector<ooo_stack *> stk;              // null for groups another rank owns
+  std::vector<cudaStream_t> st;              // one per stage (this rank's only, with a communicator)
+  std::vector<void *> out, in, dxs, dyr;     // per group: output, input, dX sent, dY received
+  std::vector<cudaEvent_t> ev_f, ev_b, ev_xf, ev_xb;   // forward done / dX released / recv done (fwd, bwd)
+  cudaEvent_t ev_fork = nullptr, ev_cj = nullptr;
   std::vector<cudaEvent_t> ev_join;          // per stage
+  cudaStream_t comm = nullptr;
+  const ooo::NcclApi *api = nullptr;
+  ncclComm_t nccl = nullptr;
+  std::vector<char> uid;
 };
 
 namespace {
 
-// sizes: per group workspace + grads; hand-off buffers (outputs, input grads)
-ooo_status plan_sizes(const ooo_pipeline_desc *d, std::vector<size_t> *ws_off, std::vector<size_t> *gr_off,
-                      std::vector<size_t> *out_off, std::vector<size_t> *dx_off, size_t *ws_total,
-                      size_t *gr_total) {
+// Per owned group: stack workspace and gradients; hand-off buffers.  Without
+// a communicator (or inside one rank) group j's input is group j-1's output
+// and its dY is group j+1's dX; across an NCCL boundary the receiver has its
+// own buffer.
+struct Layout {
+  std::vector<size_t> ws, gr, out, in, dxs, dyr;   // SIZE_MAX: none / aliased
+  size_t ws_total = 0, gr_total = 0;
+};
+
+ooo_status plan_sizes(const ooo_pipeline_desc *d, Layout *lay) {
   ooo_status st = check_desc(d);
   if (st != OOO_OK) return st;
   std::vector<GroupDesc> g = groups_of(d);
   const int G = (int)g.size();
   size_t ws = 0, gr = 0;
+  auto take = [&](size_t bytes) {
+    size_t o = ws;
+    ws += align256(bytes);
+    return o;
+  };
+  lay->ws.assign(G, SIZE_MAX);
+  lay->gr.assign(G, SIZE_MAX);
+  lay->out.assign(G, SIZE_MAX);
+  lay->in.assign(G, SIZE_MAX);
+  lay->dxs.assign(G, SIZE_MAX);
+  lay->dyr.assign(G, SIZE_MAX);
   for (int j = 0; j < G; ++j) {
+    if (!owned(d, j)) continue;
     ooo_stack_desc sd = stack_desc(d, g[j], j, 148);
     size_t w = 0, b = 0;
     if ((st = ooo_query_sizes(&sd, &w, &b)) != OOO_OK) return st;
-    if (ws_off) ws_off->push_back(ws);
-    if (gr_off) gr_off->push_back(gr);
-    ws += align256(w);
+    lay->ws[j] = take(w);
+    lay->gr[j] = gr;
     gr += align256(b);
+    const int din = d->dims[g[j].first], dout = d->dims[g[j].first + g[j].nl];
+    if (j < G - 1) lay->out[j] = take(act_bytes(d, dout));
+    if (j > 0) lay->dxs[j] = take(act_bytes(d, din));
+    if (j > 0 && xfer(d, j - 1)) lay->in[j] = take(act_bytes(d, din));
+    if (j < G - 1 && xfer(d, j)) lay->dyr[j] = take(act_bytes(d, dout));
   }
-  for (int j = 0; j < G; ++j) {   // group outputs (inputs of the next group) and input gradients
-    const size_t ob = (size_t)d->tokens * d->dims[g[j].first + g[j].nl] * 2;
-    const size_t ib = (size_t)d->tokens * d->dims[g[j].first] * 2;
-    if (out_off) out_off->push_back(j < G - 1 ? ws : SIZE_MAX);
-    if (j < G - 1) ws += align256(ob);
-    if (dx_off) dx_off->push_back(j > 0 ? ws : SIZE_MAX);
-    if (j > 0) ws += align256(ib);
-  }
-  *ws_total = std::max<size_t>(ws, 256);
-  *gr_total = std::max<size_t>(gr, 256);
+  lay->ws_total = std::max<size_t>(ws, 256);
+  lay->gr_total = std::max<size_t>(gr, 256);
   return OOO_OK;
 }
 
@@ -139,17 +175,22 @@ extern "C" {
 
 ooo_status ooo_pipeline_query_sizes(const ooo_pipeline_desc *d, size_t *workspace_bytes, size_t *grads_bytes) {
   if (!workspace_bytes || !grads_bytes) return ooo::set_error(OOO_ERR_INVALID_ARGUMENT, "NULL output");
-  return plan_sizes(d, nullptr, nullptr, nullptr, nullptr, workspace_bytes, grads_bytes);
+  Layout lay;
+  ooo_status st = plan_sizes(d, &lay);
+  if (st != OOO_OK) return st;
+  *workspace_bytes = lay.ws_total;
+  *grads_bytes = lay.gr_total;
+  return OOO_OK;
 }
 
 ooo_status ooo_pipeline_grads_offset(const ooo_pipeline_desc *d, int32_t group, int64_t *offset) {
   if (!offset) return ooo::set_error(OOO_ERR_INVALID_ARGUMENT, "NULL output");
-  std::vector<size_t> gr;
-  size_t w = 0, b = 0;
-  ooo_status st = plan_sizes(d, nullptr, &gr, nullptr, nullptr, &w, &b);
+  Layout lay;
+  ooo_status st = plan_sizes(d, &lay);
   if (st != OOO_OK) return st;
-  if (group < 0 || group >= (int)gr.size()) return ooo::set_error(OOO_ERR_INVALID_ARGUMENT, "group out of range");
-  *offset = (int64_t)gr[group];
+  if (group < 0 || group >= (int)lay.gr.size() || lay.gr[group] == SIZE_MAX)
+    return ooo::set_error(OOO_ERR_INVALID_ARGUMENT, "group out of range or owned by another rank");
+  *offset = (int64_t)lay.gr[group];
   return OOO_OK;
 }
 
@@ -159,12 +200,16 @@ ooo_status ooo_pipeline_destroy(ooo_pipeline *p) {
   if (!p) return OOO_OK;
   for (ooo_stack *s : p->stk)
     if (s) ooo_destroy(s);
+  if (p->comm) cudaStreamSynchronize(p->comm);
+  if (p->nccl && p->api) p->api->CommDestroy(p->nccl);
   for (cudaStream_t s : p->st)
     if (s) cudaStreamDestroy(s);
-  for (cudaEvent_t e : p->ev_f) if (e) cudaEventDestroy(e);
-  for (cudaEvent_t e : p->ev_b) if (e) cudaEventDestroy(e);
-  for (cudaEvent_t e : p->ev_join) if (e) cudaEventDestroy(e);
+  if (p->comm) cudaStreamDestroy(p->comm);
+  for (auto *v : {&p->ev_f, &p->ev_b, &p->ev_xf, &p->ev_xb, &p->ev_join})
+    for (cudaEvent_t e : *v)
+      if (e) cudaEventDestroy(e);
   if (p->ev_fork) cudaEventDestroy(p->ev_fork);
+  if (p->ev_cj) cudaEventDestroy(p->ev_cj);
   delete p;
   return OOO_OK;
 }
@@ -172,9 +217,8 @@ ooo_status ooo_pipeline_destroy(ooo_pipeline *p) {
 ooo_status ooo_pipeline_create(const ooo_pipeline_desc *d, ooo_pipeline **out) {
   if (!out) return ooo::set_error(OOO_ERR_INVALID_ARGUMENT, "NULL output");
   *out = nullptr;
-  std::vector<size_t> wso, gro, oo, dxo;
-  size_t wt = 0, gt = 0;
-  ooo_status st = plan_sizes(d, &wso, &gro, &oo, &dxo, &wt, &gt);
+  Layout lay;
+  ooo_status st = plan_sizes(d, &lay);
   if (st != OOO_OK) return st;
   if (!d->W || !d->b || !d->workspace || !d->grads)
     return ooo::set_error(OOO_ERR_INVALID_ARGUMENT, "W/b/workspace/grads NULL");
@@ -186,7 +230,13 @@ ooo_status ooo_pipeline_create(const ooo_pipeline_desc *d, ooo_pipeline **out) {
   p->acts.assign(d->acts, d->acts + d->num_layers);
   p->d.dims = p->dims.data();
   p->d.acts = p->acts.data();
+  if (d->nccl_unique_id) {                 // keep a copy: the mode (comm_mode) is read at every capture
+    p->uid.assign(static_cast<const char *>(d->nccl_unique_id),
+                  static_cast<const char *>(d->nccl_unique_id) + OOO_UNIQUE_ID_BYTES);
+    p->d.nccl_unique_id = p->uid.data();
+  }
   p->g = groups_of(&p->d);
+  const bool cm = comm_mode(d);
   const int G = (int)p->g.size();
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
@@ -196,88 +246,161 @@ ooo_status ooo_pipeline_create(const ooo_pipeline_desc *d, ooo_pipeline **out) {
     ooo_pipeline_destroy(p);
     return s;
   };
+  auto at = [&](size_t o) { return o == SIZE_MAX ? nullptr : static_cast<void *>(ws + o); };
+  p->stk.assign(G, nullptr);
+  p->out.assign(G, nullptr);
+  p->in.assign(G, nullptr);
+  p->dxs.assign(G, nullptr);
+  p->dyr.assign(G, nullptr);
   for (int j = 0; j < G; ++j) {
-    ooo_stack_desc sd = stack_desc(&p->d, p->g[j], j, sms);
-    size_t w = 0, b = 0;
-    if ((st = ooo_query_sizes(&sd, &w, &b)) != OOO_OK) return bail(st);
-    sd.workspace = ws + wso[j];
-    sd.grads = gr + gro[j];
-    ooo_stack *s = nullptr;
-    if ((st = ooo_create_stack(&sd, &s)) != OOO_OK) return bail(st);
-    p->stk.push_back(s);
-    p->out.push_back(oo[j] == SIZE_MAX ? nullptr : ws + oo[j]);
-    p->dx.push_back(dxo[j] == SIZE_MAX ? nullptr : ws + dxo[j]);
+    if (!owned(d, j)) continue;
+    ooo_stack_desc sd = stack_desc(d, p->g[j], j, sms);
+    sd.workspace = ws + lay.ws[j];
+    sd.grads = gr + lay.gr[j];
+    if ((st = ooo_create_stack(&sd, &p->stk[j])) != OOO_OK) return bail(st);
+    p->out[j] = at(lay.out[j]);
+    p->in[j] = at(lay.in[j]);
+    p->dxs[j] = at(lay.dxs[j]);
+    p->dyr[j] = at(lay.dyr[j]);
+  }
+  for (int j = 0; j < G; ++j) {   // same-process boundaries: the buffers are shared
+    if (!owned(d, j)) continue;
+    if (j > 0 && !xfer(d, j - 1)) p->in[j] = p->out[j - 1];
+    if (j < G - 1 && !xfer(d, j)) p->dyr[j] = p->dxs[j + 1];
   }
   int lo = 0, hi = 0;
   cudaDeviceGetStreamPriorityRange(&lo, &hi);
-  p->st.assign(d->n_stages, nullptr);
-  p->ev_join.assign(d->n_stages, nullptr);
-  for (int k = 0; k < d->n_stages; ++k) {
+  const int nst = cm ? 1 : d->n_stages;    // with a communicator this process is one stage
+  p->st.assign(nst, nullptr);
+  p->ev_join.assign(nst, nullptr);
+  for (int k = 0; k < nst; ++k) {
     if (cudaStreamCreateWithPriority(&p->st[k], cudaStreamNonBlocking, hi) != cudaSuccess ||
         cudaEventCreateWithFlags(&p->ev_join[k], cudaEventDisableTiming) != cudaSuccess)
       return bail(ooo::set_error(OOO_ERR_CUDA, "stage stream / event create failed"));
   }
-  p->ev_f.assign(G, nullptr);
-  p->ev_b.assign(G, nullptr);
-  for (int j = 0; j < G; ++j)
-    if (cudaEventCreateWithFlags(&p->ev_f[j], cudaEventDisableTiming) != cudaSuccess ||
-        cudaEventCreateWithFlags(&p->ev_b[j], cudaEventDisableTiming) != cudaSuccess)
-      return bail(ooo::set_error(OOO_ERR_CUDA, "event create failed"));
-  if (cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming) != cudaSuccess)
+  for (auto *v : {&p->ev_f, &p->ev_b, &p->ev_xf, &p->ev_xb}) {
+    v->assign(G, nullptr);
+    for (cudaEvent_t &e : *v)
+      if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+        return bail(ooo::set_error(OOO_ERR_CUDA, "event create failed"));
+  }
+  if (cudaEventCreateWithFlags(&p->ev_fork, cudaEventDisableTiming) != cudaSuccess ||
+      cudaEventCreateWithFlags(&p->ev_cj, cudaEventDisableTiming) != cudaSuccess)
     return bail(ooo::set_error(OOO_ERR_CUDA, "event create failed"));
+  if (cm) {
+    const char *why = nullptr;
+    p->api = ooo::nccl_api(&why);
+    if (!p->api) return bail(ooo::set_error(OOO_ERR_NCCL, why ? why : "NCCL unavailable"));
+    if (cudaStreamCreateWithPriority(&p->comm, cudaStreamNonBlocking, hi) != cudaSuccess)
+      return bail(ooo::set_error(OOO_ERR_CUDA, "comm stream create failed"));
+    ncclUniqueId id;
+    memcpy(&id, d->nccl_unique_id, sizeof(id));
+    ncclResult_t r;
+    if (p->api->CommInitRankConfig) {
+      ncclConfig_t cfg = NCCL_CONFIG_INITIALIZER;
+      cfg.maxCTAs = 16;                      // the SMs the engines leave free
+      r = p->api->CommInitRankConfig(&p->nccl, d->world_size, id, d->rank, &cfg);
+    } else {
+      r = p->api->CommInitRank(&p->nccl, d->world_size, id, d->rank);
+    }
+    if (r != ncclSuccess) {
+      p->nccl = nullptr;
+      return bail(ooo::set_error(OOO_ERR_NCCL, p->api->GetErrorString(r)));
+    }
+  }
   *out = p;
   return OOO_OK;
 }
 
 // One iteration enqueued on `cap` (being captured): see the header comment.
 static ooo_status enqueue_step(ooo_pipeline *p, const void *X, const void *dY, void *Y, int ff, cudaStream_t cap) {
+  const ooo_pipeline_desc *d = &p->d;
   const int G = (int)p->g.size();
-  const int n = p->d.n_stages;
+  const bool cm = p->nccl != nullptr;
+  const int nst = (int)p->st.size();
+  auto sidx = [&](int j) { return cm ? 0 : stage_of(d, j); };
   ooo_status st;
 #define PL_CU(x)                                                             \
   do {                                                                       \
     if ((x) != cudaSuccess) return ooo::set_error(OOO_ERR_CUDA, #x " failed"); \
   } while (0)
-#define PL_TRY(x)                  \
-  do {                             \
+#define PL_TRY(x)                        \
+  do {                                   \
     if ((st = (x)) != OOO_OK) return st; \
   } while (0)
+#define PL_NC(x)                                                                     \
+  do {                                                                               \
+    ncclResult_t _r = (x);                                                           \
+    if (_r != ncclSuccess) return ooo::set_error(OOO_ERR_NCCL, p->api->GetErrorString(_r)); \
+  } while (0)
   PL_CU(cudaEventRecord(p->ev_fork, cap));
-  for (int k = 0; k < n; ++k) PL_CU(cudaStreamWaitEvent(p->st[k], p->ev_fork, 0));
+  for (int k = 0; k < nst; ++k) PL_CU(cudaStreamWaitEvent(p->st[k], p->ev_fork, 0));
+  if (cm) PL_CU(cudaStreamWaitEvent(p->comm, p->ev_fork, 0));
+  // NCCL hand-off across the boundary between group a (sender) and group b
+  // (receiver); every rank issues the boundaries in the same global order
+  auto handoff = [&](int a, int b, const void *src, void *dst, size_t bytes, cudaEvent_t done) -> ooo_status {
+    const bool snd = owned(d, a), rcv = owned(d, b);
+    if (!snd && !rcv) return OOO_OK;
+    const size_t n = bytes / 2;
+    if (snd && rcv) PL_NC(p->api->GroupStart());
+    if (snd) PL_NC(p->api->Send(src, n, ncclBfloat16, stage_of(d, b) % d->world_size, p->nccl, p->comm));
+    if (rcv) PL_NC(p->api->Recv(dst, n, ncclBfloat16, stage_of(d, a) % d->world_size, p->nccl, p->comm));
+    if (snd && rcv) PL_NC(p->api->GroupEnd());
+    if (rcv) PL_CU(cudaEventRecord(done, p->comm));
+    return OOO_OK;
+  };
   // forward: group j after group j-1 (its output is group j's input)
   for (int j = 0; j < G; ++j) {
-    cudaStream_t s = p->st[stage_of(&p->d, j)];
-    if (j > 0) PL_CU(cudaStreamWaitEvent(s, p->ev_f[j - 1], 0));
-    PL_TRY(ooo_forward(p->stk[j], j == 0 ? X : p->out[j - 1], j == G - 1 ? Y : p->out[j], s));
-    PL_CU(cudaEventRecord(p->ev_f[j], s));
+    if (owned(d, j)) {
+      cudaStream_t s = p->st[sidx(j)];
+      if (j > 0) PL_CU(cudaStreamWaitEvent(s, xfer(d, j - 1) ? p->ev_xf[j] : p->ev_f[j - 1], 0));
+      PL_TRY(ooo_forward(p->stk[j], j == 0 ? X : p->in[j], j == G - 1 ? Y : p->out[j], s));
+      PL_CU(cudaEventRecord(p->ev_f[j], s));
+      if (j < G - 1 && xfer(d, j)) PL_CU(cudaStreamWaitEvent(p->comm, p->ev_f[j], 0));
+    }
+    if (j < G - 1 && xfer(d, j))
+      PL_TRY(handoff(j, j + 1, p->out[j], p->in[j + 1], act_bytes(d, d->dims[p->g[j].first + p->g[j].nl]),
+                     p->ev_xf[j + 1]));
   }
   // backward: group G-1 first; group j-1 on group j's input gradient.  A
-  // stage runs one group's kernel at a time (it is one GPU: its SM
-  // partition), so a group's backward also waits for the stage's previous one
-  std::vector<int> last(n, -1);
+  // stage runs one group's kernel at a time (it is one GPU: its SMs), so a
+  // group's backward also waits for the stage's previous one
+  std::vector<int> last(nst, -1);
   for (int j = G - 1; j >= 0; --j) {
-    const int k = stage_of(&p->d, j);
-    cudaStream_t s = p->st[k];
-    if (j < G - 1) PL_CU(cudaStreamWaitEvent(s, p->ev_b[j + 1], 0));
-    if (last[k] >= 0) PL_TRY(ooo_join(p->stk[last[k]], s));
-    last[k] = j;
-    ooo_schedule sch;
-    sch.kind = ff ? OOO_SCHED_FIRST_K : OOO_SCHED_IN_ORDER;
-    sch.k = ff ? p->g[j].nl : 0;   // fast-forwarding: every dW after the dO chain
-    PL_TRY(ooo_backward(p->stk[j], j == G - 1 ? dY : p->dx[j + 1], sch, j > 0 ? p->dx[j] : nullptr, s));
-    if (j > 0) {
-      if (ff) PL_TRY(ooo_input_grad_wait(p->stk[j], s));   // dX released mid-kernel
-      else PL_TRY(ooo_join(p->stk[j], s));                  // after the whole backward
-      PL_CU(cudaEventRecord(p->ev_b[j], s));
+    if (owned(d, j)) {
+      const int k = sidx(j);
+      cudaStream_t s = p->st[k];
+      if (j < G - 1) PL_CU(cudaStreamWaitEvent(s, xfer(d, j) ? p->ev_xb[j] : p->ev_b[j + 1], 0));
+      if (last[k] >= 0) PL_TRY(ooo_join(p->stk[last[k]], s));
+      last[k] = j;
+      ooo_schedule sch;
+      sch.kind = ff ? OOO_SCHED_FIRST_K : OOO_SCHED_IN_ORDER;
+      sch.k = ff ? p->g[j].nl : 0;   // fast-forwarding: every dW after the dO chain
+      PL_TRY(ooo_backward(p->stk[j], j == G - 1 ? dY : p->dyr[j], sch, j > 0 ? p->dxs[j] : nullptr, s));
+      if (j > 0) {
+        // dX released mid-kernel or after the whole backward
+        cudaStream_t w = xfer(d, j - 1) ? p->comm : s;
+        if (ff) PL_TRY(ooo_input_grad_wait(p->stk[j], w));
+        else PL_TRY(ooo_join(p->stk[j], w));
+        if (!xfer(d, j - 1)) PL_CU(cudaEventRecord(p->ev_b[j], s));
+      }
     }
+    if (j > 0 && xfer(d, j - 1))
+      PL_TRY(handoff(j, j - 1, p->dxs[j], p->dyr[j - 1], act_bytes(d, d->dims[p->g[j].first]), p->ev_xb[j - 1]));
   }
-  for (int j = 0; j < G; ++j) PL_TRY(ooo_join(p->stk[j], p->st[stage_of(&p->d, j)]));
-  for (int k = 0; k < n; ++k) {
+  for (int j = 0; j < G; ++j)
+    if (owned(d, j)) PL_TRY(ooo_join(p->stk[j], p->st[sidx(j)]));
+  for (int k = 0; k < nst; ++k) {
     PL_CU(cudaEventRecord(p->ev_join[k], p->st[k]));
     PL_CU(cudaStreamWaitEvent(cap, p->ev_join[k], 0));
   }
+  if (cm) {
+    PL_CU(cudaEventRecord(p->ev_cj, p->comm));
+    PL_CU(cudaStreamWaitEvent(cap, p->ev_cj, 0));
+  }
 #undef PL_CU
 #undef PL_TRY
+#undef PL_NC
   return OOO_OK;
 }
 

@@ -395,10 +395,14 @@ class OooStack:
 
 class Pipeline:
     """Cross-layer model parallelism (§5.2.1): ooo_pipeline_create over
-    caller-owned torch buffers.  placement 'contiguous' | 'modulo'; the
-    stages are SM partitions of the current GPU (include/ooo.h)."""
+    caller-owned torch buffers.  placement 'contiguous' | 'modulo'.  Without
+    unique_id the stages are SM partitions of the current GPU; with it every
+    rank is one stage (n_stages = world_size) and the hand-offs are NCCL
+    send / recv (world_size 1: loopback) -- include/ooo.h.  dW[i] / db[i] are
+    None for layers another rank owns."""
 
-    def __init__(self, dims, acts, tokens, W, b, group_layers, n_stages, placement="modulo"):
+    def __init__(self, dims, acts, tokens, W, b, group_layers, n_stages, placement="modulo", world_size=1,
+                 rank=0, unique_id: bytes | None = None):
         import torch
         lib = load()
         self.dims, self.acts, self.tokens = [int(x) for x in dims], list(acts), int(tokens)
@@ -415,6 +419,10 @@ class Pipeline:
         d.group_layers = self.group_layers
         d.n_stages = self.n_stages
         d.placement = {"contiguous": 0, "modulo": 1}[placement]
+        d.world_size, d.rank = int(world_size), int(rank)
+        if unique_id is not None:
+            keep["uid"] = ctypes.create_string_buffer(unique_id, _lib.UNIQUE_ID_BYTES)
+            d.nccl_unique_id = ctypes.cast(keep["uid"], c_void_p)
         ws, gb = c_size_t(), c_size_t()
         check(lib.ooo_pipeline_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)))
         dev = W[0].device
@@ -436,7 +444,10 @@ class Pipeline:
         self.dW, self.db = [], []
         for j in range(self.G):
             off = c_int64()
-            check(lib.ooo_pipeline_grads_offset(ctypes.byref(d), j, ctypes.byref(off)))
+            if lib.ooo_pipeline_grads_offset(ctypes.byref(d), j, ctypes.byref(off)) != 0:
+                self.dW += [None] * self.group_layers      # another rank's group
+                self.db += [None] * self.group_layers
+                continue
             lo = j * self.group_layers
             offs = grad_offsets(self.dims[lo: lo + self.group_layers + 1], self.acts[lo: lo + self.group_layers],
                                 self.tokens)

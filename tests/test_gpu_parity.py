@@ -686,3 +686,38 @@ def test_graph_host_buffer_steps():
         b["g"].close()
     stk.close()
     ref.close()
+
+
+def test_bf16_pipeline_nccl_loopback(monkeypatch):
+    """The multi-rank pipeline data plane on one GPU: a one-rank communicator
+    in loopback (every group boundary is an ncclSend / ncclRecv to itself on
+    the comm stream, dX sent after ooo_input_grad_wait mid-kernel or after the
+    whole backward) gives Y and gradients bit-identical to the SM-partition
+    pipeline, fast-forwarded and conventional."""
+    from paper_conf_eurosys_ohlks22_b200.stack import Pipeline, get_unique_id
+    monkeypatch.setenv("NCCL_ALGO", "Ring")
+    monkeypatch.setenv("NCCL_PROTO", "Simple")
+    h = 256
+    dims, acts = [h], []
+    for _ in range(4):
+        dims += [h, h, 4 * h, h]
+        acts += ["id", "id", "gelu", "id"]
+    case = Case(dims, acts, 264, "bf16")
+    Wt = [to_dev(w, "bf16") for w in case.W]
+    bt = [to_dev(v, "bf16") for v in case.b]
+    X, dY = to_dev(case.X, "bf16"), to_dev(case.dY, "bf16")
+    for ff in (True, False):
+        res = []
+        for mode in ("partition", "loopback"):
+            kw = dict(n_stages=2) if mode == "partition" else dict(n_stages=1, unique_id=get_unique_id())
+            pipe = Pipeline(dims, acts, case.M, Wt, bt, group_layers=4, placement="modulo", **kw)
+            Y = torch.empty(case.M, dims[-1], dtype=torch.bfloat16, device="cuda")
+            g = pipe.graph(X, dY, Y, fast_forward=ff)
+            for _ in range(2):
+                g.launch()
+            torch.cuda.synchronize()
+            res.append((Y.clone(), torch.cat([w.reshape(-1) for w in pipe.dW] + list(pipe.db))))
+            g.close()
+            pipe.close()
+        assert torch.equal(res[0][0], res[1][0]), ff
+        assert torch.equal(res[0][1], res[1][1]), ff

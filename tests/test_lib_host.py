@@ -144,6 +144,7 @@ def test_pipeline_host_validation(lib):
     d = _lib.PipelineDesc()
     keep = (stack._i32arr(dims), stack._i32arr([0] * 12))
     d.num_layers, d.tokens, d.group_layers, d.n_stages, d.placement = 12, 64, 3, 2, 1
+    d.world_size, d.rank = 1, 0
     d.dims = ctypes.cast(keep[0], ctypes.POINTER(ctypes.c_int32))
     d.acts = ctypes.cast(keep[1], ctypes.POINTER(ctypes.c_int32))
     ws, gb = ctypes.c_size_t(), ctypes.c_size_t()
@@ -161,4 +162,15 @@ def test_pipeline_host_validation(lib):
     d.group_layers, d.n_stages = 3, 5      # more stages than groups
     assert lib.ooo_pipeline_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)) == 1
     d.n_stages, d.placement = 3, 0         # contiguous: stages must divide the groups
+    assert lib.ooo_pipeline_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)) == 1
+    # with a communicator (sizes need no NCCL): rank 0 of 2, modulo -> it owns groups 0 and 2 only
+    uid = ctypes.create_string_buffer(128)
+    d.n_stages, d.placement, d.world_size, d.rank = 2, 1, 2, 0
+    d.nccl_unique_id = ctypes.cast(uid, ctypes.c_void_p)
+    assert lib.ooo_pipeline_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)) == 0
+    assert per_group * 2 <= gb.value < per_group * 3
+    o = ctypes.c_int64()
+    assert lib.ooo_pipeline_grads_offset(ctypes.byref(d), 2, ctypes.byref(o)) == 0
+    assert lib.ooo_pipeline_grads_offset(ctypes.byref(d), 1, ctypes.byref(o)) == 1   # rank 1's group
+    d.n_stages = 1                                  # one stage per rank required
     assert lib.ooo_pipeline_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)) == 1
