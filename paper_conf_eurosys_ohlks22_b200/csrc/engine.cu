@@ -154,7 +154,8 @@ template <int CG> struct Cfg {
   static constexpr int TASK_OFF = SLOT_OFF + 16;
   static constexpr int BIAS_OFF = (TASK_OFF + 4 * Q + 15) / 16 * 16;
   static constexpr int RED_OFF = BIAS_OFF + kMaxBN * 4;
-  static constexpr int SMEM = RED_OFF + 4 * kMaxBN * 4 + 1024;
+  static constexpr int SKF_OFF = RED_OFF + 4 * kMaxBN * 4;   // split-K "last arrival" flag
+  static constexpr int SMEM = SKF_OFF + 16 + 1024;
   static_assert(SMEM <= kSmemBudget, "engine smem budget");
   static_assert(STAGE % 1024 == 0, "stage alignment");
 };
@@ -259,6 +260,11 @@ __device__ __forceinline__ int ld_relaxed(const int32_t *p) {
   asm volatile("ld.relaxed.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ int atom_add_acq_rel(int32_t *p, int v) {
+  int old;
+  asm volatile("atom.acq_rel.gpu.global.add.s32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(v) : "memory");
+  return old;
+}
 __device__ __forceinline__ void red_release_add(int32_t *p, int v) {
   asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
@@ -294,17 +300,24 @@ __device__ __forceinline__ int op_of(const Params &p, int t) {
 
 struct TaskRt {
   int op, kind, layer, bn, nkb, m0, n0, M, N, mblk0;   // m0 / mblk0: first row (block) of the tile
+  int kb0, ks, s, tile;   // split-K: first k-block, splits, this task's split, tile index within the op
 };
 template <int CG>
 __device__ __forceinline__ TaskRt task_rt(const Params &p, int t) {
   TaskRt r;
   r.op = op_of(p, t);
   const Op &o = p.ops[r.op];
-  const int rel = t - o.first;
+  int rel = t - o.first;
   r.kind = o.kind;
   r.layer = o.layer;
   r.bn = o.bn;
-  r.nkb = o.nkb;
+  r.ks = o.ks > 1 ? o.ks : 1;
+  r.s = rel % r.ks;               // the splits of one tile are consecutive tasks
+  rel /= r.ks;
+  r.tile = rel;
+  const int kps = (o.nkb + r.ks - 1) / r.ks;
+  r.kb0 = r.s * kps;
+  r.nkb = min(o.nkb, r.kb0 + kps) - r.kb0;
   r.mblk0 = o.m_off + CG * (rel / o.nt);
   r.m0 = r.mblk0 * BM;
   r.n0 = (rel % o.nt) * o.bn;
@@ -409,7 +422,7 @@ __device__ __forceinline__ void load_b(const CUtensorMap *mB, uint32_t sb, uint3
 template <int CG, bool B_MN>
 __device__ __forceinline__ void prefetch_b(const CUtensorMap *mB, uint32_t sbase, uint32_t bar_empty,
                                            uint32_t bar_full, uint32_t L_full, bool leader, uint32_t bytes, int bn0,
-                                           int bh, int it, int npre, int nkb) {
+                                           int bh, int it, int npre, int nkb, int kb0) {
   using C = Cfg<CG>;
   int s = it % C::STAGES;
   uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;
@@ -419,7 +432,7 @@ __device__ __forceinline__ void prefetch_b(const CUtensorMap *mB, uint32_t sbase
     if (leader) mbar_expect_tx(bar_full + 8 * s, bytes * kc);
     for (int sub = 0; sub < kc; ++sub)
       load_b<CG, B_MN>(mB, sbase + s * C::STAGE + sub * C::SUB + A_BYTES, L_full + 8 * s, bn0, bh,
-                       (st * C::KPS + sub) * BK);
+                       (kb0 + st * C::KPS + sub) * BK);
     if (++s == C::STAGES) {
       s = 0;
       ph ^= 1u;
@@ -457,7 +470,7 @@ __device__ __forceinline__ void produce(const TaskRt &T, const CUtensorMap *mA, 
     const int kc = min(C::KPS, T.nkb - st * C::KPS);
     for (int sub = 0; sub < kc; ++sub) {
       ktrace(t, st * C::KPS + sub, 0);
-      load_a<CG, A_MN>(mA, sbase + s * C::STAGE + sub * C::SUB, L_full + 8 * s, am, (st * C::KPS + sub) * BK);
+      load_a<CG, A_MN>(mA, sbase + s * C::STAGE + sub * C::SUB, L_full + 8 * s, am, (T.kb0 + st * C::KPS + sub) * BK);
     }
     if (++s == C::STAGES) {
       s = 0;
@@ -473,8 +486,8 @@ __device__ __forceinline__ void produce(const TaskRt &T, const CUtensorMap *mA, 
       const int kb = st * C::KPS + sub;
       ktrace(t, kb, 0);
       const uint32_t sa = sbase + s * C::STAGE + sub * C::SUB;
-      load_a<CG, A_MN>(mA, sa, lb, am, kb * BK);
-      load_b<CG, B_MN>(mB, sa + A_BYTES, lb, bn0, bh, kb * BK);
+      load_a<CG, A_MN>(mA, sa, lb, am, (T.kb0 + kb) * BK);
+      load_b<CG, B_MN>(mB, sa + A_BYTES, lb, bn0, bh, (T.kb0 + kb) * BK);
     }
     if (++s == C::STAGES) {
       s = 0;
@@ -484,7 +497,10 @@ __device__ __forceinline__ void produce(const TaskRt &T, const CUtensorMap *mA, 
   it += nst;
 }
 
-template <int CG>
+// SK: the kernel contains the split-K epilogue path (launched only when the
+// queue has split ops -- skinny stacks), so the common path (C2, C3) carries
+// none of its registers.
+template <int CG, bool SK>
 __global__ void __launch_bounds__(kThreads, 1)
     engine_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constant__ CUtensorMap tmDX,
                   const __grid_constant__ Params p) {
@@ -504,6 +520,7 @@ __global__ void __launch_bounds__(kThreads, 1)
   volatile int *task_slot = reinterpret_cast<volatile int *>(smem + C::TASK_OFF);
   float *bias_s = reinterpret_cast<float *>(smem + C::BIAS_OFF);
   float *red = reinterpret_cast<float *>(smem + C::RED_OFF);
+  volatile int *sk_flag = reinterpret_cast<volatile int *>(smem + C::SKF_OFF);
   int32_t *ctr = p.ctr;
   const CounterLayout &cl = p.cl;
 
@@ -609,8 +626,8 @@ __global__ void __launch_bounds__(kThreads, 1)
             asm volatile("fence.proxy.async.global;" ::: "memory");
           }
           npre = min((T.nkb + C::KPS - 1) / C::KPS, C::STAGES);   // ring stages claimed for W
-          if (b_mn) prefetch_b<CG, true>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre, T.nkb);
-          else prefetch_b<CG, false>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre, T.nkb);
+          if (b_mn) prefetch_b<CG, true>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre, T.nkb, T.kb0);
+          else prefetch_b<CG, false>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre, T.nkb, T.kb0);
         }
         deps<true>(p, T, T.mblk0 + (int)rank);    // this CTA's row block (no-op after a ready claim)
         asm volatile("fence.proxy.async.global;" ::: "memory");   // TMA reads see the producers' data
@@ -620,7 +637,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           case 0: produce<CG, false, false>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, t, npre); break;
           default: produce<CG, true, true>(T, mA, mB, sbase, bar_empty, bar_full, L_full, leader, bytes, am, bn0, bh, it, t, npre); break;
         }
-        if (p.pf_dist > 0 && T.kind != EPI_WGRAD && T.m0 == 0) {
+        if (p.pf_dist > 0 && T.kind != EPI_WGRAD && T.m0 == 0 && T.s == 0) {
           // the weights pf_dist layers ahead on this chain (F: upwards, dO:
           // downwards), this tile's column slice -- issued after the tile's
           // own loads, so they never queue behind the prefetch
@@ -843,17 +860,80 @@ __global__ void __launch_bounds__(kThreads, 1)
       // publish below, from the accumulator still in TMEM (pass 2): the Z_i
       // store of an activated F_i, and the bias-gradient column sums of an
       // identity-activation dO_i (round(acc) again; act' = 1).
-      const bool late_z = T.kind == EPI_FWD && zout != nullptr && act == ACT_RELU && !(dbg & 1);
-      const bool late_db = T.kind == EPI_DGRAD && dbpart != nullptr && act == ACT_ID;
+      // split-K chain op (skinny stacks): every split stores its fp32 partial
+      // and arrives on the tile's counter (one per CTA); the last to arrive
+      // sums the partials in split order (deterministic) and runs the epilogue
+      const bool sk = SK && T.ks > 1;
+      const bool late_z = !sk && T.kind == EPI_FWD && zout != nullptr && act == ACT_RELU && !(dbg & 1);
+      const bool late_db = !sk && T.kind == EPI_DGRAD && dbpart != nullptr && act == ACT_ID;
+      // partial [s][row block][32-col chunk][8 float4 columns][128 rows] --
+      // float4 j of chunk c of this thread's row; a warp's 32 rows are 512
+      // contiguous bytes per float4 (coalesced stores and loads)
+      float4 *skrow = sk ? reinterpret_cast<float4 *>(p.skpart) + ((size_t)mblk * p.sk_nc + (T.n0 >> 5)) * 8 * 128 +
+                               (q * 32 + lane)
+                         : nullptr;
+      const size_t sk_split = (size_t)cl.MT * p.sk_nc * 8 * 128;   // float4 per split
+      if (sk) {
+        for (int c = h; c < cend; c += kEpiPerQ) {
+          uint32_t r2[32];
+          tmem_ld32_issue(tbase + (uint32_t)(c * 32), r2);
+          tmem_ld_wait(r2);
+          if (row_ok) {
+            float4 *dst = skrow + T.s * sk_split + (size_t)c * 8 * 128;
+#pragma unroll
+            for (int j = 0; j < 8; ++j)
+              __stcg(dst + j * 128, make_float4(__uint_as_float(r2[4 * j]), __uint_as_float(r2[4 * j + 1]),
+                                                __uint_as_float(r2[4 * j + 2]), __uint_as_float(r2[4 * j + 3])));
+          }
+        }
+        fence_before();                          // the accumulator is free again (TMEM no longer read)
+        __syncwarp();
+        if (lane == 0) {
+          if (leader) mbar_arrive(bar_tempty + 8 * acc);
+          else mbar_arrive_cluster(L_tempty + 8 * acc);
+        }
+        ebar();                                  // all partial stores of this CTA precede the arrival
+        if (et == 0) {
+          const int old = atom_add_acq_rel(ctr + cl.sk + o.sk_base + T.tile * CG + (int)rank, 1);
+          *sk_flag = old == T.ks - 1;
+        }
+        ebar();
+        if (!*sk_flag) continue;                 // another split finishes this tile
+      }
       uint32_t ra[32];
-      if (h < cend) tmem_ld32_issue(tbase + (uint32_t)(h * 32), ra);
+      if (!sk && h < cend) tmem_ld32_issue(tbase + (uint32_t)(h * 32), ra);
       for (int c = h; c < cend; c += kEpiPerQ) {
         const int col0 = T.n0 + c * 32;
-        tmem_ld_wait(ra);
         float v[32];
+        if (sk) {
 #pragma unroll
-        for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(ra[i]);
-        if (c + kEpiPerQ < cend) tmem_ld32_issue(tbase + (uint32_t)((c + kEpiPerQ) * 32), ra);
+          for (int i = 0; i < 32; ++i) v[i] = 0.f;
+          if (row_ok) {
+            // split order (deterministic whoever arrived last); all loads of a
+            // split issued before its adds, splits unrolled up to 8
+#pragma unroll
+            for (int s2 = 0; s2 < 8; ++s2) {
+              if (s2 < T.ks) {
+                const float4 *src = skrow + s2 * sk_split + (size_t)c * 8 * 128;
+                float4 f[8];
+#pragma unroll
+                for (int j = 0; j < 8; ++j) f[j] = __ldcg(src + j * 128);
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                  v[4 * j] += f[j].x;
+                  v[4 * j + 1] += f[j].y;
+                  v[4 * j + 2] += f[j].z;
+                  v[4 * j + 3] += f[j].w;
+                }
+              }
+            }
+          }
+        } else {
+          tmem_ld_wait(ra);
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(ra[i]);
+          if (c + kEpiPerQ < cend) tmem_ld32_issue(tbase + (uint32_t)((c + kEpiPerQ) * 32), ra);
+        }
         if (tr2 && c == h) etrace2(t, 1);
         if (T.kind == EPI_FWD) {
 #pragma unroll
@@ -946,12 +1026,15 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
         }
       }
-      // accumulator buffer free for task j+2 (the leader's barrier counts all CTAs)
-      fence_before();
-      __syncwarp();
-      if (lane == 0) {
-        if (leader) mbar_arrive(bar_tempty + 8 * acc);
-        else mbar_arrive_cluster(L_tempty + 8 * acc);
+      // accumulator buffer free for task j+2 (the leader's barrier counts all
+      // CTAs; a split-K task released it after storing its partial)
+      if (!sk) {
+        fence_before();
+        __syncwarp();
+        if (lane == 0) {
+          if (leader) mbar_arrive(bar_tempty + 8 * acc);
+          else mbar_arrive_cluster(L_tempty + 8 * acc);
+        }
       }
       if (T.kind == EPI_DGRAD && dbpart && mblk < cl.MT) {
         ebar();
@@ -1027,14 +1110,20 @@ cudaError_t engine_set_trace(void *p) {
 #endif
 
 cudaError_t engine_init() {
-  cudaError_t e = cudaFuncSetAttribute(engine_kernel<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<1>::SMEM);
+  cudaError_t e = cudaFuncSetAttribute(engine_kernel<1, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<1>::SMEM);
   if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(engine_kernel<2>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<2>::SMEM);
+    e = cudaFuncSetAttribute(engine_kernel<2, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<2>::SMEM);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(engine_kernel<1, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<1>::SMEM);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(engine_kernel<2, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg<2>::SMEM);
   return e;
 }
 
 cudaError_t launch_engine(int cg, const Params &p, const CUtensorMap *tmY, const CUtensorMap *tmDX, int ctas,
                           cudaStream_t stream, int priority) {
+  bool sk = false;
+  for (int j = 0; j < p.nops && !sk; ++j) sk = p.ops[j].ks > 1;
   cudaLaunchConfig_t cfg = {};
   cfg.blockDim = dim3(kThreads, 1, 1);
   cfg.stream = stream;
@@ -1055,13 +1144,15 @@ cudaError_t launch_engine(int cg, const Params &p, const CUtensorMap *tmY, const
     attr[2].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 3;
-    return cudaLaunchKernelEx(&cfg, engine_kernel<2>, *tmY, *tmDX, p);
+    return sk ? cudaLaunchKernelEx(&cfg, engine_kernel<2, true>, *tmY, *tmDX, p)
+              : cudaLaunchKernelEx(&cfg, engine_kernel<2, false>, *tmY, *tmDX, p);
   }
   cfg.gridDim = dim3(ctas, 1, 1);
   cfg.dynamicSmemBytes = Cfg<1>::SMEM;
   cfg.attrs = attr;
   cfg.numAttrs = 2;
-  return cudaLaunchKernelEx(&cfg, engine_kernel<1>, *tmY, *tmDX, p);
+  return sk ? cudaLaunchKernelEx(&cfg, engine_kernel<1, true>, *tmY, *tmDX, p)
+            : cudaLaunchKernelEx(&cfg, engine_kernel<1, false>, *tmY, *tmDX, p);
 }
 
 }  // namespace eng

@@ -44,7 +44,9 @@ struct Op {
   int16_t nkb;      // K / 64 (0 for EPI_COPY)
   int16_t mapA, mapB, mapX, mapZ;   // indices into the map table (or MAP_*)
   int16_t m_off;    // first row block of the group
-  int16_t pad[2];
+  int16_t ks;       // > 1: split-K chain op -- every tile is ks tasks over consecutive k-block ranges
+                    // whose fp32 partials the last-arriving task sums in split order (skinny stacks)
+  int16_t sk_base;  // its first arrival counter (sk region: one per tile and CTA of the pair)
 };
 static_assert(sizeof(Op) == 32, "Op layout");
 
@@ -69,11 +71,12 @@ static_assert(sizeof(LayerDev) == 128, "LayerDev layout");
 // Counter layout (int32, one region in the workspace; indices are absolute):
 //   [0] dispenser | [1] unused | fwd_rows[L][MT]: tiles done of row block m of X_{i+1} |
 //   xcopy[MT]: X_1 rows copied | dz_rows[L][MT] | dz_total[L] | dw_done[L] |
-//   bucket_done[nb] | ar_done[nb] | dx_total: tiles of dO_1's output (dX) published
+//   bucket_done[nb] | ar_done[nb] | dx_total: tiles of dO_1's output (dX) published |
+//   sk[nsk]: split-K arrivals (inside the forward-reset range [0, fwd_end))
 // A forward-only launch resets [0, fwd_end); a backward resets [0, total).
 struct CounterLayout {
   int L, MT, nb;
-  int fwd_rows, xcopy, fwd_end;
+  int fwd_rows, xcopy, sk, fwd_end;
   int dz_rows, dz_total, dw_done, bucket_done, ar_done, dx_total, total;
 };
 
@@ -93,6 +96,8 @@ struct Params {
                            // weights of layer i + pf_dist (i - pf_dist) -- skinny stacks, where every
                            // chain op streams its W from HBM (W does not depend on the chain)
   int32_t maps_per_layer;  // map-table slots per layer (the map of layer j = the op's map + (j-i) x this)
+  int32_t sk_nc;           // 32-column chunks per row of the split-K partial buffer (max width / 32)
+  float *skpart;           // split-K partials [ks][MT][sk_nc][128 rows][32] fp32 (workspace)
   const CUtensorMap *maps;
   int32_t *ctr;            // counter array base
   const LayerDev *layers;  // index i-1

@@ -82,6 +82,8 @@ struct LayerPlan {
   int bucket = 0;
   GemmPlan fwd, dx, dw;
   int ebn_fwd = 0, ebn_dx = 0, ebn_dw = 0;   // engine tile widths
+  int ks_fwd = 1, ks_dx = 1;                 // split-K factors of the chain ops (skinny stacks)
+  int sk_fwd = 0, sk_dx = 0;                 // their first split-K arrival counter (CounterLayout::sk)
 };
 
 // Map-table slots per layer (engine): operand loads and output stores.
@@ -100,6 +102,8 @@ struct Plan {
   bool engine = false;
   int cg = 2;                      // engine CTAs per tile (2 = CTA pairs, cta_group::2)
   size_t off_maps = 0, off_layers = 0, off_ctr = 0;
+  size_t off_skpart = 0;           // split-K partials (0 bytes when no op splits)
+  int sk_nc = 0;                   // 32-column chunks per partial row
   ooo::eng::CounterLayout cl{};
 };
 
@@ -254,6 +258,35 @@ Plan make_plan(const ooo_stack_desc *d) {
       lp.ebn_dx = engine_bn(lp.din, true, p.cg, PT, workers, lp.dout);
       lp.ebn_dw = engine_bn(lp.dout, false, p.cg, PT, workers);
     }
+    // split-K chain ops when all tokens fit one 128-row tile (C5: 16 tokens):
+    // a chain op's latency is its k-blocks at the MMA issue rate, whatever its
+    // width (profiles/r02_mainloop_issue.md), so its K is spread over up to 8
+    // workers while the split tiles still fit them (>= 4 k-blocks each: C5
+    // 1.434 -> 1.363 ms with 4 splits, 1.614 with 8 splits of 2); the
+    // fp32 partials of so few rows cost little.  With more rows the partial
+    // traffic outweighs the k-blocks saved (C4, 512 tokens: 2.90 -> 3.70 ms
+    // with 4 splits, profiles/r02_splitk.md).  Not for ReLU F_i (their Z_i
+    // store is a pass over the TMEM accumulator, which a split task no longer
+    // holds).  OOO_SPLITK=0: off; OOO_SPLITK_MAX / OOO_SPLITK_MINKB: tuning.
+    int nsk = 0, maxw = 0;
+    for (int i = 0; i <= p.L; ++i) maxw = std::max(maxw, d->dims[i]);
+    auto ksplit = [&](int N, int bn, int K, bool allowed) {
+      if (!allowed || p.M > 128 || env_int("OOO_SPLITK", 1) == 0) return 1;
+      const int tiles = PT * ((N + bn - 1) / bn);
+      const int minkb = std::max(1, env_int("OOO_SPLITK_MINKB", 4));
+      const int ks = std::min({std::min(8, env_int("OOO_SPLITK_MAX", 8)), ((K + 63) / 64) / minkb, workers / tiles});
+      return ks >= 2 ? ks : 1;
+    };
+    for (int i = 1; i <= p.L; ++i) {
+      LayerPlan &lp = p.layer[i - 1];
+      lp.ks_fwd = ksplit(lp.dout, lp.ebn_fwd, lp.din, lp.act != OOO_ACT_RELU);
+      lp.ks_dx = ksplit(lp.din, lp.ebn_dx, lp.dout, true);
+      lp.sk_fwd = nsk;
+      if (lp.ks_fwd > 1) nsk += PT * ((lp.dout + lp.ebn_fwd - 1) / lp.ebn_fwd) * p.cg;
+      lp.sk_dx = nsk;
+      if (lp.ks_dx > 1) nsk += PT * ((lp.din + lp.ebn_dx - 1) / lp.ebn_dx) * p.cg;
+    }
+    p.sk_nc = maxw / 32;
     p.off_maps = take((size_t)p.L * MS_COUNT * sizeof(CUtensorMap));
     p.off_layers = take((size_t)p.L * sizeof(ooo::eng::LayerDev));
     ooo::eng::CounterLayout &cl = p.cl;
@@ -262,7 +295,8 @@ Plan make_plan(const ooo_stack_desc *d) {
     cl.nb = p.nbuckets;
     cl.fwd_rows = 2;
     cl.xcopy = cl.fwd_rows + p.L * cl.MT;
-    cl.fwd_end = cl.xcopy + cl.MT;
+    cl.sk = cl.xcopy + cl.MT;
+    cl.fwd_end = cl.sk + nsk;
     cl.dz_rows = (int)align_up(cl.fwd_end, 32);
     cl.dz_total = cl.dz_rows + p.L * cl.MT;
     cl.dw_done = cl.dz_total + p.L;
@@ -271,6 +305,7 @@ Plan make_plan(const ooo_stack_desc *d) {
     cl.dx_total = cl.ar_done + p.nbuckets;
     cl.total = cl.dx_total + 1;
     p.off_ctr = take((size_t)cl.total * 4);
+    if (nsk > 0) p.off_skpart = take((size_t)8 * cl.MT * p.sk_nc * 128 * 32 * 4);   // up to 8 splits
   }
   p.workspace_bytes = std::max<size_t>(off, 256);
   p.grad_elems = goff;
@@ -712,12 +747,14 @@ pl::Unit unit_of(const ooo_stack *s, int kind, int i) {
     u.mt = PT;
     u.nt = (lp.dout + u.bn - 1) / u.bn;
     u.nkb = (lp.din + 63) / 64;
+    u.ks = lp.ks_fwd;
   } else if (kind == pl::DGRAD) {
     u.act = i >= 2 ? p.layer[i - 2].act : OOO_ACT_IDENTITY;
     u.bn = lp.ebn_dx;
     u.mt = PT;
     u.nt = (lp.din + u.bn - 1) / u.bn;
     u.nkb = (lp.dout + 63) / 64;
+    u.ks = lp.ks_dx;
   } else {
     u.act = OOO_ACT_IDENTITY;
     u.bn = lp.ebn_dw;
@@ -725,6 +762,8 @@ pl::Unit unit_of(const ooo_stack *s, int kind, int i) {
     u.nt = (lp.dout + u.bn - 1) / u.bn;
     u.nkb = (p.M + 63) / 64;
   }
+  u.nkb_full = u.nkb;
+  if (u.ks > 1) u.nkb = (u.nkb + u.ks - 1) / u.ks;   // the planner's per-task k-blocks
   return u;
 }
 
@@ -739,7 +778,12 @@ ooo::eng::Op op_of_unit(const ooo_stack *s, const pl::Unit &u) {
   o.m_off = (int16_t)(p.cg * u.m_off);   // 128-row blocks
   o.mt = (int16_t)u.mt;
   o.nt = (int16_t)u.nt;
-  o.nkb = (int16_t)u.nkb;
+  o.nkb = (int16_t)u.nkb_full;
+  o.ks = (int16_t)std::max(1, u.ks);
+  if (u.ks > 1) {   // arrival counters of this unit's tiles: after the op's earlier rows
+    const LayerPlan &lp = p.layer[i - 1];
+    o.sk_base = (int16_t)((u.kind == pl::FWD ? lp.sk_fwd : lp.sk_dx) + u.m_off * u.nt * p.cg);
+  }
   o.mapA = o.mapB = o.mapX = o.mapZ = ooo::eng::MAP_NONE;
   if (u.kind == pl::FWD) {
     o.mapA = (int16_t)map_index(i, MS_FWD_A);
@@ -806,6 +850,8 @@ ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const 
   // L2 (OOO_PF_DIST overrides; 0 = off)
   P.pf_dist = env_int("OOO_PF_DIST", pb.rows <= 2 ? 4 : 0);
   P.maps_per_layer = MS_COUNT;
+  P.sk_nc = p.sk_nc;
+  P.skpart = p.off_skpart ? reinterpret_cast<float *>(s->ws + p.off_skpart) : nullptr;
   P.maps = s->dmaps;
   P.ctr = s->ctr;
   P.layers = s->dlayers;
@@ -817,7 +863,7 @@ ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const 
   for (size_t j = 0; j < order.size(); ++j) {
     P.ops[j] = op_of_unit(s, order[j]);
     P.ops[j].first = first;
-    first += order[j].mt * order[j].nt;
+    first += order[j].mt * order[j].nt * std::max(1, order[j].ks);
   }
   P.nops = (int)order.size();
   P.ntasks = first;
@@ -1927,7 +1973,7 @@ extern "C" int32_t ooo_debug_last_queue(ooo_stack *s, int32_t *out, int32_t cap)
       out[5 * n + 1] = o.layer;
       out[5 * n + 2] = o.m_off;
       out[5 * n + 3] = o.mt;
-      out[5 * n + 4] = o.nt;
+      out[5 * n + 4] = o.nt * (o.ks > 1 ? o.ks : 1);   // tasks per tile row (split-K: ks per tile)
     }
     ++n;
   }

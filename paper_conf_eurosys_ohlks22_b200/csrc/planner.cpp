@@ -24,7 +24,7 @@ class Sim {
     auto init = [&](const Unit &u, int rows) {
       OpState &o = op(u.kind, u.layer);
       if (o.total == 0) {
-        o.total = rows * u.nt;
+        o.total = rows * u.nt * std::max(1, u.ks);
         o.row_cnt.assign(rows, 0);
         o.row_done.assign(rows, 0.0);
       }
@@ -117,7 +117,7 @@ class Sim {
     std::vector<double> f = disp_;
     if (d) {
       const double tkb = m_.t_kb * (0.5 + 0.5 * d->bn / 256.0);
-      for (int j = 0; j < d->mt * d->nt; ++j) {
+      for (int j = 0; j < d->mt * d->nt * std::max(1, d->ks); ++j) {
         auto it = std::min_element(f.begin(), f.end());
         const double start = std::max(*it, rd);
         *it = std::max(start, start + m_.t_fix + d->nkb * tkb - m_.stages * tkb);
@@ -150,7 +150,7 @@ class Sim {
     const double epi = epi_time(u);
     for (int r = u.m_off; r < u.m_off + u.mt; ++r) {
       const double dep = timing_ ? ready(u, r) : 0.0;
-      for (int n = 0; n < u.nt; ++n) {
+      for (int n = 0; n < u.nt * std::max(1, u.ks); ++n) {   // split-K: ks tasks per tile
         double done = 0.0;
         if (timing_) {
           const int w = (int)(std::min_element(disp_.begin(), disp_.end()) - disp_.begin());

@@ -29,6 +29,8 @@ struct Unit {
   int nkb;           // k-blocks per tile (0 for COPY)
   int bn;            // tile width
   int act;           // epilogue activation (0 = identity)
+  int ks = 1;        // split-K chain op: every tile is ks tasks of nkb = ceil(nkb_full / ks) k-blocks
+  int nkb_full = 0;  // the op's whole reduction (split-K)
   int release = -1;  // deferred units: emitted only once critical op #release (index into
                      // Problem::crit) has started (region schedule, §4.1); -1 = no constraint,
                      // >= crit.size() = after the whole chain

@@ -50,7 +50,7 @@ def report(name, ops, buf):
     cta = (raw >> np.uint64(48)).astype(np.int64)
     t = (raw & np.uint64((1 << 48) - 1)).astype(np.float64)
     valid = t[:, 3] > 0
-    t0 = t[valid, 0].min()
+    t0 = t[t[:, 0] > 0, 0].min()
     t = (t - t0) / 1e3
     # SM clock: cycles between "ready" and "acc ready" over the same interval in ns
     dc = clk[valid, 2] - clk[valid, 1]
@@ -63,10 +63,12 @@ def report(name, ops, buf):
         s = slice(first, first + n)
         first += n
         tt = t[s]
+        dn = raw[s, 3] > 0                       # split-K: only the last split of a tile publishes
+        td = tt[dn] if dn.any() else tt
         print(f"{kind} L{layer:3d} tiles {n:4d} disp {tt[:,0].min():8.1f} ready {tt[:,1].min():8.1f}"
-              f"..{tt[:,1].max():8.1f} done {tt[:,3].min():8.1f}..{tt[:,3].max():8.1f}"
+              f"..{tt[:,1].max():8.1f} done {td[:,3].min():8.1f}..{td[:,3].max():8.1f}"
               f" wait {np.mean(tt[:,1]-tt[:,0]):6.1f} main {np.mean(tt[:,2]-tt[:,1]):6.1f}"
-              f" epi {np.mean(tt[:,3]-tt[:,2]):5.1f} ctas {len(set(cta[s, 3]))}")
+              f" epi {np.mean(td[:,3]-td[:,2]):5.1f} published {int(dn.sum())} ctas {len(set(cta[s, 3]))}")
         g = allb[2 * 200000 * 8:].reshape(-1, 8)[s]
         if g[:, 7].max() > 0:
             m48 = np.uint64((1 << 48) - 1)
