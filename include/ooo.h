@@ -169,6 +169,10 @@ typedef struct {
                                   and stays bit-exact -- and the channel can switch buckets between
                                   chunks (the partitioning of [28, 38] behind P:180); <= 0 = one
                                   all-reduce per bucket */
+  int32_t average_over;        /* > 0: the gradients are scaled by 1 / average_over before the sum
+                                  all-reduce (pack/scale step, reading Q9) instead of 1 / world_size --
+                                  e.g. to average over a global batch of several local steps; 0 =
+                                  world_size (the data-parallel mean) */
   int32_t engine_ctas;         /* > 0: at most this many CTAs (SMs) for the bf16 engine kernels of this
                                   stack (one SM partition per pipeline stage, ooo_pipeline_*); <= 0 = all
                                   SMs (minus the NCCL reserve of a communicating stack) */

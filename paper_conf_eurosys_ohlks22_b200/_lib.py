@@ -46,6 +46,7 @@ class StackDesc(ctypes.Structure):
         ("comm_priority", c_int32),
         ("comm_model_gbps", c_int32),
         ("comm_chunk_bytes", c_int64),
+        ("average_over", c_int32),
         ("engine_ctas", c_int32),
     ]
 

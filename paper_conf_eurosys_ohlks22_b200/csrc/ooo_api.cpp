@@ -511,6 +511,11 @@ ooo_status end_rec(TimedRec *r, cudaStream_t st, int grid, double flops, double 
   return OOO_OK;
 }
 
+// Pack/scale factor of the gradients (reading Q9: 1/N before the sum all-reduce).
+float grad_alpha(const ooo_stack *s) {
+  return 1.0f / (float)(s->d.average_over > 0 ? s->d.average_over : s->d.world_size);
+}
+
 // ---- op launchers ------------------------------------------------------
 ooo_status launch_fwd(ooo_stack *s, int i, void *Y, cudaStream_t st, int prio) {
   const LayerPlan &lp = s->p.layer[i - 1];
@@ -562,7 +567,7 @@ ooo_status launch_dx(ooo_stack *s, int i, void *dX, cudaStream_t st, int prio) {
 ooo_status launch_dw_pack(ooo_stack *s, int i, cudaStream_t st, int prio, int sid) {
   const LayerPlan &lp = s->p.layer[i - 1];
   LayerRt &r = s->lr[i - 1];
-  const float alpha = 1.0f / (float)s->d.world_size;
+  const float alpha = grad_alpha(s);
   EpiArgs a = {};
   a.M = lp.din; a.N = lp.dout; a.K = s->p.M;
   a.kb_per_split = lp.dw.kb_per_split; a.splits = lp.dw.splits;
@@ -838,7 +843,7 @@ ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const 
   ooo::eng::Params P = {};
   P.M = p.M;
   P.R = p.R;
-  P.alpha = 1.0f / (float)s->d.world_size;
+  P.alpha = grad_alpha(s);
   P.in_order = in_order ? 1 : 0;
   P.fwd_gate = fwd_gate;
   P.dbg = env_int("OOO_DBG", 0);

@@ -23,7 +23,7 @@ def _i32arr(vals):
 
 def _desc(dims, acts, tokens, dtype, need_input_grad=False, bucket_layers=1, max_temp_bytes=0,
           world_size=1, rank=0, comm_enabled=True, nccl_max_ctas=0, wait_timeout_ms=0, comm_priority=0,
-          comm_chunk_bytes=0, comm_model_gbps=0, engine_ctas=0):
+          comm_chunk_bytes=0, comm_model_gbps=0, engine_ctas=0, average_over=0):
     keep = {}
     d = _lib.StackDesc()
     d.num_layers = len(acts)
@@ -45,6 +45,7 @@ def _desc(dims, acts, tokens, dtype, need_input_grad=False, bucket_layers=1, max
     d.comm_chunk_bytes = int(comm_chunk_bytes)
     d.comm_model_gbps = int(comm_model_gbps)
     d.engine_ctas = int(engine_ctas)
+    d.average_over = int(average_over)
     return d, keep
 
 
@@ -222,7 +223,7 @@ class OooStack:
     def __init__(self, dims, acts, tokens, W, b, dtype="bf16", need_input_grad=False, bucket_layers=1,
                  max_temp_bytes=0, world_size=1, rank=0, unique_id: bytes | None = None,
                  comm_enabled=True, nccl_max_ctas=0, wait_timeout_ms=0, comm_priority=0, comm_chunk_bytes=0,
-                 comm_model_gbps=0, engine_ctas=0):
+                 comm_model_gbps=0, engine_ctas=0, average_over=0):
         """unique_id: the NCCL bootstrap id (broadcast_unique_id); required
         for world_size > 1; with world_size == 1 it makes a one-rank
         communicator that runs the N > 1 data plane on one GPU."""
@@ -250,7 +251,7 @@ class OooStack:
         self.device = W[0].device
         d, keep = _desc(self.dims, self.acts, self.tokens, dtype, need_input_grad, bucket_layers,
                         max_temp_bytes, world_size, rank, comm_enabled, nccl_max_ctas, wait_timeout_ms,
-                        comm_priority, comm_chunk_bytes, comm_model_gbps, engine_ctas)
+                        comm_priority, comm_chunk_bytes, comm_model_gbps, engine_ctas, average_over)
         ws, gb = c_size_t(), c_size_t()
         check(lib.ooo_query_sizes(ctypes.byref(d), ctypes.byref(ws), ctypes.byref(gb)))
         self.workspace = torch.empty(ws.value, dtype=torch.uint8, device=self.device)

@@ -721,3 +721,28 @@ def test_bf16_pipeline_nccl_loopback(monkeypatch):
             pipe.close()
         assert torch.equal(res[0][0], res[1][0]), ff
         assert torch.equal(res[0][1], res[1][1]), ff
+
+
+@pytest.mark.parametrize("dtype,n", [("bf16", 4), ("bf16", 8), ("fp32", 2)])
+def test_pack_scale_average_over(dtype, n):
+    """The pack/scale step (reading Q9) with a divisor != 1 on
+    the GPU: average_over = n scales every dW_i / db_i by 1/n before the
+    all-reduce; a power of two, so the result is the unscaled gradient / n
+    exactly (bf16 and fp32), for the engine (bf16) and the per-layer path
+    (fp32), and the oracle's N-rank mean of n identical shards."""
+    case = Case([256, 512, 256, 128], ["gelu", "id", "id"], 264 if dtype == "bf16" else 64, dtype)
+    plain = case.stack()
+    scaled = case.stack(average_over=n)
+    a = case.run(plain, "first_k", 1)
+    b = case.run(scaled, "first_k", 1, graph=dtype == "bf16")
+    for x, y in zip(a["dW"] + a["db"], b["dW"] + b["db"]):
+        assert np.array_equal(x / n, y)
+    from oracle import layers as O
+    from oracle import schedule as S
+    ref = O.dp_step([case.X] * n, [case.dY] * n, case.W, case.b, case.acts, S.reverse_first_k(case.L, 1),
+                    "bf16" if dtype == "bf16" else "fp64")
+    # the oracle's mean over n identical shards is the local gradient; ours is it / n
+    _check({"dW": max(rel_fro(g * n, r) for g, r in zip(b["dW"], ref.gW)),
+            "db": max(rel_fro(g * n, r) for g, r in zip(b["db"], ref.gb))}, BF16_TOL if dtype == "bf16" else FP32_TOL)
+    plain.close()
+    scaled.close()
