@@ -106,17 +106,6 @@ constexpr int kThreads = 64 + kEpiThreads;
 constexpr int kMaxBN = 256;
 constexpr int STG_BYTES = kEpiWarps * 2048;
 constexpr int Q = 4;                                 // task ring depth
-#ifndef OOO_EARLY_WAIT
-#define OOO_EARLY_WAIT 0   // experiment: wait for k-block kb + 1 between kb's 2nd and 3rd MMA
-#endif
-#ifndef OOO_TMA_STORE
-#define OOO_TMA_STORE 0
-#endif
-// 1: the row-local chain outputs of identity-activation F_i and of dO_i leave
-// through per-warp TMA bulk stores (64B-swizzled 32 x 32 boxes) instead of
-// the smem transpose + st.global path; the early publish waits for their
-// completion (cp.async.bulk.wait_group 0) before the release.
-constexpr bool kTmaStore = OOO_TMA_STORE != 0;
 constexpr uint32_t TMEM_COLS = 512;
 // Bound of every wait (ns), from Params::timeout_ns (the stack's
 // wait_timeout_ms): a wait that exceeds it traps (the launch fails with an
@@ -693,37 +682,6 @@ __global__ void __launch_bounds__(kThreads, 1)
         const uint64_t astep = a_mn ? 128u : 2u, bstep = b_mn ? 128u : 2u;
         int s = it % C::STAGES;
         uint32_t ph = (uint32_t)(it / C::STAGES) & 1u;
-#if OOO_EARLY_WAIT
-        if (CG == 2 && C::KPS == 1) {
-          // the barrier wait (+ fence) of k-block kb + 1 runs while kb's last
-          // two MMAs execute, so the issuer's per-k-block overhead is covered
-          // by queued tensor work; kb's stage is released right after
-          mbar_wait_b(bar_full + 8 * s, ph);
-          fence_after();
-          for (int kb = 0; kb < T.nkb; ++kb) {
-            const uint64_t soff = (uint64_t)(s * (C::STAGE >> 4));
-            const uint64_t ad = a0 + soff, bd = b0 + soff;
-            umma_bf16_pair(dtm, ad, bd, ID, kb != 0 ? 1u : 0u);
-            umma_bf16_pair(dtm, ad + astep, bd + bstep, ID, 1u);
-            const int s_cur = s;
-            if (++s == C::STAGES) {
-              s = 0;
-              ph ^= 1u;
-            }
-            if (kb + 1 < T.nkb) {
-              mbar_wait_b(bar_full + 8 * s, ph);
-              fence_after();
-            }
-            umma_bf16_pair(dtm, ad + 2 * astep, bd + 2 * bstep, ID, 1u);
-            umma_bf16_pair(dtm, ad + 3 * astep, bd + 3 * bstep, ID, 1u);
-            umma_commit_pair(bar_empty + 8 * s_cur);
-          }
-          it += T.nkb;
-          umma_commit_pair(bar_tfull + 8 * acc);
-          etrace_gt(t, 5);
-          continue;
-        }
-#endif
         const int nst = (T.nkb + C::KPS - 1) / C::KPS;
         for (int st = 0; st < nst; ++st) {
           const int kb0 = st * C::KPS;
@@ -805,7 +763,6 @@ __global__ void __launch_bounds__(kThreads, 1)
         continue;
       }
       const Op &o = p.ops[T.op];
-      const CUtensorMap *mX = kTmaStore ? map_of(o.mapX, p.maps, &tmY, &tmDX) : nullptr;
       const LayerDev &Ld = p.layers[T.layer - 1];
       const int acc = ja & 1;
       const int jacc = ja++;
@@ -941,8 +898,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           uint32_t u[16];
           pack32(v, u);                                         // Z_i in bf16 (RNE)
           if (act == ACT_ID || (dbg & 1)) {
-            if (kTmaStore) stage_store32_packed(mX, stg, lane, u, col0, row0);
-            else if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);   // X_{i+1} = Z_i (or Y)
+            if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);   // X_{i+1} = Z_i (or Y)
           } else if (act == ACT_GELU) {
             // X_{i+1} = gelu(Z_i) and, for the next backward, gelu'(Z_i) in
             // the Z_i store (one Phi / e^{-z^2/2} evaluation for both; the
@@ -971,8 +927,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           pack32(v, u);                                         // dZ_{i-1} in bf16 (RNE)
 #pragma unroll
           for (int j = 0; j < 16; ++j) u[j] = row_ok ? u[j] : 0u;
-          if (kTmaStore) stage_store32_packed(mX, stg, lane, u, col0, row0);
-          else if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);  // dZ_{i-1} (or dX)
+          if (!(dbg & 2)) store32_rows_packed(out, T.N, stg, lane, u, col0, row0, T.M);  // dZ_{i-1} (or dX)
           if (dbpart && !late_db) {
             unpack32(u, v);
             red[q * kMaxBN + c * 32 + lane] = warp_colsum32(v, lane);
@@ -989,12 +944,7 @@ __global__ void __launch_bounds__(kThreads, 1)
       // release reductions are cumulative, so every store of the pass above
       // (all epilogue warps, ordered by the barrier) is visible before the count
       if (T.kind != EPI_WGRAD) {
-        if (kTmaStore) {
-          if (lane == 0) tma_store_wait_all();   // this warp's bulk stores are complete
-          __syncwarp();
-        }
         ebar();
-        if (kTmaStore && et == 0) asm volatile("fence.proxy.async.global;" ::: "memory");
         if (et == 0 && mrow0 < T.M) {
           if (T.kind == EPI_FWD) red_release_add(ctr + cl.fwd_rows + (T.layer - 1) * cl.MT + mblk, 1);
           else if (T.layer >= 2) red_release_add(ctr + cl.dz_rows + (T.layer - 2) * cl.MT + mblk, 1);

@@ -128,21 +128,6 @@ int engine_bn(int N, bool chain, int cg, int row_tiles, int workers, int K = 0) 
   // twice the pairs on each F_i / dO_i while they still fit the workers
   // (C4: 3.62 -> 3.14 ms; on C2's 16 rows the same change costs 25 %)
   if (chain && cg == 2 && N % 128 == 0 && row_tiles * (N / 128) <= workers) return 128;
-  const int narrow = env_int("OOO_EBN_NARROW", 0);   // experiment: 192-wide tiles for N <= this
-  if (narrow && cg == 1 && N <= narrow && N % 192 == 0) return 192;
-  // experiment (off: OOO_CHAIN192=1 turns it on): CTA-pair chain tiles 192
-  // wide when that still fits one wave and the cost model (waves x (first
-  // load + k-blocks at the MMA issue rate + an epilogue proportional to the
-  // width)) prefers it.  Measured on C2: first-k neutral (2.285 vs 2.283 ms),
-  // in-order +5 % (3.46 vs 3.28); C3 unaffected (1024 % 192 != 0)
-  if (chain && cg == 2 && K > 0 && N % 256 == 0 && N % 192 == 0 && env_int("OOO_CHAIN192", 0)) {
-    auto cost = [&](int bn) {
-      const int tiles = row_tiles * ((N + bn - 1) / bn);
-      const int waves = (tiles + workers - 1) / workers;
-      return waves * (1.0 + ((K + 63) / 64) * 0.45 + 2.8 * bn / 256.0);
-    };
-    if (cost(192) < cost(256) * 0.98) return 192;
-  }
   // CTA pairs split B in halves of >= 64 columns: bn in {128, 256}
   return N % 256 == 0 ? 256 : 128;
 }
@@ -425,6 +410,8 @@ struct ooo_stack {
   bool comm_stack = false;                    // a NCCL communicator (N > 1, or the one-rank mode)
   int timeout_ms = 4000;                      // engine wait bound (desc.wait_timeout_ms)
   bool test_comm_gate = false;                // OOO_TEST_COMM_GATE=1 (N = 1 only): see comm_active
+  int test_drop_flag = -1;                    // OOO_TEST_DROP_AR_FLAG=b: bucket b's flag is never written
+                                              // (tests that the engine's wait bound traps instead of hanging)
   // emulated all-reduce (N = 1 only; OOO_EMULATE_AR_N = n >= 2): each bucket's
   // S[dW] holds the comm stream for the ring time 2(n-1)/n x bytes / BW + lat
   int emu_n = 0;
@@ -949,7 +936,7 @@ ooo_status engine_comm(ooo_stack *s) {
       waited[b] = 1;
     }
     OOO_TRY(launch_allreduce(s, b, oc[j]));
-    if (--todo[b] == 0) {
+    if (--todo[b] == 0 && b != s->test_drop_flag) {
       CUresult r = write_fn(s->comm, reinterpret_cast<CUdeviceptr>(s->ctr + p.cl.ar_done + b), 1, 0);
       if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWriteValue32 failed (%d)", (int)r);
     }
@@ -1455,6 +1442,7 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
   s->comm_stack = d->world_size > 1 || d->nccl_unique_id != nullptr;
   s->timeout_ms = d->wait_timeout_ms > 0 ? d->wait_timeout_ms : (s->comm_stack ? 120000 : 4000);
   s->test_comm_gate = d->world_size == 1 && s->p.engine && env_int("OOO_TEST_COMM_GATE", 0) != 0;
+  if (s->test_comm_gate) s->test_drop_flag = env_int("OOO_TEST_DROP_AR_FLAG", -1);
   s->ws = static_cast<uint8_t *>(d->workspace);
   s->grads = static_cast<uint8_t *>(d->grads);
   const Plan &p = s->p;

@@ -318,9 +318,6 @@ __device__ __forceinline__ void stage_store(const CUtensorMap *map, uint32_t buf
   __syncwarp();
   if (lane == 0) tma_store_2d(map, buf, col0, row0);
 }
-#ifndef OOO_STG_DIRECT
-#define OOO_STG_DIRECT 0   // experiment: per-lane row stores from registers (no smem transpose)
-#endif
 #ifndef OOO_STG256
 #define OOO_STG256 1   // 32-B global stores (STG.256), 2 lanes per 64-B row segment (0: 16-B stores)
 #endif
@@ -372,24 +369,6 @@ __device__ __forceinline__ void readback_store32(__nv_bfloat16 *g, int ldc, uint
 // behind the producer's TMA loads), so nothing to wait for.
 __device__ __forceinline__ void store32_rows(__nv_bfloat16 *g, int ldc, uint32_t buf, int lane,
                                              const float (&v)[32], int col0, int row0, int M) {
-#if OOO_STG_DIRECT
-  {
-    uint32_t u[16];
-#pragma unroll
-    for (int j = 0; j < 16; ++j) u[j] = pack_bf2(v[2 * j], v[2 * j + 1]);
-    const int grow = row0 + lane;
-    if (grow < M) {
-      __nv_bfloat16 *d = g + (size_t)grow * ldc + col0;
-      asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(d), "r"(u[0]), "r"(u[1]),
-                   "r"(u[2]), "r"(u[3]), "r"(u[4]), "r"(u[5]), "r"(u[6]), "r"(u[7])
-                   : "memory");
-      asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(d + 16), "r"(u[8]),
-                   "r"(u[9]), "r"(u[10]), "r"(u[11]), "r"(u[12]), "r"(u[13]), "r"(u[14]), "r"(u[15])
-                   : "memory");
-    }
-    return;
-  }
-#endif
   __syncwarp();                            // previous read-back of buf finished
   const uint32_t rbase = buf + lane * 64;
 #pragma unroll
@@ -406,20 +385,6 @@ __device__ __forceinline__ void store32_rows(__nv_bfloat16 *g, int ldc, uint32_t
 // store32_rows for values already packed to bf16 pairs (u[j] = columns 2j, 2j+1).
 __device__ __forceinline__ void store32_rows_packed(__nv_bfloat16 *g, int ldc, uint32_t buf, int lane,
                                                     const uint32_t (&u)[16], int col0, int row0, int M) {
-#if OOO_STG_DIRECT
-  // experiment: each lane stores its own row as two full 32-B sectors
-  const int grow = row0 + lane;
-  if (grow < M) {
-    __nv_bfloat16 *d = g + (size_t)grow * ldc + col0;
-    asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(d), "r"(u[0]), "r"(u[1]),
-                 "r"(u[2]), "r"(u[3]), "r"(u[4]), "r"(u[5]), "r"(u[6]), "r"(u[7])
-                 : "memory");
-    asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" ::"l"(d + 16), "r"(u[8]),
-                 "r"(u[9]), "r"(u[10]), "r"(u[11]), "r"(u[12]), "r"(u[13]), "r"(u[14]), "r"(u[15])
-                 : "memory");
-  }
-  return;
-#endif
   __syncwarp();
   const uint32_t rbase = buf + lane * 64;
 #pragma unroll

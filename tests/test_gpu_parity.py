@@ -746,3 +746,21 @@ def test_pack_scale_average_over(dtype, n):
             "db": max(rel_fro(g * n, r) for g, r in zip(b["db"], ref.gb))}, BF16_TOL if dtype == "bf16" else FP32_TOL)
     plain.close()
     scaled.close()
+
+
+def test_wait_bound_traps_instead_of_hanging():
+    """Hang protection: with a bucket's all-reduce flag never
+    written, F_i(t+1) can never start; the engine's waits are bounded by the
+    stack's wait_timeout_ms (1.5 s here) and the step fails with a CUDA error
+    instead of hanging the GPU.  Run in child processes (a trap ends the CUDA
+    context); the control run with the flag written completes."""
+    import subprocess
+    import sys
+    import time
+    child = __file__.rsplit("/", 1)[0] + "/helpers/trap_child.py"
+    r = subprocess.run([sys.executable, child], capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, (r.returncode, r.stdout[-500:], r.stderr[-500:])
+    t0 = time.time()
+    r = subprocess.run([sys.executable, child, "drop"], capture_output=True, text=True, timeout=300)
+    assert r.returncode == 3, (r.returncode, r.stdout[-500:], r.stderr[-500:])
+    assert time.time() - t0 < 120
