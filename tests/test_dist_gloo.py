@@ -6,7 +6,13 @@
   full-batch gradient / N.
 * The collective rule of the ABI: the schedule D (and so the NCCL issue order)
   depends only on (L, k) -- every rank computes the same list.
-* The NCCL bootstrap id is broadcast over torch.distributed.
+* The NCCL bootstrap id is broadcast over torch.distributed (a failure is
+  a test failure: ncclGetUniqueId needs no GPU).
+* The rest of the N > 1 host plan is identical on every rank: the engine's
+  tile queue for a communicating stack (fwd_gate 2: F_i on its bucket's
+  all-reduce) and its topological order, the prioritised all-reduce chunk
+  order (NEXT-4), and the model-parallel pipeline's per-rank ownership
+  (NEXT-3: every group owned by exactly one rank).
 """
 import os
 import socket
@@ -60,13 +66,41 @@ def _worker(rank, world, port, q):
             Ds = [None] * world
             dist.all_gather_object(Ds, stack.schedule_order(L, "first_k", 2))
             assert all(d == Ds[0] for d in Ds)
-            try:
-                uid = stack.broadcast_unique_id()
-                ids = [None] * world
-                dist.all_gather_object(ids, uid)
-                assert len(uid) == 128 and all(x == ids[0] for x in ids)
-            except _lib.OooError:
-                pass                                 # NCCL bootstrap unavailable on this host
+            uid = stack.broadcast_unique_id()
+            ids = [None] * world
+            dist.all_gather_object(ids, uid)
+            assert len(uid) == 128 and all(x == ids[0] for x in ids)
+            # the engine queue of a communicating BERT-block stack: identical, topological
+            dims = [256, 256, 256, 256, 256, 1024, 256] * 1
+            acts = ["id", "id", "id", "id", "gelu", "id"]
+            q_ = stack.engine_plan(dims, acts, 512, "first_k", 2, fused=True, bucket_layers=2, world_size=world)
+            qs = [None] * world
+            dist.all_gather_object(qs, q_)
+            assert q_[1] and all(x == qs[0] for x in qs)
+            # the prioritised chunk order from identical predicted ready times
+            co = stack.comm_schedule([30.0, 10.0, 0.0], [[4.0, 4.0], [2.0], [3.0, 3.0, 1.0]], [1, 3, 5], "priority")
+            cos = [None] * world
+            dist.all_gather_object(cos, co)
+            assert all(x == cos[0] for x in cos)
+            # pipeline ownership: every group on exactly one rank (modulo placement)
+            import ctypes
+            d = _lib.PipelineDesc()
+            pd, pa = stack._i32arr([128] * 9), stack._i32arr([0] * 8)
+            d.num_layers, d.tokens, d.group_layers, d.n_stages, d.placement = 8, 64, 2, world, 1
+            d.dims = ctypes.cast(pd, ctypes.POINTER(ctypes.c_int32))
+            d.acts = ctypes.cast(pa, ctypes.POINTER(ctypes.c_int32))
+            d.world_size, d.rank = world, rank
+            idbuf = ctypes.create_string_buffer(uid, 128)
+            d.nccl_unique_id = ctypes.cast(idbuf, ctypes.c_void_p)
+            mine = []
+            for j in range(4):
+                o = ctypes.c_int64()
+                if _lib.load().ooo_pipeline_grads_offset(ctypes.byref(d), j, ctypes.byref(o)) == 0:
+                    mine.append(j)
+            owners = [None] * world
+            dist.all_gather_object(owners, mine)
+            assert sorted(j for m in owners for j in m) == [0, 1, 2, 3]
+            assert owners[rank] == [j for j in range(4) if j % world == rank]
         q.put((rank, out))
         dist.destroy_process_group()
     except Exception as e:  # pragma: no cover

@@ -1,7 +1,7 @@
 """Time one captured training step under different library knobs (env vars
-read at ooo_create_stack): OOO_ENGINE, OOO_EBN, OOO_ENGINE_CTAS, ...
+read at ooo_create_stack): OOO_EBN, OOO_ENGINE_CTAS, OOO_SPLITK, OOO_CG, ...
 
-    python tools/engine_sweep.py C2 "OOO_ENGINE=0" "OOO_EBN=192" "OOO_EBN=128"
+    python tools/engine_sweep.py C2 "" "OOO_EBN=128" "OOO_ENGINE_CTAS=132"
 A tuning aid, not part of the product path.
 """
 import json

@@ -26,15 +26,9 @@ def kernels(rnd, d):
     lines += ["", "The engine runs the whole step (all F / dO / dW tiles with fused epilogues; the bucket pack/scale BK5 "
               "is fused into the dW epilogue): tensor pipe active ≈ 47 % of its elapsed cycles -- the chain-latency bound "
               f"of `r{rnd}_chain_latency.md`; it is not HBM-bound (≈ 21 % of DRAM peak).  The seed (dZ_L = dY ⊙ act'(Z_L) "
-              "+ db partials) is latency-bound at ≈ 1.2 TB/s (≈ 12 µs, 0.5 % of the step).", "",
-              "## Per-layer multi-stream path (`OOO_ENGINE=0`, reverse first-k(12)): one GEMM kernel per op, split-K dW "
-              "+ `pack_kernel` (BK5)", ""]
-    lines += table(os.path.join(d, "perlayer.csv"))
-    lines += ["", "`gemm_tc_kernel<BN, A_MN, B_MN, EPI>`: EPI 0 = F_i (bias + act), 1 = dO_i (act-grad + db partials), "
-              "2 = dW_i split-K partials.  Short per-layer kernels keep the tensor pipe at 13-31 % -- the reason the "
-              "product path is the persistent engine (DESIGN.md §5).  `pack_kernel` sums the fp32 split-K and db "
-              "partials in a fixed order with the 1/N scale: ≈ 6.5 MB per launch at ≈ 850 GB/s (launch/latency-bound "
-              "at this size)."]
+              "+ db partials) is latency-bound at ≈ 1.2 TB/s (≈ 12 µs, 0.5 % of the step).  (Round 1 also "
+              "measured a per-layer multi-stream path, one GEMM kernel per op at 13-31 % tensor-pipe: deleted in "
+              "round 2.)"]
     open(os.path.join(ROOT, "profiles", f"r{rnd}_kernels.md"), "w").write("\n".join(lines) + "\n")
 
 
