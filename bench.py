@@ -297,7 +297,7 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_eurosys_ohlks22_b200 import configs, synth
-    from paper_conf_eurosys_ohlks22_b200.stack import OooStack, broadcast_unique_id
+    from paper_conf_eurosys_ohlks22_b200.stack import OooStack, broadcast_unique_id, deferral_bytes
 
     world, rank, local = dist_setup(args)
     torch.cuda.set_device(local)
@@ -723,7 +723,10 @@ def main():
         "dp_selfcheck": selfcheck,
         "nccl": nccl,
         "ooo_first_k0": {"value": 1e3 / ms_k0, "ms_per_step": ms_k0},
-        "ooo_first_k": {"k": k_best, "value": 1e3 / ms_fk if ms_fk else None, "ms_per_step": ms_fk},
+        "ooo_first_k": {"k": k_best, "value": 1e3 / ms_fk if ms_fk else None, "ms_per_step": ms_fk,
+                        "deferral_bytes": deferral_bytes(cfg.dims, cfg.acts, M, dt, k_best),
+                        "deferral_note": "extra live bytes of deferring dW_1..dW_k (sum_{i=2..k} |dZ_i|, §3 P:111, "
+                                         "E8); the engine keeps every dZ_i resident, so this is reported, not allocated"},
         "regions": regions,
         "emulated_dp": emulated,
         "step_roofline": {"ms": step_roof_ms, "frac": step_roof_ms / ms_ooo if step_roof_ms else None,
