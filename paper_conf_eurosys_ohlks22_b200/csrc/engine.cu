@@ -850,10 +850,12 @@ __global__ void __launch_bounds__(kThreads, 1)
           else mbar_arrive_cluster(L_tempty + 8 * acc);
         }
         ebar();                                  // all partial stores of this CTA precede the arrival
+        if (tr2) etrace2(t, 6);
         if (et == 0) {
           const int old = atom_add_acq_rel(ctr + cl.sk + o.sk_base + T.tile * CG + (int)rank, 1);
           *sk_flag = old == T.ks - 1;
         }
+        if (tr2) etrace2(t, 7);
         ebar();
         if (!*sk_flag) continue;                 // another split finishes this tile
       }

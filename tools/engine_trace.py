@@ -78,7 +78,13 @@ def report(name, ops, buf):
             print(f"     loads: first {np.mean(f6[ok] - tt[ok, 1]):6.1f} after ready, last {np.mean(f7[ok] - tt[ok, 1]):6.1f};"
                   f" acc {np.mean(tt[ok, 2] - f7[ok]):6.1f} after last; last-load range {f7[ok].min():8.1f}..{f7[ok].max():8.1f}")
         e = epi[s]
-        if e[:, 5].max() > 0:
+        sk = dn & (e[:, 7] > 0)                  # split-K last arrivals: phase A, arrival, reduction + epilogue
+        if sk.any():
+            es = e[sk]
+            print(f"     split-K cycles: partial store {np.median(es[:, 6] - es[:, 0]):6.0f} arrival"
+                  f" {np.median(es[:, 7] - es[:, 6]):6.0f} reduce+epilogue {np.median(es[:, 3] - es[:, 7]):6.0f}"
+                  f" publish {np.median(es[:, 5] - es[:, 3]):6.0f}")
+        elif e[:, 5].max() > 0:
             d = lambda a, b: np.median(e[:, b] - e[:, a])  # noqa: E731
             print(f"     epi cycles: tmem_ld {d(0, 1):6.0f} chunk0 {d(1, 2):6.0f} loop {d(0, 3):6.0f}"
                   f" tail {d(3, 4):6.0f} bar {d(4, 5):6.0f}")
