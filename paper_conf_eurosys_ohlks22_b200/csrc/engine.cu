@@ -618,6 +618,14 @@ __global__ void __launch_bounds__(kThreads, 1)
           if (b_mn) prefetch_b<CG, true>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre, T.nkb, T.kb0);
           else prefetch_b<CG, false>(mB, sbase, bar_empty, bar_full, L_full, leader, bytes, bn0, bh, it, npre, T.nkb, T.kb0);
         }
+        if (T.kind == EPI_DGRAD && o.mapZ >= 0 && am < T.M && !(p.dbg & 32)) {
+          // the epilogue multiplies by act'(Z_{i-1}) read from the Z_{i-1}
+          // store (written by the forward, long evicted from L2): request this
+          // CTA's rows of it now, a mainloop ahead of the epilogue's loads
+          const CUtensorMap *mZ = p.maps + o.mapZ;
+          const int ncol = min(T.bn, T.N - T.n0);
+          for (int c = 0; c < ncol; c += 64) tma_prefetch_l2_2d(mZ, T.n0 + c, am);
+        }
         deps<true>(p, T, T.mblk0 + (int)rank);    // this CTA's row block (no-op after a ready claim)
         asm volatile("fence.proxy.async.global;" ::: "memory");   // TMA reads see the producers' data
         if (leader) etrace(t, 1);

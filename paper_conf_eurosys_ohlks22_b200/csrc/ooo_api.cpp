@@ -88,7 +88,7 @@ struct LayerPlan {
 
 // Map-table slots per layer (engine): operand loads and output stores.
 enum MapSlot { MS_FWD_A = 0, MS_FWD_B, MS_FWD_X, MS_FWD_Z, MS_DX_A, MS_DX_B, MS_DZ_X, MS_DW_A, MS_DW_B,
-               MS_GW_X, MS_COUNT };
+               MS_GW_X, MS_Z_PF, MS_COUNT };
 
 struct Plan {
   int L = 0, M = 0, dtype = 0, elt = 2, R = 0, nbuckets = 0;
@@ -786,6 +786,8 @@ ooo::eng::Op op_of_unit(const ooo_stack *s, const pl::Unit &u) {
     o.mapA = (int16_t)map_index(i, MS_DX_A);
     o.mapB = (int16_t)map_index(i, MS_DX_B);
     o.mapX = (int16_t)(i >= 2 ? map_index(i - 1, MS_DZ_X) : ooo::eng::MAP_DX);
+    // the epilogue's act'(Z_{i-1}) input, L2-prefetched at dispatch
+    o.mapZ = (int16_t)(i >= 2 && s->lr[i - 2].Z ? map_index(i - 1, MS_Z_PF) : ooo::eng::MAP_NONE);
   } else if (u.kind == pl::WGRAD) {
     o.mapA = (int16_t)map_index(i, MS_DW_A);
     o.mapB = (int16_t)map_index(i, MS_DW_B);
@@ -1489,7 +1491,8 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
           (st = make_map(&m[MS_DZ_X], r.dZ, lp.dout, p.M, 32, 32, 64)) != OOO_OK ||
           (st = make_map(&m[MS_DW_A], r.X, lp.din, p.M, 64, 64)) != OOO_OK ||
           (st = make_map(&m[MS_DW_B], r.dZ, lp.dout, p.M, 64, 64)) != OOO_OK ||
-          (st = make_map(&m[MS_GW_X], r.gw, lp.dout, lp.din, 32, 32, 64)) != OOO_OK)
+          (st = make_map(&m[MS_GW_X], r.gw, lp.dout, lp.din, 32, 32, 64)) != OOO_OK ||
+          (r.Z && (st = make_map(&m[MS_Z_PF], r.Z, lp.dout, p.M, 64, 128)) != OOO_OK))
         return cleanup_fail(st);
       ooo::eng::LayerDev &L = ldev[i - 1];
       memset(&L, 0, sizeof(L));
