@@ -272,9 +272,10 @@ __device__ __forceinline__ void wait_ge(const int32_t *p, int target) {
 }
 
 __device__ __forceinline__ const CUtensorMap *map_of(int idx, const CUtensorMap *maps,
-                                                     const CUtensorMap *tmY, const CUtensorMap *tmDX) {
+                                                     const CUtensorMap *tmY, const CUtensorMap *tmDX,
+                                                     const CUtensorMap *tmX) {
   if (idx >= 0) return maps + idx;
-  return idx == MAP_Y ? tmY : tmDX;
+  return idx == MAP_Y ? tmY : (idx == MAP_DX ? tmDX : tmX);
 }
 
 // task index -> op (binary search over the ops' first task index)
@@ -333,12 +334,10 @@ __device__ __forceinline__ bool deps(const Params &p, const TaskRt &T, int mblk)
   const LayerDev &Ld = p.layers[T.layer - 1];
   bool ok = true;
   if (T.kind == EPI_FWD) {
-    if (mblk < cl.MT) {
-      if (T.layer > 1)
-        ok = dep_ge<kWait>(ctr + cl.fwd_rows + (T.layer - 2) * cl.MT + mblk, p.layers[T.layer - 2].fwd_nt);
-      else if (!(p.dbg & 8))
-        ok = dep_ge<kWait>(ctr + cl.xcopy + mblk, p.copy_nt);
-    }
+    // (F_1 reads the caller's X directly; the X -> X_1 copy for the next
+    // backward's dW_1 is off the chain)
+    if (mblk < cl.MT && T.layer > 1)
+      ok = dep_ge<kWait>(ctr + cl.fwd_rows + (T.layer - 2) * cl.MT + mblk, p.layers[T.layer - 2].fwd_nt);
     if (ok && p.fwd_gate == 1) ok = dep_ge<kWait>(ctr + cl.dw_done + (T.layer - 1), Ld.dw_tiles);   // P:84, N = 1
     else if (ok && p.fwd_gate == 2) ok = dep_ge<kWait>(ctr + cl.ar_done + Ld.bucket, 1);          // P:84, S[dW_i]
     if (ok && p.fwd_gate && T.layer < cl.L)      // WAR: dW_{i+1} reads X_{i+1}
@@ -486,12 +485,34 @@ __device__ __forceinline__ void produce(const TaskRt &T, const CUtensorMap *mA, 
   it += nst;
 }
 
+// X -> X_1 copy of one tile (epilogue threads), 8 vector loads in flight per
+// thread (a dependent load -> store loop waits one memory latency per
+// vector).  Not inlined: its registers stay out of the GEMM epilogue's
+// allocation (168-register cap, no spills).
+__device__ __noinline__ void copy_rows(const uint4 *__restrict__ src, uint4 *__restrict__ dst, size_t ld, int row0,
+                                       int c0, int vpr, int nv, int et) {
+  for (int v0 = et; v0 < nv; v0 += 8 * kEpiThreads) {
+    uint4 r[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int v = v0 + u * kEpiThreads;
+      if (v < nv) r[u] = __ldg(src + (size_t)(row0 + v / vpr) * ld + c0 + v % vpr);
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const int v = v0 + u * kEpiThreads;
+      if (v < nv) dst[(size_t)(row0 + v / vpr) * ld + c0 + v % vpr] = r[u];
+    }
+  }
+}
+
 // SK: the kernel contains the split-K epilogue path (launched only when the
 // queue has split ops -- skinny stacks), so the common path (C2, C3) carries
 // none of its registers.
 template <int CG, bool SK>
 __global__ void __launch_bounds__(kThreads, 1)
     engine_kernel(const __grid_constant__ CUtensorMap tmY, const __grid_constant__ CUtensorMap tmDX,
+                  const __grid_constant__ CUtensorMap tmX,
                   const __grid_constant__ Params p) {
   using C = Cfg<CG>;
   extern __shared__ uint8_t smem_raw[];
@@ -593,8 +614,8 @@ __global__ void __launch_bounds__(kThreads, 1)
         if (T.kind == EPI_COPY) continue;        // epilogue warps only
         const Op &o = p.ops[T.op];
         const LayerDev &Ld = p.layers[T.layer - 1];
-        const CUtensorMap *mA = map_of(o.mapA, p.maps, &tmY, &tmDX);
-        const CUtensorMap *mB = map_of(o.mapB, p.maps, &tmY, &tmDX);
+        const CUtensorMap *mA = map_of(o.mapA, p.maps, &tmY, &tmDX, &tmX);
+        const CUtensorMap *mB = map_of(o.mapB, p.maps, &tmY, &tmDX, &tmX);
         tma_prefetch(mA);      // descriptors live in global memory: warm the TMA descriptor cache
         tma_prefetch(mB);
         const bool a_mn = T.kind == EPI_WGRAD;
@@ -1080,7 +1101,8 @@ cudaError_t engine_init() {
   return e;
 }
 
-cudaError_t launch_engine(int cg, const Params &p, const CUtensorMap *tmY, const CUtensorMap *tmDX, int ctas,
+cudaError_t launch_engine(int cg, const Params &p, const CUtensorMap *tmY, const CUtensorMap *tmDX,
+                          const CUtensorMap *tmX, int ctas,
                           cudaStream_t stream, int priority) {
   bool sk = false;
   for (int j = 0; j < p.nops && !sk; ++j) sk = p.ops[j].ks > 1;
@@ -1104,15 +1126,15 @@ cudaError_t launch_engine(int cg, const Params &p, const CUtensorMap *tmY, const
     attr[2].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 3;
-    return sk ? cudaLaunchKernelEx(&cfg, engine_kernel<2, true>, *tmY, *tmDX, p)
-              : cudaLaunchKernelEx(&cfg, engine_kernel<2, false>, *tmY, *tmDX, p);
+    return sk ? cudaLaunchKernelEx(&cfg, engine_kernel<2, true>, *tmY, *tmDX, *tmX, p)
+              : cudaLaunchKernelEx(&cfg, engine_kernel<2, false>, *tmY, *tmDX, *tmX, p);
   }
   cfg.gridDim = dim3(ctas, 1, 1);
   cfg.dynamicSmemBytes = Cfg<1>::SMEM;
   cfg.attrs = attr;
   cfg.numAttrs = 2;
-  return sk ? cudaLaunchKernelEx(&cfg, engine_kernel<1, true>, *tmY, *tmDX, p)
-            : cudaLaunchKernelEx(&cfg, engine_kernel<1, false>, *tmY, *tmDX, p);
+  return sk ? cudaLaunchKernelEx(&cfg, engine_kernel<1, true>, *tmY, *tmDX, *tmX, p)
+            : cudaLaunchKernelEx(&cfg, engine_kernel<1, false>, *tmY, *tmDX, *tmX, p);
 }
 
 }  // namespace eng

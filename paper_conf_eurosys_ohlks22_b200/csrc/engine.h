@@ -30,6 +30,7 @@ constexpr int kMaxOps = 768;     // op table travels as a kernel parameter (<= 3
 constexpr int MAP_NONE = -1;
 constexpr int MAP_Y = -2;    // kernel-parameter map of the caller's Y
 constexpr int MAP_DX = -3;   // kernel-parameter map of the caller's dX
+constexpr int MAP_XIN = -4;  // kernel-parameter map of the caller's X (F_1's A operand)
 constexpr int EPI_COPY = 3;  // task kind: copy the caller's X rows into the X_1 store (no MMA)
 
 // One op of the queue = one row group of a layer GEMM (F_i, dO_i or dW_i), or
@@ -114,7 +115,8 @@ cudaError_t engine_init();
 #ifdef OOO_TRACE
 cudaError_t engine_set_trace(void *p);   // debug builds: per-task timestamps buffer
 #endif
-cudaError_t launch_engine(int cg, const Params &p, const CUtensorMap *tmY, const CUtensorMap *tmDX, int ctas,
+cudaError_t launch_engine(int cg, const Params &p, const CUtensorMap *tmY, const CUtensorMap *tmDX,
+                          const CUtensorMap *tmX, int ctas,
                           cudaStream_t stream, int priority);
 
 }  // namespace eng

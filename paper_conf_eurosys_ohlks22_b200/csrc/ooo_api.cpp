@@ -262,10 +262,12 @@ Plan make_plan(const ooo_stack_desc *d) {
       const int ks = std::min({std::min(8, env_int("OOO_SPLITK_MAX", 8)), ((K + 63) / 64) / minkb, workers / tiles});
       return ks >= 2 ? ks : 1;
     };
+    int ksmax = 1;
     for (int i = 1; i <= p.L; ++i) {
       LayerPlan &lp = p.layer[i - 1];
       lp.ks_fwd = ksplit(lp.dout, lp.ebn_fwd, lp.din, lp.act != OOO_ACT_RELU);
       lp.ks_dx = ksplit(lp.din, lp.ebn_dx, lp.dout, true);
+      ksmax = std::max({ksmax, lp.ks_fwd, lp.ks_dx});
       lp.sk_fwd = nsk;
       if (lp.ks_fwd > 1) nsk += PT * ((lp.dout + lp.ebn_fwd - 1) / lp.ebn_fwd) * p.cg;
       lp.sk_dx = nsk;
@@ -290,7 +292,7 @@ Plan make_plan(const ooo_stack_desc *d) {
     cl.dx_total = cl.ar_done + p.nbuckets;
     cl.total = cl.dx_total + 1;
     p.off_ctr = take((size_t)cl.total * 4);
-    if (nsk > 0) p.off_skpart = take((size_t)8 * cl.MT * p.sk_nc * 128 * 32 * 4);   // up to 8 splits
+    if (nsk > 0) p.off_skpart = take((size_t)ksmax * cl.MT * p.sk_nc * 128 * 32 * 4);   // [split][row block][chunk]
   }
   p.workspace_bytes = std::max<size_t>(off, 256);
   p.grad_elems = goff;
@@ -778,7 +780,7 @@ ooo::eng::Op op_of_unit(const ooo_stack *s, const pl::Unit &u) {
   }
   o.mapA = o.mapB = o.mapX = o.mapZ = ooo::eng::MAP_NONE;
   if (u.kind == pl::FWD) {
-    o.mapA = (int16_t)map_index(i, MS_FWD_A);
+    o.mapA = (int16_t)(i == 1 ? ooo::eng::MAP_XIN : map_index(i, MS_FWD_A));   // F_1 reads the caller's X
     o.mapB = (int16_t)map_index(i, MS_FWD_B);
     o.mapX = (int16_t)(i == p.L ? ooo::eng::MAP_Y : map_index(i, MS_FWD_X));
     o.mapZ = (int16_t)(s->lr[i - 1].Z ? map_index(i, MS_FWD_Z) : ooo::eng::MAP_NONE);
@@ -864,14 +866,17 @@ ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const 
 #ifdef OOO_TRACE
   s->last_queue.assign(P.ops, P.ops + P.nops);
 #endif
-  CUtensorMap tmY, tmDX;
+  CUtensorMap tmY, tmDX, tmX;
+  // F_1's A operand: the caller's X (no X -> X_1 copy on the chain); a
+  // launch without X (region profiling) reads the X_1 store instead
+  OOO_TRY(make_map(&tmX, X ? X : s->lr[0].X, s->dims[0], p.M, 64, a_box_rows(p)));
   if (Y) OOO_TRY(make_map(&tmY, Y, p.layer[p.L - 1].dout, p.M, 32, 32, 64));
   else memset(&tmY, 0, sizeof(tmY));    // unused placeholder
   if (dX) OOO_TRY(make_map(&tmDX, dX, s->dims[0], p.M, 32, 32, 64));
   else memset(&tmDX, 0, sizeof(tmDX));
   TimedRec *tr;
   OOO_TRY(begin_rec(s, s->hi, rec_kind, 0, 0, &tr));
-  CU_TRY(ooo::eng::launch_engine(p.cg, P, &tmY, &tmDX, s->engine_ctas, s->hi, s->prio_hi));
+  CU_TRY(ooo::eng::launch_engine(p.cg, P, &tmY, &tmDX, &tmX, s->engine_ctas, s->hi, s->prio_hi));
   return end_rec(tr, s->hi, s->engine_ctas, flops, 0);
 }
 
@@ -966,10 +971,12 @@ ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st)
   OOO_TRY(fork_from(s, st));
   double flops = 0;
   for (int i = 1; i <= L; ++i) flops += 2.0 * p.M * p.layer[i - 1].din * p.layer[i - 1].dout;
-  // the next forward: copy X -> X_1, then F_1..F_L (critical chain)
+  // the next forward: F_1..F_L (critical chain; F_1 reads the caller's X),
+  // then the copy X -> X_1 that the next backward's dW_1 reads (off the
+  // chain: it only waits for the pending dW_1, which still reads X_1)
   std::vector<pl::Unit> fwd;
-  if (!(env_int("OOO_DBG", 0) & 8)) fwd.push_back(unit_of(s, pl::COPY, 1));   // bit 3: timing experiments only
   for (int i = 1; i <= L; ++i) fwd.push_back(unit_of(s, pl::FWD, i));
+  if (!(env_int("OOO_DBG", 0) & 8)) fwd.push_back(unit_of(s, pl::COPY, 1));   // bit 3: timing experiments only
   if (s->eng_pending && env_int("OOO_FUSE", 1) == 0) OOO_TRY(engine_flush(s));   // experiments: unfused
   if (s->eng_pending) {
     if (s->emu_n > 1 || (s->nccl && s->d.comm_enabled)) {
@@ -988,7 +995,7 @@ ooo_status engine_forward(ooo_stack *s, const void *X, void *Y, cudaStream_t st)
     std::vector<pl::Unit> crit = s->eng_crit;
     crit.insert(crit.end(), fwd.begin(), fwd.end());
     std::vector<pl::Unit> defer = s->eng_defer;
-    const int f1 = (int)(crit.size() - L);   // index of F_1 in the chain
+    const int f1 = (int)(s->eng_crit.size());   // index of F_1 in the chain
     for (pl::Unit &u : defer)
       if (u.release <= -2) u.release = f1 + (-u.release - 1) - 1;   // region starting at F_m
     OOO_TRY(engine_launch(s, crit, defer, Y, s->eng_dX, X, s->eng_in_order, ar ? 2 : 1, 9,
@@ -1392,8 +1399,8 @@ ooo_status ooo_engine_plan(const ooo_stack_desc *d, ooo_schedule sch, int32_t fu
   double flops = 0;
   engine_bwd_units(&tmp, in_order, false, crit, defer, flops);
   if (fused) {
-    crit.push_back(unit_of(&tmp, pl::COPY, 1));
     for (int i = 1; i <= tmp.p.L; ++i) crit.push_back(unit_of(&tmp, pl::FWD, i));
+    crit.push_back(unit_of(&tmp, pl::COPY, 1));
   }
   pl::Problem pb;
   pb.L = tmp.p.L;

@@ -69,7 +69,7 @@ class Sim {
     double t = 0.0;
     switch (u.kind) {
       case FWD:
-        t = i > 1 ? row_done(FWD, i - 1, r) : row_done(COPY, 1, r);
+        t = i > 1 ? row_done(FWD, i - 1, r) : 0.0;   // F_1 reads the caller's X
         if (pb_.fwd_gate == 1) t = std::max(t, op_done(WGRAD, i));
         if (pb_.fwd_gate == 2) t = std::max(t, bucket_done(i));
         if (pb_.fwd_gate && i < pb_.L) t = std::max(t, op_done(WGRAD, i + 1));

@@ -85,10 +85,11 @@ def test_plan_small_ragged(workers, need_dx):
 
 
 def test_plan_in_order_is_d_then_forward():
-    """Conventional backprop: the queue is exactly D, then copy, F_1..F_L."""
+    """Conventional backprop: the queue is exactly D, then F_1..F_L (F_1 reads
+    the caller's X), then the X -> X_1 copy the next backward's dW_1 reads."""
     dims, acts = [256] * 7, ["id", "gelu"] * 3
     ops = _check_plan(dims, acts, 512, "in_order", 0, True, workers=74)
     names = [(n, l) for n, l, *_ in ops]
     D = S.in_order(6, False)
-    want = [("dO", o) if o > 0 else ("dW", -o) for o in D] + [("copy", 1)] + [("F", i) for i in range(1, 7)]
+    want = [("dO", o) if o > 0 else ("dW", -o) for o in D] + [("F", i) for i in range(1, 7)] + [("copy", 1)]
     assert names == want
