@@ -24,7 +24,7 @@ LIB = os.path.join(LIBDIR, "libooo.so")
 OBJDIR = os.path.join(PKG, "build_obj")
 
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-SOURCES = ["engine.cu", "gemm_simt.cu", "ew.cu", "ooo_api.cpp", "nccl_dyn.cpp", "planner.cpp", "regions.cpp", "comm_order.cpp", "pipeline.cpp"]
+SOURCES = ["engine.cu", "skinny.cu", "gemm_simt.cu", "ew.cu", "ooo_api.cpp", "nccl_dyn.cpp", "planner.cpp", "regions.cpp", "comm_order.cpp", "pipeline.cpp"]
 
 
 def _nvcc() -> str:

@@ -65,7 +65,8 @@ struct LayerDev {
   int32_t fwd_nt;          // n-tiles of F_i over d_i
   int32_t dx_nt;           // n-tiles of dO_i over d_{i-1}
   int32_t dw_tiles;        // 128-row tiles of dW_i (completion count)
-  int32_t pad1[9];
+  int32_t fwd_bn, dx_bn, dw_bn;   // tile widths of F_i / dO_i / dW_i
+  int32_t pad1[6];
 };
 static_assert(sizeof(LayerDev) == 128, "LayerDev layout");
 

@@ -30,6 +30,7 @@
 #include "kernels.h"
 #include "nccl_dyn.h"
 #include "planner.h"
+#include "skinny.h"
 
 using namespace ooo;
 
@@ -88,7 +89,7 @@ struct LayerPlan {
 
 // Map-table slots per layer (engine): operand loads and output stores.
 enum MapSlot { MS_FWD_A = 0, MS_FWD_B, MS_FWD_X, MS_FWD_Z, MS_DX_A, MS_DX_B, MS_DZ_X, MS_DW_A, MS_DW_B,
-               MS_GW_X, MS_Z_PF, MS_COUNT };
+               MS_GW_X, MS_Z_PF, MS_SK_X, MS_SK_DZ, MS_COUNT };
 
 struct Plan {
   int L = 0, M = 0, dtype = 0, elt = 2, R = 0, nbuckets = 0;
@@ -101,6 +102,7 @@ struct Plan {
   // engine (bf16): map table, layer table, completion counters
   bool engine = false;
   int cg = 2;                      // engine CTAs per tile (2 = CTA pairs, cta_group::2)
+  bool skinny = false;             // <= 16 tokens: the skinny-stack kernel (skinny.h) runs every engine launch
   size_t off_maps = 0, off_layers = 0, off_ctr = 0;
   size_t off_skpart = 0;           // split-K partials (0 bytes when no op splits)
   int sk_nc = 0;                   // 32-column chunks per partial row
@@ -243,6 +245,16 @@ Plan make_plan(const ooo_stack_desc *d) {
       lp.ebn_dx = engine_bn(lp.din, true, p.cg, PT, workers, lp.dout);
       lp.ebn_dw = engine_bn(lp.dout, false, p.cg, PT, workers);
     }
+    // <= 16 tokens: chain ops as 8-CTA clusters with a DSMEM K-split
+    // reduction (skinny.h; OOO_SKINNY=0 keeps the engine): 128-wide chain
+    // tiles where the width allows (the kernel's tile widths)
+    p.skinny = p.cg == 1 && p.M <= ooo::sk::kMaxM && env_int("OOO_SKINNY", 1) != 0;
+    if (p.skinny)
+      for (int i = 1; i <= p.L; ++i) {
+        LayerPlan &lp = p.layer[i - 1];
+        lp.ebn_fwd = lp.dout % 128 == 0 ? 128 : 64;
+        lp.ebn_dx = lp.din % 128 == 0 ? 128 : 64;
+      }
     // split-K chain ops when all tokens fit one 128-row tile (C5: 16 tokens):
     // a chain op's latency is its k-blocks at the MMA issue rate, whatever its
     // width (profiles/r02_mainloop_issue.md), so its K is spread over up to 8
@@ -256,7 +268,7 @@ Plan make_plan(const ooo_stack_desc *d) {
     int nsk = 0, maxw = 0;
     for (int i = 0; i <= p.L; ++i) maxw = std::max(maxw, d->dims[i]);
     auto ksplit = [&](int N, int bn, int K, bool allowed) {
-      if (!allowed || p.M > 128 || env_int("OOO_SPLITK", 1) == 0) return 1;
+      if (!allowed || p.M > 128 || p.skinny || env_int("OOO_SPLITK", 1) == 0) return 1;
       const int tiles = PT * ((N + bn - 1) / bn);
       const int minkb = std::max(1, env_int("OOO_SPLITK_MINKB", 4));
       const int ks = std::min({std::min(8, env_int("OOO_SPLITK_MAX", 8)), ((K + 63) / 64) / minkb, workers / tiles});
@@ -815,10 +827,86 @@ void engine_bwd_units(const ooo_stack *s, bool in_order, bool regions, std::vect
   }
 }
 
+// Skinny stacks (skinny.h): the chain ops (F_i, dO_i) in chain order for the
+// chain clusters, the dW ops in D's order (Alg. 2) and the X -> X_1 copy for
+// the dW workers; same counters, gates and stores as the engine.
+ooo_status skinny_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const std::vector<pl::Unit> &defer,
+                         void *Y, void *dX, const void *X, bool in_order, int fwd_gate, int rec_kind, double flops) {
+  const Plan &p = s->p;
+  static ooo::sk::Params P;   // ~7 KB: not on the stack (launches are serialised by the caller)
+  memset(&P, 0, sizeof(P));
+  P.L = p.L;
+  P.M = p.M;
+  P.in_order = in_order ? 1 : 0;
+  P.fwd_gate = fwd_gate;
+  P.dbg = env_int("OOO_DBG", 0);
+  P.alpha = grad_alpha(s);
+  P.timeout_ns = (uint64_t)s->timeout_ms * 1000000ull;
+  P.maps = s->dmaps;
+  P.maps_per_layer = MS_COUNT;
+  P.map_x = MS_SK_X;
+  P.map_dz = MS_SK_DZ;
+  P.map_w = MS_FWD_B;
+  P.ctr = s->ctr;
+  P.layers = s->dlayers;
+  P.cl = p.cl;
+  P.y_out = Y;
+  P.dx_out = dX;
+  P.x_in = X;
+  int max_tiles = 0, ntask = 0;
+  auto add_chain = [&](const pl::Unit &u) {
+    if (P.nchain >= ooo::sk::kMaxChain) return false;
+    P.chain[P.nchain].kind = (int16_t)u.kind;
+    P.chain[P.nchain].layer = (int16_t)u.layer;
+    ++P.nchain;
+    const LayerPlan &lp = p.layer[u.layer - 1];
+    max_tiles = std::max(max_tiles, u.kind == pl::FWD ? lp.dout / lp.ebn_fwd : lp.din / lp.ebn_dx);
+    return true;
+  };
+  auto add_dw = [&](const pl::Unit &u) {
+    if (P.ndw >= ooo::sk::kMaxDw) return false;
+    ooo::sk::DwOp &o = P.dw[P.ndw++];
+    o.kind = (int16_t)u.kind;
+    o.layer = (int16_t)u.layer;
+    o.first = ntask;
+    const LayerPlan &lp = p.layer[u.layer - 1];
+    ntask += u.kind == pl::COPY ? 1 : ((lp.din + 127) / 128) * ((lp.dout + lp.ebn_dw - 1) / lp.ebn_dw);
+    return true;
+  };
+  for (const std::vector<pl::Unit> *v : {&crit, &defer})
+    for (const pl::Unit &u : *v)
+      if ((u.kind == pl::FWD || u.kind == pl::DGRAD) && !add_chain(u))
+        return fail(OOO_ERR_UNSUPPORTED, "skinny: too many chain ops");
+  for (const std::vector<pl::Unit> *v : {&crit, &defer})
+    for (const pl::Unit &u : *v)
+      if (u.kind == pl::WGRAD && !add_dw(u)) return fail(OOO_ERR_UNSUPPORTED, "skinny: too many dW ops");
+  for (const std::vector<pl::Unit> *v : {&crit, &defer})
+    for (const pl::Unit &u : *v)
+      if (u.kind == pl::COPY && !add_dw(u)) return fail(OOO_ERR_UNSUPPORTED, "skinny: too many dW ops");
+  P.ntasks_dw = ntask;
+  // clusters: as many chain clusters as the widest chain op has tiles, at
+  // least one dW-worker cluster when there are dW tasks
+  const int total = std::min(s->engine_ctas / ooo::sk::kCl, ooo::sk::skinny_max_clusters());
+  if (total < (P.nchain > 0) + (P.ndw > 0)) return fail(OOO_ERR_UNSUPPORTED, "skinny: %d clusters fit", total);
+  P.nclu = P.nchain > 0 ? std::max(1, std::min(max_tiles, total - (P.ndw > 0 ? 1 : 0))) : 0;
+  const int clusters = P.ndw > 0 ? total : P.nclu;
+  if (env_int("OOO_SKINNY_VERBOSE", 0))
+    fprintf(stderr, "[skinny] max_clusters %d total %d chain clusters %d (widest op %d tiles) launch %d; "
+            "chain ops %d, dW ops %d (%d tasks)\n", ooo::sk::skinny_max_clusters(), total, P.nclu, max_tiles,
+            clusters, P.nchain, P.ndw, P.ntasks_dw);
+  CUtensorMap tmX;
+  OOO_TRY(make_map(&tmX, X ? X : s->lr[0].X, s->dims[0], p.M, 64, 16));
+  TimedRec *tr;
+  OOO_TRY(begin_rec(s, s->hi, rec_kind, 0, 0, &tr));
+  CU_TRY(ooo::sk::launch_skinny(P, &tmX, clusters, s->hi));
+  return end_rec(tr, s->hi, clusters * ooo::sk::kCl, flops, 0);
+}
+
 // Plans the FIFO order (planner.h) and launches the engine on it.
 ooo_status engine_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const std::vector<pl::Unit> &defer,
                          void *Y, void *dX, const void *X, bool in_order, int fwd_gate, int rec_kind, double flops) {
   const Plan &p = s->p;
+  if (p.skinny) return skinny_launch(s, crit, defer, Y, dX, X, in_order, fwd_gate, rec_kind, flops);
   pl::Problem pb;
   pb.L = p.L;
   pb.rows = (p.cl.MT + p.cg - 1) / p.cg;
@@ -1478,7 +1566,10 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
   if (p.engine) {
     static std::once_flag eng_once;
     static cudaError_t eng_err = cudaSuccess;
-    std::call_once(eng_once, [] { eng_err = ooo::eng::engine_init(); });
+    std::call_once(eng_once, [] {
+      eng_err = ooo::eng::engine_init();
+      if (eng_err == cudaSuccess) eng_err = ooo::sk::skinny_init();
+    });
     if (eng_err != cudaSuccess)
       return cleanup_fail(fail(OOO_ERR_CUDA, "engine init: %s", cudaGetErrorString(eng_err)));
     std::vector<CUtensorMap> maps((size_t)p.L * MS_COUNT);
@@ -1499,7 +1590,9 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
           (st = make_map(&m[MS_DW_A], r.X, lp.din, p.M, 64, 64)) != OOO_OK ||
           (st = make_map(&m[MS_DW_B], r.dZ, lp.dout, p.M, 64, 64)) != OOO_OK ||
           (st = make_map(&m[MS_GW_X], r.gw, lp.dout, lp.din, 32, 32, 64)) != OOO_OK ||
-          (r.Z && (st = make_map(&m[MS_Z_PF], r.Z, lp.dout, p.M, 64, 128)) != OOO_OK))
+          (r.Z && (st = make_map(&m[MS_Z_PF], r.Z, lp.dout, p.M, 64, 128)) != OOO_OK) ||
+          (p.skinny && (st = make_map(&m[MS_SK_X], r.X, lp.din, p.M, 64, 16)) != OOO_OK) ||
+          (p.skinny && (st = make_map(&m[MS_SK_DZ], r.dZ, lp.dout, p.M, 64, 16)) != OOO_OK))
         return cleanup_fail(st);
       ooo::eng::LayerDev &L = ldev[i - 1];
       memset(&L, 0, sizeof(L));
@@ -1518,6 +1611,9 @@ ooo_status ooo_create_stack(const ooo_stack_desc *d, ooo_stack **out) {
       L.fwd_nt = (lp.dout + lp.ebn_fwd - 1) / lp.ebn_fwd;
       L.dx_nt = (lp.din + lp.ebn_dx - 1) / lp.ebn_dx;
       L.dw_tiles = ((lp.din + 127) / 128) * ((lp.dout + lp.ebn_dw - 1) / lp.ebn_dw);
+      L.fwd_bn = lp.ebn_fwd;
+      L.dx_bn = lp.ebn_dx;
+      L.dw_bn = lp.ebn_dw;
     }
     cudaError_t ce = cudaMemcpy(s->ws + p.off_maps, maps.data(), maps.size() * sizeof(CUtensorMap),
                                 cudaMemcpyHostToDevice);
@@ -1963,6 +2059,10 @@ ooo_graph *wrap_graph(cudaGraph_t g, cudaGraphExec_t e) {
 // filled by the engine kernels (tools/engine_trace.py).
 extern "C" ooo_status ooo_debug_set_trace(void *dev_ptr) {
   CU_TRY(ooo::eng::engine_set_trace(dev_ptr));
+#ifdef OOO_TRACE
+  // skinny stacks: after the engine's three 200000 x 8 stamp arrays
+  CU_TRY(ooo::sk::skinny_set_trace(dev_ptr ? static_cast<char *>(dev_ptr) + (size_t)3 * 200000 * 8 * 8 : nullptr));
+#endif
   return OOO_OK;
 }
 

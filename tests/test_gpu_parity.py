@@ -152,7 +152,8 @@ def test_bf16_bert_base_full_config_end_to_end():
 
 # ------------------------------- fused step: backward(t) + forward(t+1)
 @pytest.mark.parametrize("kind,k,tokens,need_dx", [("first_k", 2, 400, False), ("first_k", 5, 264, True),
-                                                   ("in_order", 0, 512, False), ("first_k", 0, 136, False)])
+                                                   ("in_order", 0, 512, False), ("first_k", 0, 136, False),
+                                                   ("first_k", 2, 16, True), ("in_order", 0, 8, False)])
 def test_bf16_fused_step_across_iterations(kind, k, tokens, need_dx):
     """ooo_backward(t); ooo_forward(X_{t+1}) runs as one engine launch whose
     F_i tiles overlap the deferred dW tiles (Fig. 4(c)).  Over three
@@ -194,14 +195,15 @@ def test_bf16_fused_step_across_iterations(kind, k, tokens, need_dx):
     plain.close()
 
 
-def test_bf16_fused_step_comm_gated(monkeypatch):
+@pytest.mark.parametrize("tokens", [520, 16])
+def test_bf16_fused_step_comm_gated(monkeypatch, tokens):
     """The N > 1 gating of the fused step (F_i waits for its bucket's
     all-reduce flag, written by the comm stream after cuStreamWaitValue32 on
     the bucket's dW counter) on one GPU: OOO_TEST_COMM_GATE runs that
     wait/write chain without the all-reduce.  Results must be bit-identical
     to the ungated stack (the all-reduce of one rank is the identity)."""
     dims, acts = [256, 512, 256, 256, 512, 256], ["gelu", "id", "id", "gelu", "id"]
-    cases = [Case(dims, acts, 520, "bf16", step=t) for t in range(3)]
+    cases = [Case(dims, acts, tokens, "bf16", step=t) for t in range(3)]
     plain = cases[0].stack(bucket_layers=2)
     monkeypatch.setenv("OOO_TEST_COMM_GATE", "1")
     gated = cases[0].stack(bucket_layers=2)
@@ -226,13 +228,14 @@ def test_bf16_fused_step_comm_gated(monkeypatch):
     plain.close()
 
 
-@pytest.mark.parametrize("kind,k", [("first_k", 2), ("first_k", 0), ("in_order", 0)])
-def test_bf16_emulated_allreduce_graph(monkeypatch, kind, k):
+@pytest.mark.parametrize("kind,k,tokens", [("first_k", 2, 520), ("first_k", 0, 520), ("in_order", 0, 520),
+                                          ("first_k", 2, 16)])
+def test_bf16_emulated_allreduce_graph(monkeypatch, kind, k, tokens):
     """The emulated N = 8 all-reduce (OOO_EMULATE_AR_N: the comm stream held
     for each bucket's ring time, 16-SM NCCL reserve; bench.py's emulated_dp)
     through the captured step as bench.py times it: bit-identical to the
     plain stack, within the gate of the oracle."""
-    case = Case([256, 512, 256, 256, 512, 256], ["gelu", "id", "id", "gelu", "id"], 520, "bf16")
+    case = Case([256, 512, 256, 256, 512, 256], ["gelu", "id", "id", "gelu", "id"], tokens, "bf16")
     plain = case.stack(bucket_layers=2)
     base = case.run(plain, kind, k, graph=True, launches=2)
     plain.close()
@@ -257,7 +260,7 @@ def _region_plan_valid(stk, L, need_dx=False):
     return plan
 
 
-@pytest.mark.parametrize("tokens,rl,need_dx", [(384, 2, False), (264, 1, True), (136, 3, False)])
+@pytest.mark.parametrize("tokens,rl,need_dx", [(384, 2, False), (264, 1, True), (136, 3, False), (16, 2, True)])
 def test_bf16_regions_schedule_bit_exact(tokens, rl, need_dx):
     """OOO_SCHED_REGIONS (dW kernels placed by Algorithm 1 from profiled
     co-run speedups) gives the gradients of in_order bit for bit and the
@@ -424,8 +427,9 @@ def _nccl_stack(case, monkeypatch, **kw):
     return case.stack(unique_id=get_unique_id(), **kw)
 
 
-@pytest.mark.parametrize("kind,k", [("first_k", 2), ("in_order", 0), ("first_k", 5)])
-def test_bf16_nccl_one_rank_fused_steps_bit_exact(monkeypatch, kind, k):
+@pytest.mark.parametrize("kind,k,tokens", [("first_k", 2, 520), ("in_order", 0, 520), ("first_k", 5, 520),
+                                          ("first_k", 2, 16)])
+def test_bf16_nccl_one_rank_fused_steps_bit_exact(monkeypatch, kind, k, tokens):
     """A real NCCL communicator (world_size 1, ooo_get_unique_id) drives the
     whole N > 1 data plane through the captured fused step:
     per-bucket cuStreamWaitValue32 on the engine's dW counters ->
@@ -435,7 +439,7 @@ def test_bf16_nccl_one_rank_fused_steps_bit_exact(monkeypatch, kind, k):
     is the identity) and the oracle within the bf16 gate; the library's
     launch records show one all-reduce per bucket."""
     dims, acts = [256, 512, 256, 256, 512, 256], ["gelu", "id", "id", "gelu", "id"]
-    cases = [Case(dims, acts, 520, "bf16", step=t) for t in range(4)]
+    cases = [Case(dims, acts, tokens, "bf16", step=t) for t in range(4)]
     plain = cases[0].stack(bucket_layers=2)
     comm = _nccl_stack(cases[0], monkeypatch, bucket_layers=2)
     Xb = [to_dev(cases[0].X, "bf16") for _ in range(2)]

@@ -125,6 +125,36 @@ __global__ void __launch_bounds__(288, 1) epi(__nv_bfloat16 *out, int ldc, int t
       asm volatile("bar.sync 1, 256;" ::: "memory");
       continue;
     }
+    if (MODE >= 7) {
+      // GELU F epilogue as in the engine: Z = bf16(acc + b); X = gelu(Z), d = gelu'(Z)
+      // 7: both stored, 8: X only, 9: no stores (math only)
+      tmem_ld32_issue(tbase + (uint32_t)(h * 32), ra);
+      for (int c = h; c < 8; c += 2) {
+        const int col0 = (tile % 3) * 256 + c * 32;
+        tmem_ld_wait(ra);
+        float v[32];
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(ra[i]);
+        if (c + 2 < 8) tmem_ld32_issue(tbase + (uint32_t)((c + 2) * 32), ra);
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] += bias_s[c * 32 + i];
+        uint32_t u[16];
+        pack32(v, u);
+        unpack32(u, v);
+        float dd[32];
+        gelu_and_grad_chunk32(v, dd);
+        if (MODE <= 8) store32_rows(out, ldc, stg, lane, v, col0, row0, 1 << 30);
+        if (MODE == 7) store32_rows(out + (size_t)148 * 128 * ldc, ldc, stg, lane, dd, col0, row0, 1 << 30);
+        if (MODE == 9) {
+          float x = 0.f;
+#pragma unroll
+          for (int j = 0; j < 32; ++j) x += v[j] * dd[j];
+          if (x == 1234.5f) out[threadIdx.x] = __float2bfloat16(1.f);
+        }
+      }
+      asm volatile("bar.sync 1, 256;" ::: "memory");
+      continue;
+    }
     tmem_ld32_issue(tbase + (uint32_t)(h * 32), ra);
     for (int c = h; c < 8; c += 2) {
       const int col0 = (tile % 3) * 256 + c * 32;
@@ -171,7 +201,7 @@ typedef CUresult (*Enc)(CUtensorMap *, CUtensorMapDataType, cuuint32_t, void *, 
 int main() {
   __nv_bfloat16 *out;
   const int ldc = 768, rows = 148 * 128;
-  cudaMalloc(&out, (size_t)rows * ldc * 2);
+  cudaMalloc(&out, (size_t)2 * rows * ldc * 2);
   long long *d;
   cudaMalloc(&d, 148 * 8);
   void *fn = nullptr;
@@ -183,13 +213,16 @@ int main() {
   ((Enc)fn)(&om, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, out, dims, str, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
             CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   const int tiles = 200;
-  void (*ks[14])(__nv_bfloat16 *, int, int, long long *, CUtensorMap) = {epi<0, false>, epi<1, false>, epi<2, false>, epi<3, false>, epi<4, false>, epi<5, false>, epi<6, false>,
-                                                                       epi<0, true>, epi<1, true>, epi<2, true>, epi<3, true>, epi<4, true>, epi<5, true>, epi<6, true>};
-  const char *names[7] = {"TMEM ld + bias + pack, no stores", "+ smem-transpose stores", "same with stores, no-TMEM math",
+  void (*ks[20])(__nv_bfloat16 *, int, int, long long *, CUtensorMap) = {epi<0, false>, epi<1, false>, epi<2, false>, epi<3, false>, epi<4, false>, epi<5, false>, epi<6, false>,
+                                                                       epi<7, false>, epi<8, false>, epi<9, false>,
+                                                                       epi<0, true>, epi<1, true>, epi<2, true>, epi<3, true>, epi<4, true>, epi<5, true>, epi<6, true>,
+                                                                       epi<7, true>, epi<8, true>, epi<9, true>};
+  const char *names[10] = {"TMEM ld + bias + pack, no stores", "+ smem-transpose stores", "same with stores, no-TMEM math",
                           "TMA (bulk tensor) stores", "direct per-row st.global.v4 (no smem)",
-                          "64-col chunks, full 128-B row stores", "smem-transpose stores, 2 TMEM loads in flight"};
-  for (int m = 0; m < 14; ++m) {
-    if (m == 7) printf("-- with concurrent MMAs into the other TMEM half:\n");
+                          "64-col chunks, full 128-B row stores", "smem-transpose stores, 2 TMEM loads in flight",
+                          "GELU: X and gelu' stored", "GELU: X stored only", "GELU: math only, no stores"};
+  for (int m = 0; m < 20; ++m) {
+    if (m == 10) printf("-- with concurrent MMAs into the other TMEM half:\n");
     ks[m]<<<148, 288>>>(out, ldc, tiles, d, om);
     cudaError_t e = cudaDeviceSynchronize();
     long long h[148];
@@ -197,7 +230,7 @@ int main() {
     double mm = 0;
     for (int i = 0; i < 148; ++i) mm += h[i];
     mm /= 148;
-    printf("%-40s %8.0f cycles per 128x256 tile  (%s)\n", names[m % 7], mm / tiles, cudaGetErrorString(e));
+    printf("%-40s %8.0f cycles per 128x256 tile  (%s)\n", names[m % 10], mm / tiles, cudaGetErrorString(e));
   }
   return 0;
 }
