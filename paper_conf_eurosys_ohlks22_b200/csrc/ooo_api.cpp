@@ -1239,12 +1239,13 @@ ooo_status profile_launch(ooo_stack *s, const std::vector<pl::Unit> &crit, const
     return false;
   };
   std::vector<int32_t> img(cl.total, 0);
+  const int pub = p.skinny ? ooo::sk::kPubPerTile : 1;   // publications per chain tile
   for (int i = 1; i <= p.L; ++i) {
     if (!in(pl::FWD, i))
-      for (int m = 0; m < cl.MT; ++m) img[cl.fwd_rows + (i - 1) * cl.MT + m] = fwd_nt_of(p, i);
+      for (int m = 0; m < cl.MT; ++m) img[cl.fwd_rows + (i - 1) * cl.MT + m] = fwd_nt_of(p, i) * pub;
     if (i >= 2 && !in(pl::DGRAD, i)) {
-      for (int m = 0; m < cl.MT; ++m) img[cl.dz_rows + (i - 2) * cl.MT + m] = dx_nt_of(p, i);
-      img[cl.dz_total + i - 2] = cl.MT * dx_nt_of(p, i);
+      for (int m = 0; m < cl.MT; ++m) img[cl.dz_rows + (i - 2) * cl.MT + m] = dx_nt_of(p, i) * pub;
+      img[cl.dz_total + i - 2] = cl.MT * dx_nt_of(p, i) * pub;
     }
     if (!in(pl::WGRAD, i)) img[cl.dw_done + i - 1] = dw_tiles_of(p, i);
   }
@@ -1739,7 +1740,8 @@ ooo_status ooo_input_grad_wait(ooo_stack *s, void *stream) {
   static StreamValueFn wait_fn = stream_value_fn("cuStreamWaitValue32");
   if (!wait_fn) return fail(OOO_ERR_CUDA, "stream memory operations unavailable");
   // every 128-row block of dO_1's output, once per column tile (engine.cu: dx_total)
-  const uint32_t target = (uint32_t)(s->p.cl.MT * ((s->dims[0] + s->p.layer[0].ebn_dx - 1) / s->p.layer[0].ebn_dx));
+  const uint32_t target = (uint32_t)(s->p.cl.MT * ((s->dims[0] + s->p.layer[0].ebn_dx - 1) / s->p.layer[0].ebn_dx) *
+                                     (s->p.skinny ? ooo::sk::kPubPerTile : 1));
   CUresult r = wait_fn(static_cast<cudaStream_t>(stream), reinterpret_cast<CUdeviceptr>(s->ctr + s->p.cl.dx_total),
                        target, CU_STREAM_WAIT_VALUE_GEQ);
   if (r != CUDA_SUCCESS) return fail(OOO_ERR_CUDA, "cuStreamWaitValue32 failed (%d)", (int)r);

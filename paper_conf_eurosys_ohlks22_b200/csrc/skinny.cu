@@ -24,12 +24,18 @@ constexpr int A_SK = 2048;       // 16 rows x 128 B (K-major, SW128)
 constexpr int B_SK = 16384;      // <= 128 N x 64 K bf16
 constexpr int STAGE = A_SK + B_SK;
 constexpr int RING = STAGES * STAGE;
-constexpr int PROW = 528;        // partial row stride (bytes): 128 fp32 + 16 B (conflict-free v4 reads)
-constexpr int PART_OFF = RING;
-constexpr int PART = kCl * kMaxM * PROW;   // slot 0: this CTA's own partial; leader: slots 1..7 = peers
-constexpr int STG_OFF = (PART_OFF + PART + 1023) / 1024 * 1024;
+// Chain-tile reduction (reduce-scatter over the cluster): CTA o owns columns
+// [o cs, o cs + cs) of the tile (cs = tn / kCl); each CTA sends the owner its
+// fp32 partial of those columns (a block of kMaxM rows x RS floats, RS = cs + 4:
+// the pad spreads the rows over the banks) into the owner's receive slot
+// [sender], double-buffered by task parity.
+constexpr int RS_MAX = 128 / kCl + 4;
+constexpr int BLK_MAX = kMaxM * RS_MAX * 4;          // one sender -> owner block (bytes)
+constexpr int SEND_OFF = RING;                       // [2][kCl owners][BLK_MAX]
+constexpr int RECV_OFF = SEND_OFF + 2 * kCl * BLK_MAX;   // [2][kCl senders][BLK_MAX]
+constexpr int STG_OFF = (RECV_OFF + 2 * kCl * BLK_MAX + 1023) / 1024 * 1024;
 constexpr int BAR_OFF = STG_OFF + 4 * 2048;
-constexpr int NBARS = 2 * STAGES + 4 + 8 + 8;
+constexpr int NBARS = 2 * STAGES + 6 + 8 + 8;
 constexpr int SLOT_OFF = BAR_OFF + NBARS * 8;
 constexpr int SMEM = SLOT_OFF + 64 + 1024;
 constexpr int DW_BUF = 16384;    // dW role: A (2 panels x 2 KB) + B (<= 4 panels x 2 KB) per buffer
@@ -80,10 +86,6 @@ __device__ __forceinline__ void cluster_sync() {
 }
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
-}
-__device__ __forceinline__ void st_cluster_v4(uint32_t addr, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
-  asm volatile("st.shared::cluster.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d)
-               : "memory");
 }
 // non-blocking phase test (try_wait may suspend the thread for a while: the
 // producer's loop polls two cursors and must not stall on either)
@@ -136,12 +138,6 @@ __device__ __forceinline__ void red_release_add(int32_t *p, int v) {
   asm volatile("red.release.gpu.global.add.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-// 32 bf16 already packed in pairs -> 64 contiguous bytes
-__device__ __forceinline__ void st_bf16x32_packed(__nv_bfloat16 *p, const uint32_t (&u)[16]) {
-  uint4 *q = reinterpret_cast<uint4 *>(p);
-#pragma unroll
-  for (int j = 0; j < 4; ++j) q[j] = make_uint4(u[4 * j], u[4 * j + 1], u[4 * j + 2], u[4 * j + 3]);
-}
 
 // The chain op's shape: output width N, reduction length K, tile width.
 struct OpShape {
@@ -213,10 +209,10 @@ __device__ __forceinline__ bool input_ok(const Params &p, const OpShape &sh) {
   const int i = sh.layer;
   if (sh.kind == EPI_FWD) {
     if (i == 1) return true;
-    return reached(p.ctr + cl.fwd_rows + (i - 2) * cl.MT, p.layers[i - 2].fwd_nt);
+    return reached(p.ctr + cl.fwd_rows + (i - 2) * cl.MT, p.layers[i - 2].fwd_nt * kPubPerTile);
   }
   if (i == cl.L) return true;
-  return reached(p.ctr + cl.dz_rows + (i - 1) * cl.MT, p.layers[i].dx_nt);
+  return reached(p.ctr + cl.dz_rows + (i - 1) * cl.MT, p.layers[i].dx_nt * kPubPerTile);
 }
 
 __global__ void __launch_bounds__(kThreads, 1)
@@ -228,9 +224,9 @@ __global__ void __launch_bounds__(kThreads, 1)
   const uint32_t bar_empty = bar_full + 8 * STAGES;
   const uint32_t c_accfull = bar_empty + 8 * STAGES;
   const uint32_t c_accfree = c_accfull + 8;
-  const uint32_t redfull = c_accfree + 8;   // leader: the 7 peers' partials have landed
-  const uint32_t redfree = redfull + 8;     // peer: the leader has read its partial
-  const uint32_t d_buffull = redfree + 8;   // [2]
+  const uint32_t rfull = c_accfree + 8;     // [2] owner: every sender's block of its columns landed
+  const uint32_t rfree = rfull + 16;        // [2] sender: every owner has read its block
+  const uint32_t d_buffull = rfree + 16;    // [2]
   const uint32_t d_bufempty = d_buffull + 16;
   const uint32_t d_accfull = d_bufempty + 16;
   const uint32_t d_accfree = d_accfull + 16;
@@ -254,8 +250,10 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     mbar_init(c_accfull, 1);
     mbar_init(c_accfree, 1);
-    mbar_init(redfull, 1);   // the leader's expect_tx; the peers' bulk copies complete_tx
-    mbar_init(redfree, 1);
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(rfull + 8 * b, 1);     // the owner's expect_tx; the senders' bulk copies complete_tx
+      mbar_init(rfree + 8 * b, kCl);   // one arrival per owner
+    }
     for (int b = 0; b < 2; ++b) {
       mbar_init(d_buffull + 8 * b, 1);
       mbar_init(d_bufempty + 8 * b, 1);
@@ -396,20 +394,24 @@ __global__ void __launch_bounds__(kThreads, 1)
         cur_next(p, c, clu, sh);
       }
     } else if (warp < 4) {
-      // ---- partial sums -> the leader; the leader's 4 warps reduce them in
-      // rank order (deterministic) and run the epilogue.  Warp 0 reads the
-      // accumulator (TMEM lanes 0-31 = token rows) into this CTA's slot 0;
-      // a peer then bulk-copies slot 0 into the leader's slot `rank` over
-      // DSMEM, completing on the leader's redfull barrier (complete_tx).
+      // ---- reduce-scatter of the K-split partials, then the epilogue of this
+      // CTA's column slice.  Warp 0 reads the accumulator (TMEM lanes 0-15 =
+      // token rows) into the send buffer, one block per owner, and bulk-copies
+      // block o into owner o's receive slot [rank] over DSMEM (complete_tx on
+      // the owner's rfull).  Every CTA (4 warps) then sums the kCl senders'
+      // blocks of its cs columns in rank order (deterministic; the same order
+      // as a single reducer) and runs the epilogue on 16 x cs outputs: 1-2 per
+      // thread, so its latency is a fraction of one reducer's 16 per thread.
       Cur c = {-1, 0, false};
       OpShape sh = {};
       cur_next(p, c, clu, sh);
       int uses = 0, k = 0;
       const int M = p.M;
       const int et = threadIdx.x;                 // 0..127
-      const uint32_t part = sbase + PART_OFF;     // [8 slots][16 rows][PROW]
-      float *red_s = reinterpret_cast<float *>(smem + STG_OFF);   // [16 rows][128] dbpart staging
-      const int er = et >> 3, ec = (et & 7) * 16; // epilogue: row, first of 16 columns
+      const uint32_t sendb = sbase + SEND_OFF;
+      const uint32_t recvb = sbase + RECV_OFF;
+      float *red_s = reinterpret_cast<float *>(smem + STG_OFF);   // [16 rows][cs] dbpart staging
+      const int er = et >> 3;                     // epilogue: row, and 1-2 columns of the slice
       while (!c.done) {
         const int kb0 = kb_lo(sh.nkb, rank), kb1 = kb_lo(sh.nkb, rank + 1);
         const bool mine = kb1 > kb0;
@@ -417,211 +419,172 @@ __global__ void __launch_bounds__(kThreads, 1)
         const int i = sh.layer;
         const LayerDev &Ld = p.layers[i - 1];
         const int n0 = c.t * sh.tn;
+        const int cs = sh.tn / kCl;               // owned columns (8 or 16)
+        const int RS = cs + 4;
+        const int blk = kMaxM * RS * 4;
+        const int ncol = cs / 8;                  // per thread
+        const int ec = (et & 7) * ncol;           // within the slice
+        const int gc = n0 + (int)rank * cs + ec;  // global column
+        const int b = k & 1;
         // epilogue inputs that do not depend on the chain, requested first
-        uint4 pre[2] = {make_uint4(0, 0, 0, 0), make_uint4(0, 0, 0, 0)};
-        if (rank == 0 && ec < sh.tn) {
-          if (sh.kind == EPI_FWD) {
-            const uint4 *bp = reinterpret_cast<const uint4 *>(reinterpret_cast<const __nv_bfloat16 *>(Ld.bias) + n0 + ec);
-            pre[0] = __ldg(bp);
-            pre[1] = __ldg(bp + 1);
-          } else if (i >= 2 && p.layers[i - 2].act != ACT_ID && p.layers[i - 2].Z && er < M) {
-            const uint4 *zp = reinterpret_cast<const uint4 *>(
-                reinterpret_cast<const __nv_bfloat16 *>(p.layers[i - 2].Z) + (size_t)er * sh.N + n0 + ec);
-            pre[0] = __ldg(zp);
-            pre[1] = __ldg(zp + 1);
-          }
+        uint32_t pre = 0;
+        if (sh.kind == EPI_FWD) {
+          const __nv_bfloat16 *bp = reinterpret_cast<const __nv_bfloat16 *>(Ld.bias) + gc;
+          pre = ncol == 2 ? __ldg(reinterpret_cast<const uint32_t *>(bp))
+                          : (uint32_t)__bfloat16_as_ushort(bp[0]);
+        } else if (i >= 2 && p.layers[i - 2].act != ACT_ID && p.layers[i - 2].Z && er < M) {
+          const __nv_bfloat16 *zp = reinterpret_cast<const __nv_bfloat16 *>(p.layers[i - 2].Z) + (size_t)er * sh.N + gc;
+          pre = ncol == 2 ? __ldg(reinterpret_cast<const uint32_t *>(zp)) : (uint32_t)__bfloat16_as_ushort(zp[0]);
         }
-        if (warp == 0) {
-          if (rank != 0 && k > 0) wait_bar(redfree, (k - 1) & 1, true);   // slot 0's last copy was read
-          if (rank == 0 && et == 0) {
-            int contrib = 0;
-            for (int rr = 1; rr < kCl; ++rr) contrib += kb_lo(sh.nkb, rr + 1) > kb_lo(sh.nkb, rr);
-            mbar_expect_tx(redfull, (uint32_t)(contrib * kMaxM * PROW));
-            sktrace(c.j, c.t, 0);
-          }
-          if (mine) {
-            wait_bar(c_accfull, uses & 1, true);
-            fence_after();
-            if (rank == 0 && et == 0) sktrace(c.j, c.t, 1);
-            const uint32_t dst = part + lane * PROW;
-            for (int ch = 0; ch < nch; ch += 2) {
-              uint32_t r0[32], r1[32];
-              tmem_ld32_issue(tmem + (uint32_t)(ch * 32), r0);
-              tmem_ld32_issue(tmem + (uint32_t)((ch + 1) * 32), r1);
-              tmem_ld_wait(r0);
-              tmem_ld_wait(r1);
-              if (lane < kMaxM) {
-#pragma unroll
-                for (int j = 0; j < 8; ++j)
-                  asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst + ch * 128 + 16 * j),
-                               "r"(r0[4 * j]), "r"(r0[4 * j + 1]), "r"(r0[4 * j + 2]), "r"(r0[4 * j + 3])
-                               : "memory");
-#pragma unroll
-                for (int j = 0; j < 8; ++j)
-                  asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(dst + (ch + 1) * 128 + 16 * j),
-                               "r"(r1[4 * j]), "r"(r1[4 * j + 1]), "r"(r1[4 * j + 2]), "r"(r1[4 * j + 3])
-                               : "memory");
-              }
-            }
-            fence_before();
-            if (rank != 0) asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // slot 0 -> bulk copy
-            __syncwarp();
-            if (lane == 0) {
-              mbar_arrive(c_accfree);
-              if (rank != 0)
-                asm volatile(
-                    "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-                        mapa(part + rank * kMaxM * PROW, 0)),
-                    "r"(part), "r"(kMaxM * PROW), "r"(mapa(redfull, 0))
-                    : "memory");
-            }
-            ++uses;
-          }
+        int contrib = 0;
+        for (int rr = 0; rr < kCl; ++rr) contrib += kb_lo(sh.nkb, rr + 1) > kb_lo(sh.nkb, rr);
+        if (et == 0) {
+          mbar_expect_tx(rfull + 8 * b, (uint32_t)(contrib * blk));
+          if (rank == 0) sktrace(c.j, c.t, 0);
         }
-        if (rank == 0) {
-          // ---- leader: all peers' partials landed -> reduce + epilogue (4 warps)
-          wait_bar(redfull, k & 1, true);
-          asm volatile("bar.sync 1, 128;" ::: "memory");   // slot 0 (own partial) written by warp 0
-          if (et == 0) sktrace(c.j, c.t, 2);
-          const bool act_row = er < M && ec < sh.tn;
-          float v[16];
+        if (warp == 0 && mine) {
+          // send slot b free: every owner has read task k-2's blocks
+          if (k >= 2) wait_bar(rfree + 8 * b, ((k >> 1) - 1) & 1, true);
+          wait_bar(c_accfull, uses & 1, true);
+          fence_after();
+          if (rank == 0 && et == 0) sktrace(c.j, c.t, 1);
+          const uint32_t sb = sendb + b * kCl * BLK_MAX + lane * RS * 4;
+          for (int ch = 0; ch < nch; ch += 2) {
+            uint32_t r0[32], r1[32];
+            tmem_ld32_issue(tmem + (uint32_t)(ch * 32), r0);
+            tmem_ld32_issue(tmem + (uint32_t)((ch + 1) * 32), r1);
+            tmem_ld_wait(r0);
+            tmem_ld_wait(r1);
+            if (lane < kMaxM) {
 #pragma unroll
-          for (int q = 0; q < 16; ++q) v[q] = 0.f;
-          if (act_row) {
-            for (int rr = 0; rr < kCl; ++rr) {
-              if (kb_lo(sh.nkb, rr + 1) == kb_lo(sh.nkb, rr)) continue;   // that CTA had no k-blocks
-              const uint32_t src = part + (rr * kMaxM + er) * PROW + ec * 4;
-#pragma unroll
-              for (int j = 0; j < 4; ++j) {
-                float x, y, z, w;
-                asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
-                             : "=f"(x), "=f"(y), "=f"(z), "=f"(w)
-                             : "r"(src + 16 * j)
+              for (int q = 0; q < 16; ++q) {       // 4 columns per store, one owner each (cs % 4 == 0)
+                const int col = ch * 32 + 4 * q;
+                const uint32_t *rr = q < 8 ? &r0[4 * q] : &r1[4 * (q - 8)];
+                const int o = col / cs;
+                asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(sb + o * blk + (col - o * cs) * 4),
+                             "r"(rr[0]), "r"(rr[1]), "r"(rr[2]), "r"(rr[3])
                              : "memory");
-                v[4 * j] += x;
-                v[4 * j + 1] += y;
-                v[4 * j + 2] += z;
-                v[4 * j + 3] += w;
               }
             }
           }
-          const uint32_t pw[8] = {pre[0].x, pre[0].y, pre[0].z, pre[0].w, pre[1].x, pre[1].y, pre[1].z, pre[1].w};
-          const int col0 = n0 + ec;
-          const size_t off = (size_t)er * sh.N + col0;
-          bool publish_db = false;
-          if (sh.kind == EPI_FWD) {
-            uint32_t u[8];
-#pragma unroll
-            for (int q = 0; q < 8; ++q) {
-              v[2 * q] += bf_lo(pw[q]);
-              v[2 * q + 1] += bf_hi(pw[q]);
-              u[q] = pack_bf2(v[2 * q], v[2 * q + 1]);   // Z_i in bf16 (RNE)
-              v[2 * q] = bf_lo(u[q]);
-              v[2 * q + 1] = bf_hi(u[q]);
-            }
-            __nv_bfloat16 *out = reinterpret_cast<__nv_bfloat16 *>(i == cl.L ? p.y_out : Ld.Xn);
-            __nv_bfloat16 *zst = reinterpret_cast<__nv_bfloat16 *>(const_cast<void *>(Ld.Z));
-            uint32_t o[8], d[8];
-            if (Ld.act == ACT_ID) {
-#pragma unroll
-              for (int q = 0; q < 8; ++q) o[q] = u[q];
-            } else if (Ld.act == ACT_GELU) {
-              // X_{i+1} = gelu(Z_i); the Z_i store keeps gelu'(Z_i) for the backward
-#pragma unroll
-              for (int q = 0; q < 8; ++q) {
-                float g[2], gd[2];
-#pragma unroll
-                for (int h = 0; h < 2; ++h) {
-                  float Phi, ez;
-                  gauss_cdf_exp(v[2 * q + h], Phi, ez);
-                  gd[h] = fmaf(v[2 * q + h] * 0.39894228040143268f, ez, Phi);
-                  g[h] = v[2 * q + h] * Phi;
-                }
-                o[q] = pack_bf2(g[0], g[1]);
-                d[q] = pack_bf2(gd[0], gd[1]);
-              }
-            } else {
-#pragma unroll
-              for (int q = 0; q < 8; ++q) o[q] = pack_bf2(fmaxf(v[2 * q], 0.f), fmaxf(v[2 * q + 1], 0.f));
-            }
-            if (act_row) {
-              uint4 *op = reinterpret_cast<uint4 *>(out + off);
-              op[0] = make_uint4(o[0], o[1], o[2], o[3]);
-              op[1] = make_uint4(o[4], o[5], o[6], o[7]);
-              if (Ld.act == ACT_GELU) {
-                uint4 *zp = reinterpret_cast<uint4 *>(zst + off);
-                zp[0] = make_uint4(d[0], d[1], d[2], d[3]);
-                zp[1] = make_uint4(d[4], d[5], d[6], d[7]);
-              } else if (Ld.act == ACT_RELU) {
-                uint4 *zp = reinterpret_cast<uint4 *>(zst + off);   // ReLU: Z_i
-                zp[0] = make_uint4(u[0], u[1], u[2], u[3]);
-                zp[1] = make_uint4(u[4], u[5], u[6], u[7]);
-              }
-            }
-          } else {
-            // dO_i: dZ_{i-1} = (dZ_i W_i^T) * act'_{i-1}(Z_{i-1}) (GELU: the stored gelu')
-            __nv_bfloat16 *out = reinterpret_cast<__nv_bfloat16 *>(i >= 2 ? p.layers[i - 2].dZ : p.dx_out);
-            const int pact = i >= 2 ? p.layers[i - 2].act : ACT_ID;
-            if (pact != ACT_ID && p.layers[i - 2].Z) {
-#pragma unroll
-              for (int q = 0; q < 8; ++q) {
-                const float z0 = bf_lo(pw[q]), z1 = bf_hi(pw[q]);
-                if (pact == ACT_GELU) {
-                  v[2 * q] *= z0;
-                  v[2 * q + 1] *= z1;
-                } else {
-                  v[2 * q] = z0 > 0.f ? v[2 * q] : 0.f;
-                  v[2 * q + 1] = z1 > 0.f ? v[2 * q + 1] : 0.f;
-                }
-              }
-            }
-            uint32_t u[8];
-#pragma unroll
-            for (int q = 0; q < 8; ++q) u[q] = act_row ? pack_bf2(v[2 * q], v[2 * q + 1]) : 0u;   // dZ_{i-1} (RNE)
-            if (act_row && out) {
-              uint4 *op = reinterpret_cast<uint4 *>(out + off);
-              op[0] = make_uint4(u[0], u[1], u[2], u[3]);
-              op[1] = make_uint4(u[4], u[5], u[6], u[7]);
-            }
-            if (i >= 2 && p.layers[i - 2].dbpart) {
-              publish_db = true;
-              if (er < kMaxM && ec < sh.tn) {
-#pragma unroll
-                for (int q = 0; q < 8; ++q) {
-                  red_s[er * 128 + ec + 2 * q] = bf_lo(u[q]);
-                  red_s[er * 128 + ec + 2 * q + 1] = bf_hi(u[q]);
-                }
-              }
-            }
-          }
-          asm volatile("bar.sync 1, 128;" ::: "memory");   // partials read, outputs stored
-          if (et == 0) sktrace(c.j, c.t, 6);
-          if (publish_db && et < sh.tn) {
-            // bias-gradient partial of the only row block: column sums of the
-            // rounded dZ_{i-1} over the token rows, in row order
-            float sum = 0.f;
-            for (int r = 0; r < M; ++r) sum += red_s[r * 128 + et];
-            p.layers[i - 2].dbpart[n0 + et] = sum;
-          }
-          if (publish_db) asm volatile("bar.sync 1, 128;" ::: "memory");
-          if (et == 0) {
-            // publish the tile: cumulative over the 4 warps' stores (ordered by bar.sync)
-            asm volatile("fence.acq_rel.gpu;" ::: "memory");
-            sktrace(c.j, c.t, 7);
-            if (sh.kind == EPI_FWD) {
-              red_add(ctr + cl.fwd_rows + (i - 1) * cl.MT, 1);
-            } else if (i >= 2) {
-              red_add(ctr + cl.dz_rows + (i - 2) * cl.MT, 1);
-              red_add(ctr + cl.dz_total + (i - 2), 1);
-            } else {
-              red_add(ctr + cl.dx_total, 1);
-            }
-            sktrace(c.j, c.t, 3);
-          }
+          fence_before();
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // send blocks -> bulk copies
           __syncwarp();
-          // partials read: free the peers' slots (one lane per peer, in parallel;
-          // after the publish, which is what the chain waits for)
-          if (warp == 0 && lane >= 1 && lane < kCl) mbar_arrive_cluster(mapa(redfree, lane));
+          if (lane == 0) mbar_arrive(c_accfree);
+          if (lane < kCl) {                        // one lane per owner
+            const uint32_t src = sendb + b * kCl * BLK_MAX + lane * blk;
+            asm volatile(
+                "cp.async.bulk.shared::cluster.shared::cta.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                    mapa(recvb + (b * kCl + (int)rank) * BLK_MAX, lane)),
+                "r"(src), "r"(blk), "r"(mapa(rfull + 8 * b, lane))
+                : "memory");
+          }
+          ++uses;
+        }
+        // ---- owner: every sender's block of this CTA's columns landed
+        wait_bar(rfull + 8 * b, (k >> 1) & 1, true);
+        if (rank == 0 && et == 0) sktrace(c.j, c.t, 2);
+        const bool act_row = er < M;
+        float v[2] = {0.f, 0.f};
+        {
+          const uint32_t src0 = recvb + b * kCl * BLK_MAX + (er * RS + ec) * 4;
+          for (int rr = 0; rr < kCl; ++rr) {
+            if (kb_lo(sh.nkb, rr + 1) == kb_lo(sh.nkb, rr)) continue;   // that CTA had no k-blocks
+            float x, y = 0.f;
+            if (ncol == 2)
+              asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(x), "=f"(y) : "r"(src0 + rr * BLK_MAX) : "memory");
+            else
+              asm volatile("ld.shared.f32 %0, [%1];" : "=f"(x) : "r"(src0 + rr * BLK_MAX) : "memory");
+            v[0] += x;
+            v[1] += y;
+          }
+        }
+        asm volatile("bar.sync 1, 128;" ::: "memory");   // receive slot b read by all threads
+        if (warp == 0 && lane < kCl) mbar_arrive_cluster(mapa(rfree + 8 * b, lane));
+        const int off = er * sh.N + gc;
+        bool publish_db = false;
+        const float p0 = __uint_as_float(pre << 16), p1 = __uint_as_float(pre & 0xFFFF0000u);
+        if (sh.kind == EPI_FWD) {
+          // Z_i = acc + b_i in bf16 (RNE); X_{i+1} = act(Z_i)
+          const uint32_t u = pack_bf2(v[0] + p0, v[1] + p1);
+          const float z0 = bf_lo(u), z1 = bf_hi(u);
+          __nv_bfloat16 *out = reinterpret_cast<__nv_bfloat16 *>(i == cl.L ? p.y_out : Ld.Xn);
+          __nv_bfloat16 *zst = reinterpret_cast<__nv_bfloat16 *>(const_cast<void *>(Ld.Z));
+          uint32_t o = u, d = 0;
+          if (Ld.act == ACT_GELU) {
+            // X_{i+1} = gelu(Z_i); the Z_i store keeps gelu'(Z_i) for the backward
+            float g[2], gd[2];
+            const float zz[2] = {z0, z1};
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              float Phi, ez;
+              gauss_cdf_exp(zz[h], Phi, ez);
+              gd[h] = fmaf(zz[h] * 0.39894228040143268f, ez, Phi);
+              g[h] = zz[h] * Phi;
+            }
+            o = pack_bf2(g[0], g[1]);
+            d = pack_bf2(gd[0], gd[1]);
+          } else if (Ld.act == ACT_RELU) {
+            o = pack_bf2(fmaxf(z0, 0.f), fmaxf(z1, 0.f));
+            d = u;                                  // ReLU: Z_i
+          }
+          if (act_row) {
+            if (ncol == 2) {
+              *reinterpret_cast<uint32_t *>(out + off) = o;
+              if (Ld.act != ACT_ID) *reinterpret_cast<uint32_t *>(zst + off) = d;
+            } else {
+              out[off] = __ushort_as_bfloat16((unsigned short)(o & 0xFFFFu));
+              if (Ld.act != ACT_ID) zst[off] = __ushort_as_bfloat16((unsigned short)(d & 0xFFFFu));
+            }
+          }
+        } else {
+          // dO_i: dZ_{i-1} = (dZ_i W_i^T) * act'_{i-1}(Z_{i-1}) (GELU: the stored gelu')
+          __nv_bfloat16 *out = reinterpret_cast<__nv_bfloat16 *>(i >= 2 ? p.layers[i - 2].dZ : p.dx_out);
+          const int pact = i >= 2 ? p.layers[i - 2].act : ACT_ID;
+          if (pact != ACT_ID && p.layers[i - 2].Z) {
+            if (pact == ACT_GELU) {
+              v[0] *= p0;
+              v[1] *= p1;
+            } else {
+              v[0] = p0 > 0.f ? v[0] : 0.f;
+              v[1] = p1 > 0.f ? v[1] : 0.f;
+            }
+          }
+          const uint32_t u = act_row ? pack_bf2(v[0], v[1]) : 0u;   // dZ_{i-1} (RNE)
+          if (act_row && out) {
+            if (ncol == 2) *reinterpret_cast<uint32_t *>(out + off) = u;
+            else out[off] = __ushort_as_bfloat16((unsigned short)(u & 0xFFFFu));
+          }
+          if (i >= 2 && p.layers[i - 2].dbpart) {
+            publish_db = true;
+            red_s[er * 16 + ec] = bf_lo(u);
+            if (ncol == 2) red_s[er * 16 + ec + 1] = bf_hi(u);
+          }
+        }
+        asm volatile("bar.sync 1, 128;" ::: "memory");   // outputs stored
+        if (rank == 0 && et == 0) sktrace(c.j, c.t, 6);
+        if (publish_db && et < cs) {
+          // bias-gradient partial of the only row block: column sums of the
+          // rounded dZ_{i-1} over the token rows, in row order
+          float sum = 0.f;
+          for (int r = 0; r < M; ++r) sum += red_s[r * 16 + et];
+          p.layers[i - 2].dbpart[n0 + (int)rank * cs + et] = sum;
+        }
+        if (publish_db) asm volatile("bar.sync 1, 128;" ::: "memory");
+        if (et == 0) {
+          // publish this CTA's slice: cumulative over the 4 warps' stores
+          // (ordered by bar.sync); a tile completes with kCl slices
+          asm volatile("fence.acq_rel.gpu;" ::: "memory");
+          if (rank == 0) sktrace(c.j, c.t, 7);
+          if (sh.kind == EPI_FWD) {
+            red_add(ctr + cl.fwd_rows + (i - 1) * cl.MT, 1);
+          } else if (i >= 2) {
+            red_add(ctr + cl.dz_rows + (i - 2) * cl.MT, 1);
+            red_add(ctr + cl.dz_total + (i - 2), 1);
+          } else {
+            red_add(ctr + cl.dx_total, 1);
+          }
+          if (rank == 0) sktrace(c.j, c.t, 3);
         }
         ++k;
         cur_next(p, c, clu, sh);
@@ -666,7 +629,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         const LayerDev &L = p.layers[i - 1];
         const int b = g & 1;
         if (g >= 2) wait_bar(d_bufempty + 8 * b, ((g >> 1) - 1) & 1, false);
-        if (i < cl.L) wait_ge(ctr + cl.dz_total + (i - 1), cl.MT * p.layers[i].dx_nt);   // dZ_i complete
+        if (i < cl.L) wait_ge(ctr + cl.dz_total + (i - 1), cl.MT * p.layers[i].dx_nt * kPubPerTile);   // dZ_i complete
         asm volatile("fence.proxy.async.global;" ::: "memory");
         const uint32_t buf = sbase + b * DW_BUF;
         const int npb = L.dw_bn / 64;

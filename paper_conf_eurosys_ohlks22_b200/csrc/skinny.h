@@ -35,6 +35,10 @@ constexpr int kCl = 8;          // CTAs per cluster (the K split of one chain ti
 constexpr int kMaxM = 16;       // token rows of a skinny stack
 constexpr int kMaxChain = 800;  // chain ops per launch (2L + 1)
 constexpr int kMaxDw = 400;     // dW ops (+ the copy) per launch
+// Every CTA of a chain cluster publishes its column slice of a tile: the
+// fwd_rows / dz_rows / dz_total / dx_total counters of a skinny launch count
+// kPubPerTile per tile (the engine's count 1; targets scale with it).
+constexpr int kPubPerTile = kCl;
 
 struct ChainOp {
   int16_t kind;    // eng::EPI_FWD / EPI_DGRAD
