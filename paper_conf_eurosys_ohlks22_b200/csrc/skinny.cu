@@ -215,6 +215,154 @@ __device__ __forceinline__ bool input_ok(const Params &p, const OpShape &sh) {
   return reached(p.ctr + cl.dz_rows + (i - 1) * cl.MT, p.layers[i].dx_nt * kPubPerTile);
 }
 
+// dW workers: a dynamic queue of dW_i tiles in D's order
+// (Alg. 2) and the X -> X_1 copy; warps 0-3 epilogue, 4 dispenser +
+// producer, 5 MMA.  dw_base: 2 x DW_BUF operand buffers; stg_base: 4 x 2 KB
+// store staging; the barrier addresses are this CTA's.
+__device__ __forceinline__ void dw_worker(const Params &p, int warp, int lane, uint32_t tmem, uint32_t dw_base,
+                                          uint32_t stg_base, volatile int *task_slot, uint32_t d_buffull,
+                                          uint32_t d_bufempty, uint32_t d_accfull, uint32_t d_accfree,
+                                          uint32_t qfull, uint32_t qempty) {
+  const CounterLayout &cl = p.cl;
+  int32_t *ctr = p.ctr;
+  // ================================================================ dW workers
+  const int M = p.M;
+  const int ksteps = (M + 15) / 16;   // 16-deep MMA K steps over the tokens (TMA zero-fills rows >= M)
+  auto decode = [&](int t, int &op, int &rt, int &ct) {
+    int lo = 0, hi = p.ndw - 1;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (p.dw[mid].first <= t) lo = mid; else hi = mid - 1;
+    }
+    op = lo;
+    const int rel = t - p.dw[op].first;
+    if (p.dw[op].kind == EPI_COPY) {
+      rt = ct = 0;
+      return;
+    }
+    const LayerDev &L = p.layers[p.dw[op].layer - 1];
+    const int nt = (L.dout + L.dw_bn - 1) / L.dw_bn;   // the last tile may be ragged
+    rt = rel / nt;
+    ct = rel % nt;
+  };
+  if (warp == 4 && lane == 0) {
+    // ---- dispenser + producer
+    int g = 0;
+    for (int j = 0;; ++j) {
+      const int slot = j % Q;
+      if (j >= Q) wait_bar(qempty + 8 * slot, ((j / Q) - 1) & 1, false);
+      int t = atomicAdd(ctr + 1, 1);
+      if (t >= p.ntasks_dw) t = -1;
+      task_slot[slot] = t;
+      mbar_arrive(qfull + 8 * slot);
+      if (t < 0) break;
+      int op, rt, ct;
+      decode(t, op, rt, ct);
+      if (p.dw[op].kind == EPI_COPY) continue;
+      const int i = p.dw[op].layer;
+      const LayerDev &L = p.layers[i - 1];
+      const int b = g & 1;
+      if (g >= 2) wait_bar(d_bufempty + 8 * b, ((g >> 1) - 1) & 1, false);
+      if (i < cl.L) wait_ge(ctr + cl.dz_total + (i - 1), cl.MT * p.layers[i].dx_nt * kPubPerTile);   // dZ_i complete
+      asm volatile("fence.proxy.async.global;" ::: "memory");
+      const uint32_t buf = dw_base + b * DW_BUF;
+      const int npb = L.dw_bn / 64;
+      mbar_expect_tx(d_buffull + 8 * b, 2 * 2048 + npb * 2048);
+      const CUtensorMap *mX = p.maps + (size_t)(i - 1) * p.maps_per_layer + p.map_x;
+      const CUtensorMap *mD = p.maps + (size_t)(i - 1) * p.maps_per_layer + p.map_dz;
+      for (int c = 0; c < 2; ++c) tma_load_2d(buf + 2048 * c, mX, d_buffull + 8 * b, rt * 128 + 64 * c, 0);
+      for (int c = 0; c < npb; ++c) tma_load_2d(buf + 4096 + 2048 * c, mD, d_buffull + 8 * b, ct * L.dw_bn + 64 * c, 0);
+      ++g;
+    }
+  } else if (warp == 5 && lane == 0) {
+    // ---- MMA: dW tile = X_i^T (MN-major, 128 features) x dZ_i (MN-major), K = tokens
+    int g = 0;
+    for (int j = 0;; ++j) {
+      const int slot = j % Q;
+      wait_bar(qfull + 8 * slot, (j / Q) & 1, false);
+      const int t = task_slot[slot];
+      mbar_arrive(qempty + 8 * slot);
+      if (t < 0) break;
+      int op, rt, ct;
+      decode(t, op, rt, ct);
+      if (p.dw[op].kind == EPI_COPY) continue;
+      const LayerDev &L = p.layers[p.dw[op].layer - 1];
+      const int b = g & 1;
+      if (g >= 2) wait_bar(d_accfree + 8 * b, ((g >> 1) - 1) & 1, false);
+      wait_bar(d_buffull + 8 * b, (g >> 1) & 1, false);
+      fence_after();
+      const uint32_t buf = dw_base + b * DW_BUF;
+      const uint64_t ad = sdesc(buf, 2048, 1024), bd = sdesc(buf + 4096, 2048, 1024);
+      const uint32_t ID = idesc_rt(L.dw_bn, true, true);
+      for (int kk = 0; kk < ksteps; ++kk)
+        umma_bf16(tmem + (uint32_t)(b * 256), ad + 128u * kk, bd + 128u * kk, ID, kk > 0 ? 1u : 0u);
+      umma_commit(d_bufempty + 8 * b);
+      umma_commit(d_accfull + 8 * b);
+      ++g;
+    }
+  } else if (warp < 4) {
+    // ---- epilogue: scaled bf16 dW_i into the gradient bucket; db_i; the X -> X_1 copy
+    const int q = warp;
+    const int et = threadIdx.x;   // 0..127
+    const uint32_t stg = stg_base + q * 2048;
+    int g = 0;
+    for (int j = 0;; ++j) {
+      const int slot = j % Q;
+      wait_bar(qfull + 8 * slot, (j / Q) & 1, true);
+      const int t = task_slot[slot];
+      epi_bar();
+      if (et == 0) mbar_arrive(qempty + 8 * slot);
+      if (t < 0) break;
+      int op, rt, ct;
+      decode(t, op, rt, ct);
+      if (p.dw[op].kind == EPI_COPY) {
+        // caller's X -> X_1 store (the next backward's dW_1 input); the
+        // pending dW_1 still reads X_1: wait for it first
+        if (p.fwd_gate && et == 0) wait_ge(ctr + cl.dw_done, p.layers[0].dw_tiles);
+        epi_bar();
+        const int n = M * p.layers[0].din / 8;
+        const uint4 *src = reinterpret_cast<const uint4 *>(p.x_in);
+        uint4 *dst = reinterpret_cast<uint4 *>(p.layers[0].X);
+        for (int v = et; v < n; v += 128) dst[v] = __ldg(src + v);
+        continue;
+      }
+      const int i = p.dw[op].layer;
+      const LayerDev &L = p.layers[i - 1];
+      const int b = g & 1;
+      wait_bar(d_accfull + 8 * b, (g >> 1) & 1, true);
+      fence_after();
+      const uint32_t tb = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(b * 256);
+      __nv_bfloat16 *gw = reinterpret_cast<__nv_bfloat16 *>(L.gw);
+      const int cend = min(L.dw_bn, L.dout - ct * L.dw_bn) / 32;   // chunks inside dW_i's columns
+      for (int ch = 0; ch < cend; ++ch) {
+        uint32_t r[32];
+        tmem_ld32(tb + (uint32_t)(ch * 32), r);
+        float v[32];
+#pragma unroll
+        for (int x = 0; x < 32; ++x) v[x] = __uint_as_float(r[x]) * p.alpha;
+        store32_rows(gw, L.dout, stg, lane, v, ct * L.dw_bn + ch * 32, rt * 128 + q * 32, L.din);
+      }
+      fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(d_accfree + 8 * b);
+      if (rt == 0) {
+        // db_i = (1/N) x the bias-gradient partial of the only row block
+        __nv_bfloat16 *db = reinterpret_cast<__nv_bfloat16 *>(L.db_out);
+        for (int cc = et; cc < L.dw_bn; cc += 128) {
+          const int col = ct * L.dw_bn + cc;
+          if (col < L.dout) db[col] = __float2bfloat16_rn(__ldcg(L.dbpart + col) * p.alpha);
+        }
+      }
+      epi_bar();
+      if (et == 0) {
+        red_release_add(ctr + cl.dw_done + (i - 1), 1);
+        red_add(ctr + cl.bucket_done + L.bucket, 1);
+      }
+      ++g;
+    }
+  }
+}
+
 __global__ void __launch_bounds__(kThreads, 1)
     skinny_kernel(const __grid_constant__ CUtensorMap tmX, const __grid_constant__ Params p) {
   extern __shared__ uint8_t smem_raw[];
@@ -591,142 +739,8 @@ __global__ void __launch_bounds__(kThreads, 1)
       }
     }
   } else {
-    // ================================================================ dW workers
-    const int M = p.M;
-    const int ksteps = (M + 15) / 16;   // 16-deep MMA K steps over the tokens (TMA zero-fills rows >= M)
-    auto decode = [&](int t, int &op, int &rt, int &ct) {
-      int lo = 0, hi = p.ndw - 1;
-      while (lo < hi) {
-        const int mid = (lo + hi + 1) >> 1;
-        if (p.dw[mid].first <= t) lo = mid; else hi = mid - 1;
-      }
-      op = lo;
-      const int rel = t - p.dw[op].first;
-      if (p.dw[op].kind == EPI_COPY) {
-        rt = ct = 0;
-        return;
-      }
-      const LayerDev &L = p.layers[p.dw[op].layer - 1];
-      const int nt = (L.dout + L.dw_bn - 1) / L.dw_bn;   // the last tile may be ragged
-      rt = rel / nt;
-      ct = rel % nt;
-    };
-    if (warp == 4 && lane == 0) {
-      // ---- dispenser + producer
-      int g = 0;
-      for (int j = 0;; ++j) {
-        const int slot = j % Q;
-        if (j >= Q) wait_bar(qempty + 8 * slot, ((j / Q) - 1) & 1, false);
-        int t = atomicAdd(ctr + 1, 1);
-        if (t >= p.ntasks_dw) t = -1;
-        task_slot[slot] = t;
-        mbar_arrive(qfull + 8 * slot);
-        if (t < 0) break;
-        int op, rt, ct;
-        decode(t, op, rt, ct);
-        if (p.dw[op].kind == EPI_COPY) continue;
-        const int i = p.dw[op].layer;
-        const LayerDev &L = p.layers[i - 1];
-        const int b = g & 1;
-        if (g >= 2) wait_bar(d_bufempty + 8 * b, ((g >> 1) - 1) & 1, false);
-        if (i < cl.L) wait_ge(ctr + cl.dz_total + (i - 1), cl.MT * p.layers[i].dx_nt * kPubPerTile);   // dZ_i complete
-        asm volatile("fence.proxy.async.global;" ::: "memory");
-        const uint32_t buf = sbase + b * DW_BUF;
-        const int npb = L.dw_bn / 64;
-        mbar_expect_tx(d_buffull + 8 * b, 2 * 2048 + npb * 2048);
-        const CUtensorMap *mX = p.maps + (size_t)(i - 1) * p.maps_per_layer + p.map_x;
-        const CUtensorMap *mD = p.maps + (size_t)(i - 1) * p.maps_per_layer + p.map_dz;
-        for (int c = 0; c < 2; ++c) tma_load_2d(buf + 2048 * c, mX, d_buffull + 8 * b, rt * 128 + 64 * c, 0);
-        for (int c = 0; c < npb; ++c) tma_load_2d(buf + 4096 + 2048 * c, mD, d_buffull + 8 * b, ct * L.dw_bn + 64 * c, 0);
-        ++g;
-      }
-    } else if (warp == 5 && lane == 0) {
-      // ---- MMA: dW tile = X_i^T (MN-major, 128 features) x dZ_i (MN-major), K = tokens
-      int g = 0;
-      for (int j = 0;; ++j) {
-        const int slot = j % Q;
-        wait_bar(qfull + 8 * slot, (j / Q) & 1, false);
-        const int t = task_slot[slot];
-        mbar_arrive(qempty + 8 * slot);
-        if (t < 0) break;
-        int op, rt, ct;
-        decode(t, op, rt, ct);
-        if (p.dw[op].kind == EPI_COPY) continue;
-        const LayerDev &L = p.layers[p.dw[op].layer - 1];
-        const int b = g & 1;
-        if (g >= 2) wait_bar(d_accfree + 8 * b, ((g >> 1) - 1) & 1, false);
-        wait_bar(d_buffull + 8 * b, (g >> 1) & 1, false);
-        fence_after();
-        const uint32_t buf = sbase + b * DW_BUF;
-        const uint64_t ad = sdesc(buf, 2048, 1024), bd = sdesc(buf + 4096, 2048, 1024);
-        const uint32_t ID = idesc_rt(L.dw_bn, true, true);
-        for (int kk = 0; kk < ksteps; ++kk)
-          umma_bf16(tmem + (uint32_t)(b * 256), ad + 128u * kk, bd + 128u * kk, ID, kk > 0 ? 1u : 0u);
-        umma_commit(d_bufempty + 8 * b);
-        umma_commit(d_accfull + 8 * b);
-        ++g;
-      }
-    } else if (warp < 4) {
-      // ---- epilogue: scaled bf16 dW_i into the gradient bucket; db_i; the X -> X_1 copy
-      const int q = warp;
-      const int et = threadIdx.x;   // 0..127
-      const uint32_t stg = sbase + STG_OFF + q * 2048;
-      int g = 0;
-      for (int j = 0;; ++j) {
-        const int slot = j % Q;
-        wait_bar(qfull + 8 * slot, (j / Q) & 1, true);
-        const int t = task_slot[slot];
-        epi_bar();
-        if (et == 0) mbar_arrive(qempty + 8 * slot);
-        if (t < 0) break;
-        int op, rt, ct;
-        decode(t, op, rt, ct);
-        if (p.dw[op].kind == EPI_COPY) {
-          // caller's X -> X_1 store (the next backward's dW_1 input); the
-          // pending dW_1 still reads X_1: wait for it first
-          if (p.fwd_gate && et == 0) wait_ge(ctr + cl.dw_done, p.layers[0].dw_tiles);
-          epi_bar();
-          const int n = M * p.layers[0].din / 8;
-          const uint4 *src = reinterpret_cast<const uint4 *>(p.x_in);
-          uint4 *dst = reinterpret_cast<uint4 *>(p.layers[0].X);
-          for (int v = et; v < n; v += 128) dst[v] = __ldg(src + v);
-          continue;
-        }
-        const int i = p.dw[op].layer;
-        const LayerDev &L = p.layers[i - 1];
-        const int b = g & 1;
-        wait_bar(d_accfull + 8 * b, (g >> 1) & 1, true);
-        fence_after();
-        const uint32_t tb = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(b * 256);
-        __nv_bfloat16 *gw = reinterpret_cast<__nv_bfloat16 *>(L.gw);
-        const int cend = min(L.dw_bn, L.dout - ct * L.dw_bn) / 32;   // chunks inside dW_i's columns
-        for (int ch = 0; ch < cend; ++ch) {
-          uint32_t r[32];
-          tmem_ld32(tb + (uint32_t)(ch * 32), r);
-          float v[32];
-#pragma unroll
-          for (int x = 0; x < 32; ++x) v[x] = __uint_as_float(r[x]) * p.alpha;
-          store32_rows(gw, L.dout, stg, lane, v, ct * L.dw_bn + ch * 32, rt * 128 + q * 32, L.din);
-        }
-        fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(d_accfree + 8 * b);
-        if (rt == 0) {
-          // db_i = (1/N) x the bias-gradient partial of the only row block
-          __nv_bfloat16 *db = reinterpret_cast<__nv_bfloat16 *>(L.db_out);
-          for (int cc = et; cc < L.dw_bn; cc += 128) {
-            const int col = ct * L.dw_bn + cc;
-            if (col < L.dout) db[col] = __float2bfloat16_rn(__ldcg(L.dbpart + col) * p.alpha);
-          }
-        }
-        epi_bar();
-        if (et == 0) {
-          red_release_add(ctr + cl.dw_done + (i - 1), 1);
-          red_add(ctr + cl.bucket_done + L.bucket, 1);
-        }
-        ++g;
-      }
-    }
+    dw_worker(p, warp, lane, tmem, sbase, sbase + STG_OFF, task_slot, d_buffull, d_bufempty, d_accfull,
+              d_accfree, qfull, qempty);
   }
 
   fence_before();
@@ -737,6 +751,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(TMEM_COLS) : "memory");
   }
 }
+
 
 int g_max_clusters = 0;
 
