@@ -170,8 +170,32 @@ __device__ __forceinline__ uint32_t mapa(uint32_t addr, uint32_t rank) {
 __device__ __forceinline__ void cluster_sync() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
+// Release arrive on a peer CTA's barrier: publishes this thread's prior
+// writes at cluster scope -- compiled to MEMBAR.ALL.GPU, which waits for every
+// global store the thread has in flight (~1 us after an epilogue's stores).
+// Only for arrivals that publish data (the leader's task-slot write).
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+// Relaxed arrive (a bare SYNCS.ARRIVE): for the peer's "slot read" and
+// "accumulator read" signals, which publish no memory -- the slot reads are
+// performed before it (CTA barrier), the TMEM reads completed (tcgen05.wait::ld
+// + fence::before_thread_sync).  OOO_RELAXED_ARRIVE=0: release arrives (A/B).
+#ifndef OOO_RELAXED_ARRIVE
+#define OOO_RELAXED_ARRIVE 1
+#endif
+__device__ __forceinline__ void mbar_arrive_cluster_signal(uint32_t cluster_addr) {
+  if (OOO_RELAXED_ARRIVE)
+    asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+  else
+    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+// Acquire of shared::cluster data (a peer's st.shared::cluster into this CTA's
+// smem, released by its arrive): no instruction on sm_100a, where
+// fence.acq_rel.cluster is MEMBAR.ALL.GPU + CCTL.IVALL.
+__device__ __forceinline__ void acquire_cluster_smem() {
+  if (OOO_RELAXED_ARRIVE) asm volatile("fence.acquire.sync_restrict::shared::cluster.cluster;" ::: "memory");
+  else asm volatile("fence.acq_rel.cluster;" ::: "memory");
 }
 __device__ __forceinline__ void st_cluster_u32(uint32_t cluster_addr, int v) {
   asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(cluster_addr), "r"(v) : "memory");
@@ -206,11 +230,11 @@ __device__ __forceinline__ void mbar_wait_sleep(uint32_t bar, uint32_t parity) {
     }
   }
 }
-// For barriers that receive arrivals from the peer CTA (release.cluster):
-// one cluster-scope acquire fence after the wait, not one per poll.
+// For barriers that receive arrivals from the peer CTA: one acquire of the
+// shared::cluster data after the wait, not one per poll.
 __device__ __forceinline__ void mbar_wait_cl(uint32_t bar, uint32_t parity) {
   mbar_wait_b(bar, parity);
-  asm volatile("fence.acq_rel.cluster;" ::: "memory");
+  acquire_cluster_smem();
 }
 __device__ __forceinline__ void tma_load_2d_pair(uint32_t dst, const CUtensorMap *map, uint32_t leader_bar,
                                                  int c0, int c1) {
@@ -607,7 +631,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         } else {
           mbar_wait_cl(bar_qfull + 8 * slot, (j / Q) & 1);
           t = task_slot[slot];
-          mbar_arrive_cluster(L_qempty + 8 * slot);
+          mbar_arrive_cluster_signal(L_qempty + 8 * slot);
         }
         if (t < 0) break;
         const TaskRt T = task_rt<CG>(p, t);
@@ -759,12 +783,12 @@ __global__ void __launch_bounds__(kThreads, 1)
     for (int j = 0, ja = 0;; ++j) {
       const int slot = j % Q;
       mbar_wait_sleep(bar_qfull + 8 * slot, (j / Q) & 1);
-      if (!leader) asm volatile("fence.acq_rel.cluster;" ::: "memory");
+      if (!leader) acquire_cluster_smem();   // the leader's st.shared::cluster of the slot
       const int t = task_slot[slot];
       ebar();                                   // everyone read the slot; previous task done with smem
       if (et == 0) {
         if (leader) mbar_arrive(bar_qempty + 8 * slot);
-        else mbar_arrive_cluster(L_qempty + 8 * slot);
+        else mbar_arrive_cluster_signal(L_qempty + 8 * slot);
       }
       if (t < 0) break;
       const TaskRt T = task_rt<CG>(p, t);
@@ -876,7 +900,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         __syncwarp();
         if (lane == 0) {
           if (leader) mbar_arrive(bar_tempty + 8 * acc);
-          else mbar_arrive_cluster(L_tempty + 8 * acc);
+          else mbar_arrive_cluster_signal(L_tempty + 8 * acc);
         }
         ebar();                                  // all partial stores of this CTA precede the arrival
         if (tr2) etrace2(t, 6);
@@ -1014,7 +1038,7 @@ __global__ void __launch_bounds__(kThreads, 1)
         __syncwarp();
         if (lane == 0) {
           if (leader) mbar_arrive(bar_tempty + 8 * acc);
-          else mbar_arrive_cluster(L_tempty + 8 * acc);
+          else mbar_arrive_cluster_signal(L_tempty + 8 * acc);
         }
       }
       if (T.kind == EPI_DGRAD && dbpart && mblk < cl.MT) {

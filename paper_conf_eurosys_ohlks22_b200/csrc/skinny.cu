@@ -84,8 +84,12 @@ __device__ __forceinline__ uint32_t mapa(uint32_t addr, uint32_t rank) {
 __device__ __forceinline__ void cluster_sync() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
+// Relaxed arrive on a peer's barrier (a bare SYNCS.ARRIVE; the release form
+// is a MEMBAR.ALL.GPU that waits for this thread's global stores in flight):
+// the receive-slot "free" signal publishes no memory -- the slot's reads are
+// performed before it (CTA barrier).
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
-  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+  asm volatile("mbarrier.arrive.relaxed.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
 }
 // non-blocking phase test (try_wait may suspend the thread for a while: the
 // producer's loop polls two cursors and must not stall on either)
@@ -647,8 +651,6 @@ __global__ void __launch_bounds__(kThreads, 1)
             v[1] += y;
           }
         }
-        asm volatile("bar.sync 1, 128;" ::: "memory");   // receive slot b read by all threads
-        if (warp == 0 && lane < kCl) mbar_arrive_cluster(mapa(rfree + 8 * b, lane));
         const int off = er * sh.N + gc;
         bool publish_db = false;
         const float p0 = __uint_as_float(pre << 16), p1 = __uint_as_float(pre & 0xFFFF0000u);
@@ -734,6 +736,11 @@ __global__ void __launch_bounds__(kThreads, 1)
           }
           if (rank == 0) sktrace(c.j, c.t, 3);
         }
+        // receive slot b read by every thread (the barriers above): free it
+        // in every sender -- after the publish, which is what the chain waits
+        // for (a cluster-scope release arrive costs ~1 us on the critical path)
+        __syncwarp();
+        if (warp == 0 && lane < kCl) mbar_arrive_cluster(mapa(rfree + 8 * b, lane));
         ++k;
         cur_next(p, c, clu, sh);
       }
