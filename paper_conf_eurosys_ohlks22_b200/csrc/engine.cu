@@ -780,6 +780,17 @@ __global__ void __launch_bounds__(kThreads, 1)
     const int h = (warp - 2) >> 2;           // column slot: 32-col chunks c = h, h + kEpiPerQ, ...
     const int et = threadIdx.x - 64;         // 0..255
     const uint32_t stg = sbase + C::STG_OFF + (warp - 2) * 2048;
+    // epilogue thread 0, after a barrier that orders every epilogue store of
+    // the publication: +1 on counters a, b, c (indices; -1 none).  One release
+    // fence (a MEMBAR.ALL.GPU: it waits for the stores in flight) for all of
+    // them, then relaxed increments -- a red.release per counter would pay
+    // the MEMBAR once per counter (dW tiles publish two)
+    auto publish = [&](int a, int b, int c) {
+      asm volatile("fence.acq_rel.gpu;" ::: "memory");
+      if (a >= 0) asm volatile("red.relaxed.gpu.global.add.s32 [%0], 1;" ::"l"(ctr + a) : "memory");
+      if (b >= 0) asm volatile("red.relaxed.gpu.global.add.s32 [%0], 1;" ::"l"(ctr + b) : "memory");
+      if (c >= 0) asm volatile("red.relaxed.gpu.global.add.s32 [%0], 1;" ::"l"(ctr + c) : "memory");
+    };
     for (int j = 0, ja = 0;; ++j) {
       const int slot = j % Q;
       mbar_wait_sleep(bar_qfull + 8 * slot, (j / Q) & 1);
@@ -1001,9 +1012,9 @@ __global__ void __launch_bounds__(kThreads, 1)
       if (T.kind != EPI_WGRAD) {
         ebar();
         if (et == 0 && mrow0 < T.M) {
-          if (T.kind == EPI_FWD) red_release_add(ctr + cl.fwd_rows + (T.layer - 1) * cl.MT + mblk, 1);
-          else if (T.layer >= 2) red_release_add(ctr + cl.dz_rows + (T.layer - 2) * cl.MT + mblk, 1);
-          else red_release_add(ctr + cl.dx_total, 1);   // dX (the input gradient a previous stage waits for)
+          if (T.kind == EPI_FWD) publish(cl.fwd_rows + (T.layer - 1) * cl.MT + mblk, -1, -1);
+          else if (T.layer >= 2) publish(cl.dz_rows + (T.layer - 2) * cl.MT + mblk, -1, -1);
+          else publish(cl.dx_total, -1, -1);   // dX (the input gradient a previous stage waits for)
           if (leader) etrace(t, 3);
         }
       }
@@ -1074,10 +1085,9 @@ __global__ void __launch_bounds__(kThreads, 1)
         // (F_i: nothing left to publish -- its Z_i store is ordered before the
         // next backward by the launch boundary)
         if (T.kind == EPI_DGRAD) {
-          if (T.layer >= 2) red_release_add(ctr + cl.dz_total + (T.layer - 2), 1);   // + the db partials
+          if (T.layer >= 2) publish(cl.dz_total + (T.layer - 2), -1, -1);   // + the db partials
         } else if (T.kind == EPI_WGRAD) {
-          red_release_add(ctr + cl.dw_done + (T.layer - 1), 1);
-          red_release_add(ctr + cl.bucket_done + Ld.bucket, 1);
+          publish(cl.dw_done + (T.layer - 1), cl.bucket_done + Ld.bucket, -1);
           if (leader) etrace(t, 3);
         }
       }
