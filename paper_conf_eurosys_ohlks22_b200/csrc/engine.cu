@@ -170,13 +170,6 @@ __device__ __forceinline__ uint32_t mapa(uint32_t addr, uint32_t rank) {
 __device__ __forceinline__ void cluster_sync() {
   asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
 }
-// Release arrive on a peer CTA's barrier: publishes this thread's prior
-// writes at cluster scope -- compiled to MEMBAR.ALL.GPU, which waits for every
-// global store the thread has in flight (~1 us after an epilogue's stores).
-// Only for arrivals that publish data (the leader's task-slot write).
-__device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
-  asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
-}
 // Relaxed arrive (a bare SYNCS.ARRIVE): for the peer's "slot read" and
 // "accumulator read" signals, which publish no memory -- the slot reads are
 // performed before it (CTA barrier), the TMEM reads completed (tcgen05.wait::ld
@@ -196,9 +189,6 @@ __device__ __forceinline__ void mbar_arrive_cluster_signal(uint32_t cluster_addr
 __device__ __forceinline__ void acquire_cluster_smem() {
   if (OOO_RELAXED_ARRIVE) asm volatile("fence.acquire.sync_restrict::shared::cluster.cluster;" ::: "memory");
   else asm volatile("fence.acq_rel.cluster;" ::: "memory");
-}
-__device__ __forceinline__ void st_cluster_u32(uint32_t cluster_addr, int v) {
-  asm volatile("st.shared::cluster.u32 [%0], %1;" ::"r"(cluster_addr), "r"(v) : "memory");
 }
 // Bounded mbarrier wait with the default (CTA-scope) semantics.  Spinning
 // with .acquire.cluster would emit an L1 invalidation (CCTL.IVALL) on every
@@ -574,8 +564,9 @@ __global__ void __launch_bounds__(kThreads, 1)
       mbar_init(bar_tempty + 8 * a, CG * kEpiWarps);   // epilogue warps of all CTAs (leader's copy)
     }
     for (int s = 0; s < Q; ++s) {
-      mbar_init(bar_qfull + 8 * s, 1);          // leader's producer
+      mbar_init(bar_qfull + 8 * s, 1);          // leader: its producer; peer: its own arm (+ the leader's st.async bytes)
       mbar_init(bar_qempty + 8 * s, 2 * CG);    // MMA + epi (+ peer producer + peer epi)
+      if (CG == 2 && rank != 0) mbar_expect_tx(bar_qfull + 8 * s, 4);   // phase 0 armed
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -625,12 +616,18 @@ __global__ void __launch_bounds__(kThreads, 1)
           task_slot[slot] = t;
           mbar_arrive(bar_qfull + 8 * slot);
           if (CG == 2) {
-            st_cluster_u32(P_slot + 4 * slot, t);
-            mbar_arrive_cluster(P_qfull + 8 * slot);
+            // the peer's copy of the slot: a remote store that completes 4
+            // transaction bytes on the peer's full barrier (armed by the peer)
+            // -- no release fence (MEMBAR.ALL.GPU) on the dispenser's path
+            asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b32 [%0], %1, [%2];" ::"r"(
+                             P_slot + 4 * slot),
+                         "r"(t), "r"(P_qfull + 8 * slot)
+                         : "memory");
           }
         } else {
           mbar_wait_cl(bar_qfull + 8 * slot, (j / Q) & 1);
           t = task_slot[slot];
+          if (t >= 0) mbar_expect_tx(bar_qfull + 8 * slot, 4);   // arm the slot's next phase
           mbar_arrive_cluster_signal(L_qempty + 8 * slot);
         }
         if (t < 0) break;
