@@ -255,7 +255,8 @@ Plan make_plan(const ooo_stack_desc *d) {
         lp.ebn_fwd = lp.dout % 128 == 0 ? 128 : 64;
         lp.ebn_dx = lp.din % 128 == 0 ? 128 : 64;
       }
-    // split-K chain ops when all tokens fit one 128-row tile (C5: 16 tokens):
+    // split-K chain ops when all tokens fit one 128-row tile (C5 through the
+    // engine, OOO_SKINNY=0 / > 16 tokens):
     // a chain op's latency is its k-blocks at the MMA issue rate, whatever its
     // width (profiles/r02_mainloop_issue.md), so its K is spread over up to 8
     // workers while the split tiles still fit them (>= 4 k-blocks each: C5
@@ -267,8 +268,14 @@ Plan make_plan(const ooo_stack_desc *d) {
     // holds).  OOO_SPLITK=0: off; OOO_SPLITK_MAX / OOO_SPLITK_MINKB: tuning.
     int nsk = 0, maxw = 0;
     for (int i = 0; i <= p.L; ++i) maxw = std::max(maxw, d->dims[i]);
+    // with more rows, only the long-K chain ops split (>= longk k-blocks: C4's
+    // K = 4096 ops, 8 tiles x 64 k-blocks = 28 us each on the chain): C4
+    // 2.82 -> 2.72 ms; the split epilogue (~10 us: its fp32 partial round
+    // trips through L2) loses on shorter K.  OOO_SPLITK_LONGK=0: off
+    const int longk = env_int("OOO_SPLITK_LONGK", 64);
     auto ksplit = [&](int N, int bn, int K, bool allowed) {
-      if (!allowed || p.M > 128 || p.skinny || env_int("OOO_SPLITK", 1) == 0) return 1;
+      if (!allowed || p.skinny || env_int("OOO_SPLITK", 1) == 0) return 1;
+      if (p.M > 128 && (longk <= 0 || (K + 63) / 64 < longk)) return 1;
       const int tiles = PT * ((N + bn - 1) / bn);
       const int minkb = std::max(1, env_int("OOO_SPLITK_MINKB", 4));
       const int ks = std::min({std::min(8, env_int("OOO_SPLITK_MAX", 8)), ((K + 63) / 64) / minkb, workers / tiles});

@@ -112,6 +112,24 @@ def test_bf16_full_size_block_slice(cfg):
     assert torch.equal(out["raw"], base["raw"])
 
 
+def test_bf16_long_k_split_many_rows():
+    """Long-K chain ops split over K with more than one 128-row block
+    (OOO_SPLITK_LONGK, default 64 k-blocks: F_2 and dO_1 have K = 4096),
+    ragged rows (264 tokens): within the oracle's gate, every schedule
+    bit-exact, graph == eager."""
+    case = Case([256, 4096, 256], ["gelu", "id"], 264, "bf16", need_dx=True)
+    stk = case.stack()
+    base = case.run(stk, "in_order", 0)
+    _check(max_err(base, case.oracle(0)), BF16_TOL)
+    for k in (1, 2, 3):
+        out = case.run(stk, "first_k", k)
+        assert torch.equal(out["raw"], base["raw"]), k
+        assert np.array_equal(out["dX"], base["dX"])
+    g = case.run(stk, "first_k", 2, graph=True, launches=2)
+    assert torch.equal(g["raw"], base["raw"])
+    stk.close()
+
+
 def test_bf16_mlp96_full_config():
     """Config 4 at full size (96 layers, M = 16).  End-to-end bf16 error of a
     96-layer stack is bounded by the rounding random walk:
