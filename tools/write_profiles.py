@@ -24,8 +24,8 @@ def kernels(rnd, d):
              "", "## Product path: the fused engine step (Algorithm 1 regions) + the seed kernel (BK4)", ""]
     lines += table(os.path.join(d, "engine_kernels.csv"))
     lines += ["", "The engine runs the whole step (all F / dO / dW tiles with fused epilogues; the bucket pack/scale BK5 "
-              "is fused into the dW epilogue): tensor pipe active ≈ 47 % of its elapsed cycles -- the chain-latency bound "
-              f"of `r{rnd}_chain_latency.md`; it is not HBM-bound (≈ 21 % of DRAM peak).  The seed (dZ_L = dY ⊙ act'(Z_L) "
+              "is fused into the dW epilogue): tensor pipe active as in the table -- the chain-latency bound "
+              f"of DESIGN.md §10; it is not HBM-bound (DRAM % of peak in the table).  The seed (dZ_L = dY ⊙ act'(Z_L) "
               "+ db partials) is latency-bound at ≈ 1.2 TB/s (≈ 12 µs, 0.5 % of the step).  (Round 1 also "
               "measured a per-layer multi-stream path, one GEMM kernel per op at 13-31 % tensor-pipe: deleted in "
               "round 2.)"]
