@@ -1,6 +1,7 @@
 """Small workload for compute-sanitizer (memcheck / racecheck / synccheck /
-initcheck): the bf16 engine eager (forward, backward + join), the captured
-fused step, the comm-gated step (OOO_TEST_COMM_GATE) and the one-rank NCCL
+initcheck): the bf16 engine (CTA pairs; 1-CTA tiles with split-K; pairs with
+a long-K split) and the skinny cluster kernel, eager (forward, backward +
+join) and the captured fused step, the comm-gated step (OOO_TEST_COMM_GATE) and the one-rank NCCL
 data plane, plus the fp32 per-layer path.  Engine waits are bounded at
 10 min (the sanitizer slows the spin-waiting CTAs by orders of magnitude).
 
@@ -48,7 +49,11 @@ def run(dims, acts, M, dtype, label, **kw):
 
 dims, acts = [256, 512, 256, 256, 512], ["gelu", "id", "relu", "id"]
 run(dims, acts, 264, "bf16", "engine pairs (M=264)")
-run(dims, acts, 16, "bf16", "engine 1-CTA tiles (M=16)")
+run(dims, acts, 16, "bf16", "skinny cluster kernel (M=16)")
+os.environ["OOO_SKINNY"] = "0"
+run(dims, acts, 16, "bf16", "engine 1-CTA tiles, split-K (M=16)")
+del os.environ["OOO_SKINNY"]
+run([256, 4096, 256], ["gelu", "id"], 264, "bf16", "engine pairs, long-K split (M=264)")
 os.environ["OOO_TEST_COMM_GATE"] = "1"
 run(dims, acts, 264, "bf16", "comm-gated fused step")
 del os.environ["OOO_TEST_COMM_GATE"]
