@@ -390,11 +390,19 @@ def main():
         from paper_conf_eurosys_ohlks22_b200.ksearch import search_k
         probe = max(5, min(20, args.steps // 2))
 
+        g_ref = graph_for("first_k", 0)
+
         def tput(k):
+            # throughput relative to first_k(0), the two timed interleaved
+            # (ABAB): clock / power drift over the search cancels in the ratio
+            # (timing each candidate alone favoured whichever ran first)
             g = graph_for("first_k", k)
             for _ in range(2):
                 g.launch(stream)
-            return 1e3 / interleaved([g], probe, 1)[0][0]
+            if k == 0:
+                return 1.0
+            a, r = interleaved([g, g_ref], probe, 2)
+            return (sum(r) / len(r)) / (sum(a) / len(a))
         k_best, visited = search_k(L, tput)
     else:
         k_best, visited = int(args.k), []
