@@ -1,6 +1,6 @@
 """A/B of library knobs (environment variables read at stack creation /
 graph capture) on one box, all graphs timed in interleaved runs:
-    python tools/ab_env.py C2 "" "OOO_CHAIN192=0" [...]
+    python tools/ab_env.py C4 "" "OOO_SPLITK_LONGK=0" "OOO_EBN=128" [...]
 Prints ms per step of first_k(0) and in_order for each variant.  A tuning
 aid, not part of the product path."""
 import json

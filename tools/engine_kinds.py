@@ -6,7 +6,6 @@ import sys
 
 ROOT = __file__.rsplit("/tools/", 1)[0]
 os.environ.setdefault("OOO_LIB", os.path.join(ROOT, "paper_conf_eurosys_ohlks22_b200", "lib", "libooo_trace.so"))
-os.environ["OOO_GROUPS"] = "1"
 sys.path.insert(0, ROOT)
 import ctypes  # noqa: E402
 
